@@ -1,0 +1,225 @@
+"""Pins for the oracle scheduler (oracle/scheduler.py) -- CPU only.
+
+Pinned against: hand-worked values of Eq.3 + threshold (L165)
+and Eq.4 (L181), the hand-worked trace
+W1 (tests/golden/w1_trace.txt), the hand-built C0 / C0b streams whose slots
+follow from the closed form slot = bt[pos//16]*16 + pos%16, and invariants.
+"""
+import os
+
+import numpy as np
+import pytest
+
+from oracle.scheduler import Scheduler, run, throttle_decode, throttle_prefill
+from workloads.configs import SCHED, SchedParams
+from workloads.streams import Request, Stream, make_stream
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+DEF = SchedParams(num_blocks=1000)   # #T=8, MaxP=2048, MinP=32, thresh=1/20 (L248)
+
+
+@pytest.mark.parametrize("wp,free,expect", [
+    (10000, 1000, 1250),   # E1: WP/T = 1250 < cap 2048
+    (10000, 500, 970),     # E2: cap = floor(2048*9000/19000)
+    (100, 1000, 32),       # E3: floor(12.5) -> MinP
+    (20, 1000, 20),        # E4: MinP capped by WP (R11)
+    (10000, 49, 0),        # E5: KV_free 0.049 < 0.05 -> suspended (L165)
+    (10000, 50, 32),       # E6: equality uses Eq.3 (L167 ">="): cap 0 -> MinP
+    (0, 1000, 0),          # E7: nothing waiting
+    (20000, 1000, 2048),   # E8: MaxP
+    (3000, 300, 375),      # E9: cap 538 > 375
+])
+def test_eq3_examples(wp, free, expect):
+    assert throttle_prefill(DEF, wp, free) == expect
+
+
+def test_eq3_matches_exact_rational_floor():
+    # floor is monotone, so the integer reading equals floor(Eq.3) evaluated in exact rationals.
+    from fractions import Fraction as F
+    rng = np.random.default_rng(0)
+    for _ in range(2000):
+        n = int(rng.integers(1, 5000))
+        cfg = SchedParams(iterp=int(rng.integers(1, 17)), maxp=int(rng.integers(1, 4096)),
+                          minp=int(rng.integers(0, 64)), kvthresh_num=int(rng.integers(0, 5)),
+                          kvthresh_den=int(rng.integers(5, 40)), num_blocks=n)
+        wp = int(rng.integers(0, 50000))
+        free = int(rng.integers(0, n + 1))
+        kvf, th = F(free, n), F(cfg.kvthresh_num, cfg.kvthresh_den)
+        if wp == 0 or kvf < th:
+            ref = 0
+        else:
+            eq3 = max(min(F(wp, cfg.iterp), cfg.maxp * (kvf - th) / (1 - th)), cfg.minp)
+            ref = min(int(eq3), wp)      # int() == floor for non-negative rationals
+        assert throttle_prefill(cfg, wp, free) == ref
+
+
+def test_eq1_eq2_special_cases():
+    # thresh = 0 and KV fully free: Eq.3 reduces to Eq.1 (WT only)
+    cfg = SchedParams(kvthresh_num=0, kvthresh_den=20, num_blocks=100)
+    for wp in [1, 31, 32, 33, 255, 256, 1000, 16384, 16385, 99999]:
+        eq1 = min(max(wp // 8, 32), 2048)
+        assert throttle_prefill(cfg, wp, 100) == min(eq1, wp)
+    # WP huge: Eq.3 reduces to Eq.2 with KV_free rescaled over the threshold
+    for free in [0, 1, 5, 50, 99, 100]:
+        eq2 = max((2048 * free) // 100, 32)
+        assert throttle_prefill(cfg, 10 ** 9, free) == (eq2 if free > 0 else 32)
+
+
+def test_eq4_examples():
+    c4 = SchedParams(pp_depth=4)
+    assert throttle_decode(c4, 1000) == 250
+    assert throttle_decode(c4, 10) == 3          # ceil (R6)
+    assert throttle_decode(c4, 0) == 0
+    assert throttle_decode(SchedParams(pp_depth=1), 7) == 7
+
+
+def test_eq4_steady_pattern_and_ready_cap():
+    # RD=10 at PP=4, decode-only, long outputs: per-tick decode counts 3,3,3,1 repeating (Fig.8)
+    cfg = SchedParams(pp_depth=4, num_blocks=4096, iterp=1, maxp=4096, minp=1)
+    reqs = [Request(i, 0, 16, 1000, np.zeros(16 + 999, np.int32)) for i in range(10)]
+    s = Scheduler(cfg, reqs)
+    counts = [len(s.build_batch().decodes) for _ in range(24)]
+    steady = counts[8:20]
+    assert steady == [3, 3, 3, 1] * 3, counts
+    # RD=10 but only 2 ready -> 2 (L183 "schedule all of them")
+    cfg2 = SchedParams(pp_depth=4, num_blocks=4096)
+    s2 = Scheduler(cfg2)
+    for i in range(10):
+        s2.admitted.append(_warm_req(s2, i))
+    for r in s2.admitted[2:]:
+        r.inflight = 1
+    assert len(s2.build_batch(auto_retire=False).decodes) == 2
+
+
+def _warm_req(s, i):
+    from oracle.scheduler import _Req
+    r = _Req(i, 0, 20, 50, np.zeros(80, np.int32))
+    r.prefill_len = r.sched_prompt = r.done_prompt = 20
+    r.gen = 1
+    s._alloc(r, [])
+    s._alloc(r, [])
+    return r
+
+
+def _parse_w1():
+    rows = []
+    with open(os.path.join(GOLDEN, "w1_trace.txt")) as f:
+        for line in f:
+            if line.startswith("#") or not line.strip():
+                continue
+            tick, pd, ch, dec, slots, free = [x.strip() for x in line.split("|")]
+            P, D = map(int, pd.split())
+            chunks = [] if ch == "-" else [tuple(map(int, c.split(":"))) for c in ch.split(",")]
+            decs = [] if dec == "-" else [tuple(map(int, d.split(":"))) for d in dec.split(",")]
+            sl = [] if slots == "-" else list(map(int, slots.split(",")))
+            rows.append((int(tick), P, D, chunks, decs, sl, int(free)))
+    return rows
+
+
+def test_w1_full_trace():
+    cfg = SchedParams(iterp=2, maxp=16, minp=2, kvthresh_num=1, kvthresh_den=4,
+                      pp_depth=2, num_blocks=16, block_size=4)
+    st = Stream("W1", [Request(0, 0, 12, 3, np.zeros(14, np.int32)),
+                       Request(1, 1, 5, 2, np.zeros(6, np.int32))])
+    s, batches = run(cfg, st)
+    gold = _parse_w1()
+    assert len(batches) == len(gold)
+    for b, (tick, P, D, chunks, decs, sl, free) in zip(batches, gold):
+        assert b.tick == tick
+        assert (b.P, b.D) == (P, D), tick
+        assert [(c[0], c[1], c[2]) for c in b.chunks] == chunks, tick
+        assert list(b.decodes) == decs, tick
+        assert list(b.slot_mapping) == sl, tick
+        assert b.stats[3] == free, tick
+    assert sorted(s.free) == list(range(16))
+
+
+def test_c0_trace():
+    cfg = SCHED["C0"]
+    st = make_stream("C0", 512)
+    s = Scheduler(cfg, st.requests)
+    b0 = s.build_batch()
+    assert b0.P == 245 and b0.num_tokens == 245 and len(b0.chunks) == 8
+    assert cfg.num_blocks - len(s.free) == 19
+    b1 = s.build_batch()
+    assert b1.stats[2] == 45                      # free after retire
+    assert [(c[0], c[1], c[2]) for c in b1.chunks] == [(8, 0, 64)]
+    assert len(b1.decodes) == 8 and b1.num_tokens == 72
+    assert list(b1.slot_mapping[64:]) == [1, 31, 304, 65, 111, 320, 177, 292]
+    assert cfg.num_blocks - len(s.free) == 25
+    # decodes sit on block edges 15/16/17, 31/32/33
+    assert [p for (_, p) in b1.decodes] == [1, 15, 16, 17, 31, 32, 33, 100]
+    assert list(b1.sample_idx) == [63] + list(range(64, 72))
+
+
+def test_c0b_trace():
+    st = make_stream("C0b", 512)
+    s, bs = run(SCHED["C0b"], st)
+    assert [[(c[1], c[2]) for c in b.chunks] for b in bs[:3]] == [[(0, 40)], [(40, 38)], [(78, 26)]]
+    # tick-1 UT cap: floor(40*(61*20-64)/(64*19)) = 38  (Eq.3 UT term, L169)
+    assert bs[1].P == 38 and bs[1].stats[2] == 61
+    assert bs[3].decodes == [(0, 104)] and list(bs[3].slot_mapping) == [104]
+
+
+def _check_invariants(cfg, st, max_ticks=None):
+    s = Scheduler(cfg, st.requests, st.warm)
+    live = {}       # slot -> (req, pos)
+    total_p = 0
+    while not s.done() and (max_ticks is None or s.tick < max_ticks):
+        b = s.build_batch()
+        total_p += b.num_prefill_tokens
+        # live slots unique within a batch
+        assert len(set(b.slot_mapping.tolist())) == b.num_tokens
+        # block tables: no block held by two live requests
+        owners = {}
+        for r in s.admitted:
+            for blk in r.blocks:
+                assert blk not in owners, "block double-allocated"
+                owners[blk] = r.req_id
+        assert len(owners) + len(s.free) == cfg.num_blocks
+        assert len(set(s.free)) == len(s.free)
+        # slots of this batch lie in blocks owned by the token's request
+        for t, slot in enumerate(b.slot_mapping):
+            seq = np.searchsorted(b.cu_q, t, side="right") - 1
+            assert owners[int(slot) // cfg.block_size] == int(b.seq_req_ids[seq])
+        # KV_free bookkeeping: free after build == free before - allocations + preemption releases
+        assert b.stats[3] == len(s.free)
+        assert b.num_tokens <= cfg.maxp + -(-max(b.stats[0], 1) // cfg.pp_depth) or cfg.policy == 1
+    return s, total_p
+
+
+def test_invariants_and_prompt_conservation_small_stream():
+    st = make_stream("C1", 1024, n=300)
+    cfg = SchedParams(pp_depth=2, num_blocks=2000)
+    s, total_p = _check_invariants(cfg, st)
+    assert s.done()
+    assert total_p == sum(r.prompt_len for r in st.requests) + 0 * s.preemptions
+    assert sorted(s.free) == list(range(cfg.num_blocks))
+    assert all(r.gen == r.output_len for r in s.finished)
+
+
+def test_preemption_recompute_tiny_pool():
+    # pool so small that decodes run out of blocks -> preemption by recompute (R14)
+    st = make_stream("C1", 1024, n=60)
+    cfg = SchedParams(pp_depth=2, num_blocks=120, kvthresh_num=0, kvthresh_den=20)
+    s, total_p = _check_invariants(cfg, st)
+    assert s.done()
+    assert s.preemptions > 0
+    # every prompt token prefilled at least once; recompute adds the regenerated tokens
+    assert total_p >= sum(r.prompt_len for r in st.requests)
+    assert sorted(s.free) == list(range(cfg.num_blocks))
+    assert all(r.gen == r.output_len for r in s.finished)
+
+
+def test_decode_fairness_once_per_pp_ticks():
+    # with enough KV, every decode-phase request is scheduled at least once every PP..2PP ticks
+    st = make_stream("C1", 1024, n=150)
+    cfg = SchedParams(pp_depth=4, num_blocks=5000)
+    s = Scheduler(cfg, st.requests)
+    last = {}
+    while not s.done():
+        b = s.build_batch()
+        for (rid, _p) in b.decodes:
+            if rid in last:
+                assert b.tick - last[rid] >= cfg.pp_depth
+            last[rid] = b.tick

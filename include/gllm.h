@@ -1,0 +1,217 @@
+/* gllm.h -- C ABI of the B200-native per-stage mixed-batch forward of gLLM
+ * (Guo et al., "gLLM: Global Balanced Pipeline Parallelism Systems for
+ * Distributed LLMs Serving with Token Throttling", SC'25).
+ * Citations "Lnnn" are line numbers of /root/reference/PAPER.md.
+ *
+ * Conventions
+ *   - Every call returns int: 0 = GLLM_OK, > 0 = benign status, < 0 = error.
+ *     gllm_last_error() returns the thread-local message of the last error.
+ *     No C++ exception crosses the ABI; nothing aborts or prints.
+ *   - "host" pointers are ordinary CPU memory; "device" pointers are CUDA
+ *     global memory of the stage's device.  Buffers passed in are owned by the
+ *     caller unless stated otherwise; the library never frees them.
+ *   - No torch types appear here; PyTorch only allocates hidden buffers /
+ *     streams and exchanges the NCCL unique id (north_star).
+ */
+#ifndef GLLM_H
+#define GLLM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define GLLM_API __attribute__((visibility("default")))
+#else
+#define GLLM_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  GLLM_OK = 0,
+  GLLM_EMPTY = 1,      /* tick had nothing to schedule (R16) */
+  GLLM_EINVAL = -1,    /* argument / batch validation failed */
+  GLLM_ENOMEM = -2,    /* device or host allocation failed */
+  GLLM_ECUDA = -3,     /* CUDA runtime error (message has cudaGetErrorString) */
+  GLLM_ENCCL = -4,     /* NCCL error */
+  GLLM_ESTATE = -5     /* call out of order (e.g. retire of an unknown tick) */
+};
+
+GLLM_API const char* gllm_last_error(void);
+/* Library build tag: "gllm-b200 sm_100a <git-less version>". */
+GLLM_API const char* gllm_version(void);
+
+/* ------------------------------------------------------------------------ */
+/* Model (the decoder-only transformer of L73 §2.1; Llama / Qwen2 shapes of  */
+/* the paper's evaluation, L218/L224).                                        */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int32_t n_layers, hidden, n_heads, n_kv_heads, head_dim, intermediate, vocab;
+  float rms_eps, rope_theta;
+  int32_t qkv_bias;      /* 1 = Qwen2-style q/k/v biases */
+  uint64_t weight_seed;  /* O4 counter-based weight generator seed */
+} gllm_model_cfg;
+
+/* ------------------------------------------------------------------------ */
+/* Scheduler: Token Throttling (L145-L183 §3.1-3.2) + paged-KV block manager */
+/* (L136 Fig.6).  Host-only, deterministic, single-threaded per object. */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int32_t iterp;          /* #T  (Eq.1/Eq.3; default 8, L248) */
+  int32_t maxp, minp;     /* #MaxP, #MinP (L151; 2048 / 32, L248) */
+  int32_t kvthresh_num;   /* KV_thresh = num/den (L165; 0.05 = 1/20, L248); 0 <= num < den */
+  int32_t kvthresh_den;
+  int32_t pp_depth;       /* #PP_depth (Eq.4) = max micro-batches in flight (L179) */
+  int32_t num_blocks;     /* N, KV blocks shared by all stages (L136) */
+  int32_t block_size;     /* tokens per KV block (16) */
+  int32_t max_seqs;       /* max running sequences (1024, L575) */
+  int32_t policy;         /* 0 = Token Throttling; 1 = Sarathi-Serve (decodes first, prefill to budget) */
+  int32_t token_budget;   /* Sarathi only (2048, L248) */
+} gllm_sched_cfg;
+
+typedef struct gllm_sched gllm_sched;
+
+/* Creates a scheduler.  EINVAL on non-positive sizes or kvthresh outside [0,1). */
+GLLM_API int gllm_sched_create(const gllm_sched_cfg* cfg, gllm_sched** out);
+GLLM_API int gllm_sched_free(gllm_sched* s);
+
+/* Queues a request arriving at `arrival_tick` (reading R4: arrivals in ticks).
+ * token_ids: host, prompt_len + output_len - 1 ids (prompt, then the
+ * teacher-forced outputs t1..t_{out-1}, R17); copied.  EINVAL on
+ * prompt_len < 1, output_len < 1 or a duplicate req_id. */
+GLLM_API int gllm_sched_add_request(gllm_sched* s, int64_t req_id, int64_t arrival_tick,
+                           int32_t prompt_len, int32_t output_len, const int32_t* token_ids);
+
+/* Adds a sequence already in decode (warm start, C4): context_len tokens are
+ * cached (blocks allocated now, lowest first) and remaining_out decodes follow.
+ * token_ids: host, context_len + remaining_out ids; copied.  ENOMEM if the
+ * pool cannot hold the context. */
+GLLM_API int gllm_sched_add_warm(gllm_sched* s, int64_t req_id, int32_t context_len,
+                        int32_t remaining_out, const int32_t* token_ids);
+
+/* Pure Eq.3 + L165 threshold (P) and Eq.4 (D) in exact integer arithmetic
+ * (readings R6, R10, R11):
+ *   P = 0 if wp == 0 or free*den < num*N, else
+ *   P = min(max(min(wp / iterp, MaxP*(free*den - num*N) / (N*(den-num))), MinP), wp)
+ *   D = ceil(rd / pp_depth)                              (all divisions floor) */
+GLLM_API int gllm_throttle_counts(const gllm_sched_cfg* cfg, int64_t wp, int64_t rd, int32_t free_blocks,
+                         int32_t* P, int32_t* D);
+
+/* One scheduled micro-batch (D3/D4 of SURVEY §2.3).  Layout (R15): prefill
+ * chunks first (selection order), then decode tokens.  All arrays are host
+ * memory owned by the scheduler and valid until gllm_retire_batch(tick). */
+typedef struct {
+  int64_t tick;
+  int32_t P, D;                 /* counts computed by Eq.3 / Eq.4 this tick */
+  int32_t num_prefill_tokens, num_decode_tokens, num_tokens;
+  int32_t num_seqs, num_prefill_seqs, max_blocks_per_seq, num_samples;
+  const int32_t* token_ids;     /* [num_tokens] */
+  const int32_t* positions;     /* [num_tokens] absolute positions */
+  const int32_t* slot_mapping;  /* [num_tokens] slot = bt[pos/bs]*bs + pos%bs (O2) */
+  const int32_t* cu_q;          /* [num_seqs+1] token offsets of each sequence */
+  const int32_t* kv_len;        /* [num_seqs] keys visible to the sequence's last token */
+  const int32_t* block_table;   /* [num_seqs * max_blocks_per_seq], -1 padded */
+  const int32_t* sample_token_idx; /* [num_samples] rows whose next token is sampled */
+  const int64_t* seq_req_ids;   /* [num_seqs] */
+} gllm_batch_desc;
+
+/* Builds the micro-batch of the current tick k and advances the tick:
+ * retires batch k - pp_depth first (R1), admits arrivals, computes the global
+ * statistics #WP, #RD, KV_free (L151, L161, L183), throttles (Eq.3, Eq.4),
+ * selects decodes then prefill chunks, allocates blocks (decode first, lowest
+ * free block first) and fills *out.  Returns GLLM_EMPTY (with *out valid,
+ * num_tokens == 0) for a tick with nothing scheduled; the tick still occupies
+ * an in-flight slot (R16). */
+GLLM_API int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out);
+
+/* Optionally records the sampled ids of `tick` early (the automatic retire in
+ * build_batch k+pp_depth then applies them).  sampled_ids: host
+ * [num_samples] or NULL.  ESTATE if tick is not in flight. */
+GLLM_API int gllm_retire_batch(gllm_sched* s, int64_t tick, const int32_t* sampled_ids);
+
+/* 1 when every request has finished and no arrival is pending. */
+GLLM_API int gllm_sched_done(const gllm_sched* s);
+
+/* Scheduler statistics: [0] tick, [1] running requests, [2] free blocks,
+ * [3] preemptions so far, [4] finished requests, [5] requests admitted. */
+GLLM_API int gllm_sched_stats(const gllm_sched* s, int64_t* out6);
+
+/* Canonical little-endian int64 trace of the LAST built tick (layout in
+ * DESIGN.md §3; identical to oracle.scheduler.trace_bytes).  *used receives
+ * the byte count; EINVAL if cap is too small (then *used is the size needed). */
+GLLM_API int gllm_sched_trace(gllm_sched* s, void* buf, size_t cap, size_t* used);
+
+/* ------------------------------------------------------------------------ */
+/* Stage: one pipeline stage's layers on one GPU (P1, L90-L92, L198).         */
+/* ------------------------------------------------------------------------ */
+typedef struct gllm_stage gllm_stage;
+
+/* init_stage(layers, kv_blocks): allocates on `device` the bf16 weights of
+ * layers [layer_begin, layer_end) (+ embedding if layer_begin == 0, + final
+ * norm and LM head if layer_end == n_layers), fills them with the O4
+ * generator on the GPU, allocates the paged KV cache (kv_blocks x block_size
+ * tokens for every local layer) and workspaces for up to max_tokens tokens and
+ * max_seqs sequences per micro-batch.  EINVAL for inconsistent shapes
+ * (head_dim != 128 and != 64, hidden % 64, intermediate % 128, ...), ENOMEM
+ * when HBM does not fit. */
+GLLM_API int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t layer_end,
+                    int32_t kv_blocks, int32_t block_size, int32_t max_tokens,
+                    int32_t max_seqs, int32_t device, gllm_stage** out);
+GLLM_API int gllm_free_stage(gllm_stage* st);
+
+/* stage_forward(batch_desc, hidden_in, hidden_out): enqueues the whole stage
+ * forward on `stream` (a cudaStream_t, NULL = the legacy default stream) and
+ * returns immediately.  The desc is validated (T <= max_tokens, S <= max_seqs,
+ * block ids < kv_blocks, positions < kv_len -> EINVAL) and snapshotted into
+ * stage-owned pinned staging before return, so the caller may reuse it.
+ *   hidden_in:   device fp32 [num_tokens, hidden]; ignored (may be NULL) on stage 0.
+ *   hidden_out:  device fp32 [num_tokens, hidden] residual after the last local
+ *                layer; may be NULL on the last stage; may equal hidden_in.
+ *   sampled_out: device int32 [num_samples] greedy ids (last stage only; may be NULL).
+ * Async CUDA errors surface on the next call or on gllm_stage_sync. */
+GLLM_API int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* desc, const void* hidden_in,
+                       void* hidden_out, int32_t* sampled_out, void* stream);
+
+/* Pipeline hand-off (a12; activations over NCCL, L222).  comm_init joins an
+ * NCCL communicator of `world` ranks (unique_id: 128 bytes from ncclGetUniqueId,
+ * exchanged by the caller).  send/recv move num_tokens x hidden fp32 rows of a
+ * device buffer to/from rank dst/src on `stream`. */
+GLLM_API int gllm_get_unique_id(void* out128);
+GLLM_API int gllm_comm_init(gllm_stage* st, const void* nccl_unique_id, int32_t rank, int32_t world);
+GLLM_API int gllm_send_hidden(gllm_stage* st, const void* buf, int32_t num_tokens, int32_t dst, void* stream);
+GLLM_API int gllm_recv_hidden(gllm_stage* st, void* buf, int32_t num_tokens, int32_t src, void* stream);
+GLLM_API int gllm_stage_sync(gllm_stage* st);
+
+/* Introspection for parity tests (host outputs, synchronous). */
+/* Copies element range [row0, row0+nrows) x all columns of a logical weight
+ * ("wq","wk","wv","wo","wg","wu","wd","bq","bk","bv","embed","lm_head") of
+ * `layer` as fp32 into host `out`. */
+GLLM_API int gllm_stage_read_weight(gllm_stage* st, int32_t layer, const char* name, int64_t row0,
+                           int64_t nrows, float* out);
+/* Reads K and V of `n` cache slots of local `layer` as fp32 host [n, n_kv_heads, head_dim]. */
+GLLM_API int gllm_stage_read_kv(gllm_stage* st, int32_t layer, const int32_t* slots, int32_t n,
+                       float* k_out, float* v_out);
+/* Device slot mapping produced by the last stage_forward, host int32 [num_tokens]. */
+GLLM_API int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n);
+/* Fills the KV cache of local layer `layer` (or all layers if layer < 0) with the
+ * O4-style generator (warm start): element i of K (resp. V) of layer l has
+ * tensor id 0xEE0000 + 2*l (+1 for V).  Used by benchmarks for warm decode state. */
+GLLM_API int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed);
+
+/* Timing of the last forward from CUDA events recorded on the forward's own
+ * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).
+ * out[n] receives milliseconds per category (synchronises on the events):
+ *   [0] whole forward  [1] QKV GEMM  [2] O GEMM  [3] gate_up GEMM  [4] down GEMM
+ *   [5] prefill attention  [6] decode attention  [7] RoPE+KV append  [8] RMSNorm
+ *   [9] final norm + LM head + argmax  [10] other (prep, embedding) */
+GLLM_API int gllm_stage_set_profiling(gllm_stage* st, int32_t on);
+GLLM_API int gllm_stage_last_timing(gllm_stage* st, float* out, int32_t n);
+/* Number of kernels the last stage_forward launched. */
+GLLM_API int gllm_stage_last_launches(gllm_stage* st, int32_t* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GLLM_H */

@@ -1,0 +1,432 @@
+// Varlen paged causal attention (a7): prefill chunks on tensor cores, decode rows as
+// bandwidth-bound paged gathers with warp-level softmax reductions.
+//
+//   prefill chunk i (c_i tokens at offset s_i): token j attends keys [0, s_i + j]
+//   decode row j (position L_j - 1):           attends keys [0, L_j - 1]
+//   softmax(q k^T / sqrt(D)) v, GQA: q head h uses kv head h / G, G = Hq / Hkv
+//
+// Cache layout per layer: K, V each [kv_blocks][Hkv][16][D] bf16, so one
+// (block, kv head) page is a contiguous 16 x D tile (4 KB at D = 128).
+#include <cuda_bf16.h>
+
+#include "attention.cuh"
+#include "common.h"
+#include "ptx.cuh"
+
+namespace gllm {
+
+namespace {
+
+constexpr float LOG2E = 1.4426950408889634f;
+
+__device__ __forceinline__ float dot8(const uint4& a, const uint4& b) {
+  const __nv_bfloat162* x = reinterpret_cast<const __nv_bfloat162*>(&a);
+  const __nv_bfloat162* y = reinterpret_cast<const __nv_bfloat162*>(&b);
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const float2 p = __bfloat1622float2(x[i]), q = __bfloat1622float2(y[i]);
+    s = fmaf(p.x, q.x, s);
+    s = fmaf(p.y, q.y, s);
+  }
+  return s;
+}
+
+// ------------------------------------------------------------------ decode
+// CTA = (decode row, key split) x kv head; 4 warps stride over the split's 16-token pages.
+// Within a warp: LPT lanes cover one token's D dims (8 bf16 per lane), TPI tokens per
+// 16-byte load, so a page is NI loads per lane for K and NI for V.
+template <int D, int G>
+__global__ void __launch_bounds__(128) decode_attn_kernel(const AttnArgs a, const DecodeItem* __restrict__ items) {
+  constexpr int LPT = D / 8;
+  constexpr int TPI = 32 / LPT;
+  constexpr int NI = 16 / TPI;
+  __shared__ float sm_m[4][G], sm_l[4][G];
+  __shared__ float sm_acc[4][G][D];
+
+  const DecodeItem it = items[blockIdx.x];
+  const int kvh = blockIdx.y;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int t = a.cu_q[it.seq];
+  const int L = a.kv_len[it.seq];
+  const int k0 = it.split * a.split_len;
+  const int k1 = min(L, k0 + a.split_len);
+  const int nb0 = k0 / 16, nb1 = (k1 + 15) / 16;
+  const int d0 = (lane % LPT) * 8;
+  const int tk = lane / LPT;
+  const float sl2 = LOG2E * rsqrtf((float)D);
+
+  uint4 qv[G];
+#pragma unroll
+  for (int h = 0; h < G; ++h)
+    qv[h] = *reinterpret_cast<const uint4*>(a.q + (size_t)t * a.q_stride + (size_t)(kvh * G + h) * D + d0);
+  float m[G], l[G], acc[G][8];
+#pragma unroll
+  for (int h = 0; h < G; ++h) {
+    m[h] = -INFINITY;
+    l[h] = 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[h][j] = 0.f;
+  }
+  const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
+  for (int b = nb0 + warp; b < nb1; b += 4) {
+    const size_t page = (size_t)bt[b];
+    const __nv_bfloat16* kb = a.kc + ((page * a.Hkv + kvh) * 16) * D;
+    const __nv_bfloat16* vb = a.vc + ((page * a.Hkv + kvh) * 16) * D;
+    uint4 kr[NI], vr[NI];
+#pragma unroll
+    for (int i = 0; i < NI; ++i) kr[i] = ptx::ld_nc_v4(kb + (tk + i * TPI) * D + d0);
+#pragma unroll
+    for (int i = 0; i < NI; ++i) vr[i] = ptx::ld_nc_v4(vb + (tk + i * TPI) * D + d0);
+    float s[NI][G];
+#pragma unroll
+    for (int i = 0; i < NI; ++i)
+#pragma unroll
+      for (int h = 0; h < G; ++h) s[i][h] = dot8(qv[h], kr[i]);
+#pragma unroll
+    for (int o = 1; o < LPT; o <<= 1)
+#pragma unroll
+      for (int i = 0; i < NI; ++i)
+#pragma unroll
+        for (int h = 0; h < G; ++h) s[i][h] += __shfl_xor_sync(0xffffffffu, s[i][h], o);
+#pragma unroll
+    for (int i = 0; i < NI; ++i) {
+      const bool ok = b * 16 + tk + i * TPI < k1;
+#pragma unroll
+      for (int h = 0; h < G; ++h) s[i][h] = ok ? s[i][h] * sl2 : -INFINITY;
+    }
+#pragma unroll
+    for (int h = 0; h < G; ++h) {
+      float mx = s[0][h];
+#pragma unroll
+      for (int i = 1; i < NI; ++i) mx = fmaxf(mx, s[i][h]);
+#pragma unroll
+      for (int o = LPT; o < 32; o <<= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+      const float mn = fmaxf(m[h], mx);
+      const float corr = exp2f(m[h] - mn);
+      m[h] = mn;
+      l[h] *= corr;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[h][j] *= corr;
+#pragma unroll
+      for (int i = 0; i < NI; ++i) {
+        const float p = exp2f(s[i][h] - mn);
+        l[h] += p;
+        const __nv_bfloat162* v2 = reinterpret_cast<const __nv_bfloat162*>(&vr[i]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const float2 vf = __bfloat1622float2(v2[j]);
+          acc[h][2 * j] = fmaf(p, vf.x, acc[h][2 * j]);
+          acc[h][2 * j + 1] = fmaf(p, vf.y, acc[h][2 * j + 1]);
+        }
+      }
+    }
+  }
+  // combine the TPI token groups of the warp (m is warp-uniform)
+#pragma unroll
+  for (int o = LPT; o < 32; o <<= 1)
+#pragma unroll
+    for (int h = 0; h < G; ++h) {
+      l[h] += __shfl_xor_sync(0xffffffffu, l[h], o);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[h][j] += __shfl_xor_sync(0xffffffffu, acc[h][j], o);
+    }
+  if (tk == 0) {
+#pragma unroll
+    for (int h = 0; h < G; ++h) {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) sm_acc[warp][h][d0 + j] = acc[h][j];
+      if (lane == 0) {
+        sm_m[warp][h] = m[h];
+        sm_l[warp][h] = l[h];
+      }
+    }
+  }
+  __syncthreads();
+  for (int idx = threadIdx.x; idx < G * D; idx += blockDim.x) {
+    const int h = idx / D, d = idx % D;
+    float M = sm_m[0][h];
+#pragma unroll
+    for (int w = 1; w < 4; ++w) M = fmaxf(M, sm_m[w][h]);
+    float Ls = 0.f, A = 0.f;
+#pragma unroll
+    for (int w = 0; w < 4; ++w) {
+      const float f = exp2f(sm_m[w][h] - M);
+      Ls += sm_l[w][h] * f;
+      A += sm_acc[w][h][d] * f;
+    }
+    if (it.part < 0) {
+      a.out[(size_t)t * a.Hq * D + (size_t)(kvh * G + h) * D + d] = __float2bfloat16_rn(A / Ls);
+    } else {
+      const size_t base = ((size_t)it.part * a.Hkv + kvh) * G + h;
+      a.part_o[base * D + d] = A;
+      if (d == 0) {
+        a.part_ml[base * 2] = M;
+        a.part_ml[base * 2 + 1] = Ls;
+      }
+    }
+  }
+}
+
+template <int D, int G>
+__global__ void __launch_bounds__(128) decode_merge_kernel(const AttnArgs a, const MergeItem* __restrict__ merges) {
+  const MergeItem mi = merges[blockIdx.x];
+  const int kvh = blockIdx.y;
+  const int t = a.cu_q[mi.seq];
+  for (int idx = threadIdx.x; idx < G * D; idx += blockDim.x) {
+    const int h = idx / D, d = idx % D;
+    float M = -INFINITY;
+    for (int s = 0; s < mi.nsplit; ++s)
+      M = fmaxf(M, a.part_ml[(((size_t)(mi.first + s) * a.Hkv + kvh) * G + h) * 2]);
+    float Ls = 0.f, A = 0.f;
+    for (int s = 0; s < mi.nsplit; ++s) {
+      const size_t base = ((size_t)(mi.first + s) * a.Hkv + kvh) * G + h;
+      const float f = exp2f(a.part_ml[base * 2] - M);
+      Ls += a.part_ml[base * 2 + 1] * f;
+      A += a.part_o[base * D + d] * f;
+    }
+    a.out[(size_t)t * a.Hq * D + (size_t)(kvh * G + h) * D + d] = __float2bfloat16_rn(A / Ls);
+  }
+}
+
+// ------------------------------------------------------------------ prefill
+// CTA = 64 flattened (token, group head) rows of one chunk x one kv head; 4 warps x 16 rows.
+// K/V tiles of 64 keys (4 pages) double-buffered in SMEM with cp.async; S = Q K^T and
+// O += P V on mma.sync m16n8k16 (bf16 in, fp32 accumulate); online softmax in registers.
+template <int D>
+struct PrefillSmem {
+  static constexpr int ROW_BYTES = D * 2;
+  static constexpr int TILE_BYTES = 64 * ROW_BYTES;
+  static constexpr int BYTES = 5 * TILE_BYTES;  // Q + 2 x (K, V)
+};
+
+// swizzled byte offset of (row, 16-byte chunk) in a [64][D] bf16 tile
+template <int D>
+__device__ __forceinline__ uint32_t swz(int row, int chunk) {
+  return row * (D * 2) + ((chunk ^ (row & 7)) << 4);
+}
+
+template <int D>
+__global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
+  constexpr int NCH = D / 8;  // 16-byte chunks per row
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint8_t* sQ = smem;
+  uint8_t* sK[2] = {smem + PrefillSmem<D>::TILE_BYTES, smem + 2 * PrefillSmem<D>::TILE_BYTES};
+  uint8_t* sV[2] = {smem + 3 * PrefillSmem<D>::TILE_BYTES, smem + 4 * PrefillSmem<D>::TILE_BYTES};
+
+  const PrefillItem it = items[blockIdx.x];
+  const int kvh = blockIdx.y;
+  const int G = a.Hq / a.Hkv;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int t0 = a.cu_q[it.seq];
+  const int c = a.cu_q[it.seq + 1] - t0;
+  const int s0 = a.kv_len[it.seq] - c;  // chunk offset
+  const int nrows = c * G;
+  const int row_last = min(it.row0 + 63, nrows - 1);
+  const int max_pos = s0 + row_last / G;
+  const int n_kt = (max_pos + 64) / 64;  // key tiles covering [0, max_pos]
+  const int nblk_seq = (a.kv_len[it.seq] + 15) / 16;
+  const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
+  const float sl2 = LOG2E * rsqrtf((float)D);
+
+  // ---- Q tile -> SMEM (rows beyond the chunk are clamped to the last row; never stored)
+  for (int idx = threadIdx.x; idx < 64 * NCH; idx += 128) {
+    const int r = idx / NCH, ch = idx % NCH;
+    const int rr = min(it.row0 + r, nrows - 1);
+    const int tok = rr / G, h = kvh * G + rr % G;
+    const __nv_bfloat16* src = a.q + (size_t)(t0 + tok) * a.q_stride + (size_t)h * D + ch * 8;
+    ptx::cp_async16(ptx::smem_u32(sQ) + swz<D>(r, ch), src, true);
+  }
+  auto load_kv = [&](int kt, int buf) {
+    for (int idx = threadIdx.x; idx < 64 * NCH; idx += 128) {
+      const int r = idx / NCH, ch = idx % NCH;
+      const int key = kt * 64 + r;
+      const int blk = key >> 4;
+      const bool ok = blk < nblk_seq;
+      const size_t page = ok ? (size_t)bt[blk] : 0;
+      const size_t off = ((page * a.Hkv + kvh) * 16 + (key & 15)) * D + ch * 8;
+      ptx::cp_async16(ptx::smem_u32(sK[buf]) + swz<D>(r, ch), a.kc + off, ok);
+      ptx::cp_async16(ptx::smem_u32(sV[buf]) + swz<D>(r, ch), a.vc + off, ok);
+    }
+  };
+  load_kv(0, 0);
+  ptx::cp_async_commit();
+
+  // per-thread rows of the m16n8 fragments: g and g + 8 of this warp's 16 rows
+  const int g = lane >> 2, tq = lane & 3;
+  int pos_r[2];
+#pragma unroll
+  for (int hr = 0; hr < 2; ++hr) {
+    const int rr = min(it.row0 + warp * 16 + g + hr * 8, nrows - 1);
+    pos_r[hr] = s0 + rr / G;
+  }
+  const int pos_min_warp = s0 + min(it.row0 + warp * 16, nrows - 1) / G;
+
+  uint32_t qa[D / 16][4];
+  float o[D / 8][4];
+#pragma unroll
+  for (int n = 0; n < D / 8; ++n) o[n][0] = o[n][1] = o[n][2] = o[n][3] = 0.f;
+  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
+
+  for (int kt = 0; kt < n_kt; ++kt) {
+    if (kt + 1 < n_kt) load_kv(kt + 1, (kt + 1) & 1);
+    ptx::cp_async_commit();
+    ptx::cp_async_wait<1>();
+    __syncthreads();
+    if (kt == 0) {
+#pragma unroll
+      for (int ks = 0; ks < D / 16; ++ks) {
+        const int r = warp * 16 + (lane & 15);
+        const int ch = ks * 2 + (lane >> 4);
+        ptx::ldsm_x4(ptx::smem_u32(sQ) + swz<D>(r, ch), qa[ks][0], qa[ks][1], qa[ks][2], qa[ks][3]);
+      }
+    }
+    const int buf = kt & 1;
+    // ---- S = Q K^T  (16 rows x 64 keys per warp)
+    float s[8][4];
+#pragma unroll
+    for (int n = 0; n < 8; ++n) s[n][0] = s[n][1] = s[n][2] = s[n][3] = 0.f;
+#pragma unroll
+    for (int ks = 0; ks < D / 16; ++ks) {
+#pragma unroll
+      for (int np = 0; np < 4; ++np) {
+        const int r = np * 16 + ((lane >> 4) << 3) + (lane & 7);
+        const int ch = ks * 2 + ((lane >> 3) & 1);
+        uint32_t b0, b1, b2, b3;
+        ptx::ldsm_x4(ptx::smem_u32(sK[buf]) + swz<D>(r, ch), b0, b1, b2, b3);
+        ptx::mma_bf16_16816(s[2 * np], qa[ks], b0, b1);
+        ptx::mma_bf16_16816(s[2 * np + 1], qa[ks], b2, b3);
+      }
+    }
+    // ---- scale, causal mask, online softmax
+    const bool need_mask = kt * 64 + 63 > pos_min_warp;
+#pragma unroll
+    for (int n = 0; n < 8; ++n)
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const int key = kt * 64 + n * 8 + 2 * tq + (e & 1);
+        const int hr = e >> 1;
+        s[n][e] = (need_mask && key > pos_r[hr]) ? -INFINITY : s[n][e] * sl2;
+      }
+    float corr[2];
+#pragma unroll
+    for (int hr = 0; hr < 2; ++hr) {
+      float mx = -INFINITY;
+#pragma unroll
+      for (int n = 0; n < 8; ++n) mx = fmaxf(mx, fmaxf(s[n][2 * hr], s[n][2 * hr + 1]));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
+      const float mn = fmaxf(mrow[hr], mx);
+      corr[hr] = exp2f(mrow[hr] - mn);
+      mrow[hr] = mn;
+      float sum = 0.f;
+#pragma unroll
+      for (int n = 0; n < 8; ++n) {
+        s[n][2 * hr] = exp2f(s[n][2 * hr] - mn);
+        s[n][2 * hr + 1] = exp2f(s[n][2 * hr + 1] - mn);
+        sum += s[n][2 * hr] + s[n][2 * hr + 1];
+      }
+      lrow[hr] = lrow[hr] * corr[hr] + sum;
+    }
+#pragma unroll
+    for (int n = 0; n < D / 8; ++n) {
+      o[n][0] *= corr[0];
+      o[n][1] *= corr[0];
+      o[n][2] *= corr[1];
+      o[n][3] *= corr[1];
+    }
+    // ---- O += P V
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk) {
+      uint32_t pa[4];
+      pa[0] = ptx::pack_bf16(s[2 * kk][0], s[2 * kk][1]);
+      pa[1] = ptx::pack_bf16(s[2 * kk][2], s[2 * kk][3]);
+      pa[2] = ptx::pack_bf16(s[2 * kk + 1][0], s[2 * kk + 1][1]);
+      pa[3] = ptx::pack_bf16(s[2 * kk + 1][2], s[2 * kk + 1][3]);
+#pragma unroll
+      for (int dp = 0; dp < D / 16; ++dp) {
+        const int r = kk * 16 + (lane & 7) + (((lane >> 3) & 1) << 3);
+        const int ch = dp * 2 + (lane >> 4);
+        uint32_t b0, b1, b2, b3;
+        ptx::ldsm_x4_t(ptx::smem_u32(sV[buf]) + swz<D>(r, ch), b0, b1, b2, b3);
+        ptx::mma_bf16_16816(o[2 * dp], pa, b0, b1);
+        ptx::mma_bf16_16816(o[2 * dp + 1], pa, b2, b3);
+      }
+    }
+    __syncthreads();
+  }
+  // ---- normalise and store
+#pragma unroll
+  for (int hr = 0; hr < 2; ++hr) {
+    float lt = lrow[hr];
+    lt += __shfl_xor_sync(0xffffffffu, lt, 1);
+    lt += __shfl_xor_sync(0xffffffffu, lt, 2);
+    const float inv = 1.f / lt;
+    const int rr = it.row0 + warp * 16 + g + hr * 8;
+    if (rr < nrows) {
+      const int tok = rr / G, h = kvh * G + rr % G;
+      __nv_bfloat16* dst = a.out + (size_t)(t0 + tok) * a.Hq * D + (size_t)h * D;
+#pragma unroll
+      for (int n = 0; n < D / 8; ++n)
+        *reinterpret_cast<uint32_t*>(dst + n * 8 + 2 * tq) = ptx::pack_bf16(o[n][2 * hr] * inv, o[n][2 * hr + 1] * inv);
+    }
+  }
+}
+
+template <int D, int G>
+int launch_decode_t(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges,
+                    cudaStream_t s) {
+  if (n_items > 0) decode_attn_kernel<D, G><<<dim3(n_items, a.Hkv), 128, 0, s>>>(a, items);
+  if (n_merges > 0) decode_merge_kernel<D, G><<<dim3(n_merges, a.Hkv), 128, 0, s>>>(a, merges);
+  return GLLM_OK;
+}
+
+template <int D>
+int launch_decode_d(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges,
+                    cudaStream_t s) {
+  switch (a.Hq / a.Hkv) {
+    case 1: return launch_decode_t<D, 1>(a, items, n_items, merges, n_merges, s);
+    case 2: return launch_decode_t<D, 2>(a, items, n_items, merges, n_merges, s);
+    case 4: return launch_decode_t<D, 4>(a, items, n_items, merges, n_merges, s);
+    case 5: return launch_decode_t<D, 5>(a, items, n_items, merges, n_merges, s);
+    case 8: return launch_decode_t<D, 8>(a, items, n_items, merges, n_merges, s);
+  }
+  return set_error(GLLM_EINVAL, "decode attention: unsupported GQA group %d", a.Hq / a.Hkv);
+}
+
+}  // namespace
+
+int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
+  if (n_items <= 0) return GLLM_OK;
+  if (a.D == 128) {
+    static bool set = false;
+    if (!set) {
+      cudaFuncSetAttribute(prefill_attn_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           PrefillSmem<128>::BYTES);
+      set = true;
+    }
+    prefill_attn_kernel<128><<<dim3(n_items, a.Hkv), 128, PrefillSmem<128>::BYTES, s>>>(a, items);
+  } else if (a.D == 64) {
+    prefill_attn_kernel<64><<<dim3(n_items, a.Hkv), 128, PrefillSmem<64>::BYTES, s>>>(a, items);
+  } else {
+    return set_error(GLLM_EINVAL, "prefill attention: head_dim %d unsupported", a.D);
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GLLM_OK : set_error(GLLM_ECUDA, "prefill attention launch: %s", cudaGetErrorString(e));
+}
+
+int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
+                            int n_merges, cudaStream_t s) {
+  int rc;
+  if (a.D == 128)
+    rc = launch_decode_d<128>(a, items, n_items, merges, n_merges, s);
+  else if (a.D == 64)
+    rc = launch_decode_d<64>(a, items, n_items, merges, n_merges, s);
+  else
+    return set_error(GLLM_EINVAL, "decode attention: head_dim %d unsupported", a.D);
+  if (rc) return rc;
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GLLM_OK : set_error(GLLM_ECUDA, "decode attention launch: %s", cudaGetErrorString(e));
+}
+
+}  // namespace gllm

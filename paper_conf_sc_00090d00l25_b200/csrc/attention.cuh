@@ -1,0 +1,42 @@
+// Varlen paged causal attention over one mixed batch (a7 of DESIGN.md §2) -- internal interface.
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace gllm {
+
+// work item of the prefill kernel: chunk `seq`, flattened (token, group-head) rows [row0, row0+64)
+struct PrefillItem {
+  int32_t seq, row0;
+};
+// work item of the decode kernel: decode row `seq`, key split `split`; `part` = partial slot or -1
+struct DecodeItem {
+  int32_t seq, split, part, nsplit;
+};
+// merge job: decode seq `seq`, partial slots [first, first + nsplit)
+struct MergeItem {
+  int32_t seq, first, nsplit, pad;
+};
+
+struct AttnArgs {
+  const __nv_bfloat16* q;  // [T, q_stride] (rotated q heads first in each row)
+  int q_stride;
+  const __nv_bfloat16* kc;  // [kv_blocks][Hkv][bs][D]
+  const __nv_bfloat16* vc;
+  int Hq, Hkv, D, bs;
+  const int32_t* cu_q;
+  const int32_t* kv_len;
+  const int32_t* block_table;
+  int maxblk;
+  __nv_bfloat16* out;  // [T, Hq*D]
+  float* part_o;       // [nparts, Hkv, G, D]
+  float* part_ml;      // [nparts, Hkv, G, 2]
+  int split_len;       // decode keys per split (multiple of 16)
+};
+
+int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
+int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
+                            int n_merges, cudaStream_t s);
+
+}  // namespace gllm

@@ -1,0 +1,38 @@
+// tcgen05 GEMM  Y[M,N] = X[M,K] . W[N,K]^T  with fused epilogues (internal interface).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace gllm {
+
+enum GemmEpi : int {
+  EPI_STORE_BF16 = 0,  // out bf16 [M, ldo] = acc (+ bias[col] if bias)
+  EPI_ADD_F32 = 1,     // out fp32 [M, ldo] += acc          (residual add, a8 / a10)
+  EPI_SILU_MUL = 2,    // out bf16 [M, ldo] = silu(gate) * up; W rows interleaved per 128 (a9)
+  EPI_ARGMAX = 3,      // per (row, n-tile) max & argmax of acc -> partial buffers (a11)
+};
+
+struct GemmArgs {
+  int M, N, K;
+  void* out;
+  int ldo;
+  const float* bias;
+  float* part_val;   // EPI_ARGMAX: [M, num_n_tiles]
+  int32_t* part_idx; // EPI_ARGMAX: [M, num_n_tiles]
+  int num_m_tiles, num_n_tiles;
+};
+
+constexpr int GEMM_BM = 128, GEMM_BN = 256, GEMM_BK = 64, GEMM_STAGES = 4;
+
+// Encodes a 2-D bf16 K-major tensor map (rows x cols, cols contiguous) with a
+// (box_rows x 64) box and 128-byte swizzle.  Returns 0 or a GLLM_* error.
+int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols, uint32_t box_rows);
+
+// Launches the persistent GEMM on `stream`.  A map: box 128 rows; B map: box 256 rows.
+int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const GemmArgs& args,
+                cudaStream_t stream, int num_sms);
+
+int num_sms_of_current_device();
+
+}  // namespace gllm

@@ -1,0 +1,252 @@
+// Bandwidth-bound kernels of the stage forward: O4 weight init,
+// slot mapping (O2, a2), embedding gather (a3), RMSNorm (a4), fused RoPE +
+// paged KV append (a6) and the greedy argmax reduction (a11).
+#include <cuda_bf16.h>
+
+#include "kernels.cuh"
+
+namespace gllm {
+
+namespace {
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
+  x += 0x9E3779B97F4A7C15ull;
+  uint64_t z = x;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// O4: x = (u - 2^23) 2^-23 exactly, then one correctly rounded fp32 multiply by the scale.
+__device__ __forceinline__ float o4(uint64_t seed, uint64_t tid, uint64_t i, float scale) {
+  const uint64_t u = splitmix64(seed ^ (tid << 40) ^ i) >> 40;
+  const float x = (float)((int64_t)u - (int64_t)(1 << 23)) * 0x1p-23f;
+  return __fmul_rn(x, scale);
+}
+
+__global__ void init_bf16_kernel(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid,
+                                 float scale, int mode, int64_t row_offset) {
+  const int64_t n = rows * cols;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / cols, c = i - r * cols;
+    int64_t pr;
+    if (mode == 0)
+      pr = r + row_offset;
+    else
+      pr = (r / 128) * 256 + (mode == 2 ? 128 : 0) + (r % 128);
+    dst[pr * cols + c] = __float2bfloat16_rn(o4(seed, tid, (uint64_t)i, scale));
+  }
+}
+
+__global__ void init_f32_kernel(float* dst, int64_t n, uint64_t seed, uint64_t tid, float scale) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = __bfloat162float(__float2bfloat16_rn(o4(seed, tid, (uint64_t)i, scale)));
+}
+
+__global__ void fill_f32_kernel(float* dst, int64_t n, float v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = v;
+}
+
+__global__ void fill_kv_kernel(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, uint64_t seed, uint64_t tid) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    kc[i] = __float2bfloat16_rn(o4(seed, tid, (uint64_t)i, 1.7320508f));
+    vc[i] = __float2bfloat16_rn(o4(seed, tid + 1, (uint64_t)i, 1.7320508f));
+  }
+}
+
+// One thread per token: slot = bt[seq][pos / bs] * bs + pos % bs, seq found by binary search in cu_q.
+// Threads also fill the RoPE table cs[t][i] = (cos, sin)(pos * theta^(-2i/D)) in double precision.
+__global__ void prep_kernel(const int32_t* __restrict__ positions, const int32_t* __restrict__ cu_q,
+                            const int32_t* __restrict__ bt, int T, int S, int maxblk, int bs, int32_t* slots,
+                            float2* cs, int half, double log2_theta) {
+  const int t = blockIdx.x;
+  if (t >= T) return;
+  const int pos = positions[t];
+  if (threadIdx.x == 0) {
+    int lo = 0, hi = S;  // largest seq with cu_q[seq] <= t
+    while (hi - lo > 1) {
+      const int mid = (lo + hi) >> 1;
+      if (cu_q[mid] <= t) lo = mid; else hi = mid;
+    }
+    slots[t] = bt[(int64_t)lo * maxblk + pos / bs] * bs + pos % bs;
+  }
+  for (int i = threadIdx.x; i < half; i += blockDim.x) {
+    const double inv_freq = exp2(-(2.0 * i / (2.0 * half)) * log2_theta);
+    double sn, cn;
+    sincos((double)pos * inv_freq, &sn, &cn);
+    cs[(int64_t)t * half + i] = make_float2((float)cn, (float)sn);
+  }
+}
+
+__global__ void embed_kernel(const __nv_bfloat16* __restrict__ E, const int32_t* __restrict__ ids, float* x, int H) {
+  const int t = blockIdx.x;
+  const __nv_bfloat16* row = E + (int64_t)ids[t] * H;
+  float* out = x + (int64_t)t * H;
+  for (int c = threadIdx.x * 8; c < H; c += blockDim.x * 8) {
+    const uint4 v = *reinterpret_cast<const uint4*>(row + c);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&v);
+    float4 a, b;
+    float2 f0 = __bfloat1622float2(h[0]), f1 = __bfloat1622float2(h[1]);
+    float2 f2 = __bfloat1622float2(h[2]), f3 = __bfloat1622float2(h[3]);
+    a = make_float4(f0.x, f0.y, f1.x, f1.y);
+    b = make_float4(f2.x, f2.y, f3.x, f3.y);
+    *reinterpret_cast<float4*>(out + c) = a;
+    *reinterpret_cast<float4*>(out + c + 4) = b;
+  }
+}
+
+template <int NT>
+__device__ __forceinline__ float block_sum(float v, float* red) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < NT / 32; ++i) s += red[i];
+  return s;
+}
+
+// One CTA of 256 threads per row; fp32 math (a4).
+__global__ void __launch_bounds__(256) rmsnorm_kernel(const float* __restrict__ x, const float* __restrict__ g,
+                                                      __nv_bfloat16* y, const int32_t* __restrict__ rows, int H,
+                                                      float eps) {
+  __shared__ float red[8];
+  const int r = blockIdx.x;
+  const int src = rows ? rows[r] : r;
+  const float* xr = x + (int64_t)src * H;
+  float ss = 0.f;
+  for (int c = threadIdx.x * 4; c < H; c += 256 * 4) {
+    const float4 v = *reinterpret_cast<const float4*>(xr + c);
+    ss += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
+  }
+  ss = block_sum<256>(ss, red);
+  const float inv = rsqrtf(ss / (float)H + eps);
+  __nv_bfloat16* yr = y + (int64_t)r * H;
+  for (int c = threadIdx.x * 4; c < H; c += 256 * 4) {
+    const float4 v = *reinterpret_cast<const float4*>(xr + c);
+    const float4 gg = *reinterpret_cast<const float4*>(g + c);
+    uint2 o;
+    __nv_bfloat162 a = __floats2bfloat162_rn(v.x * inv * gg.x, v.y * inv * gg.y);
+    __nv_bfloat162 b = __floats2bfloat162_rn(v.z * inv * gg.z, v.w * inv * gg.w);
+    o.x = *reinterpret_cast<uint32_t*>(&a);
+    o.y = *reinterpret_cast<uint32_t*>(&b);
+    *reinterpret_cast<uint2*>(yr + c) = o;
+  }
+}
+
+// One CTA per token.  Work unit = one (head, i) rotation pair, i < D/2 (rotate-half convention):
+//   x'[i] = x[i] cos - x[i+D/2] sin ;  x'[i+D/2] = x[i+D/2] cos + x[i] sin
+__global__ void rope_kv_kernel(__nv_bfloat16* qkv, int Hq, int Hkv, int D, const float2* __restrict__ cs,
+                               const int32_t* __restrict__ slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int bs) {
+  const int t = blockIdx.x;
+  const int half = D / 2;
+  const int ld = (Hq + 2 * Hkv) * D;
+  __nv_bfloat16* row = qkv + (int64_t)t * ld;
+  const float2* c = cs + (int64_t)t * half;
+  const int slot = slots[t];
+  const int64_t blk = slot / bs, off = slot % bs;
+  const int nq = Hq * half, nk = Hkv * half;
+  for (int u = threadIdx.x; u < nq + nk; u += blockDim.x) {
+    const bool is_k = u >= nq;
+    const int uu = is_k ? u - nq : u;
+    const int h = uu / half, i = uu % half;
+    __nv_bfloat16* base = row + (is_k ? Hq * D : 0) + h * D;
+    const float x1 = __bfloat162float(base[i]), x2 = __bfloat162float(base[i + half]);
+    const float2 r = c[i];
+    const float y1 = x1 * r.x - x2 * r.y, y2 = x2 * r.x + x1 * r.y;
+    if (!is_k) {
+      base[i] = __float2bfloat16_rn(y1);
+      base[i + half] = __float2bfloat16_rn(y2);
+    } else {
+      __nv_bfloat16* dst = kc + ((blk * Hkv + h) * bs + off) * D;
+      dst[i] = __float2bfloat16_rn(y1);
+      dst[i + half] = __float2bfloat16_rn(y2);
+    }
+  }
+  const __nv_bfloat16* vrow = row + (Hq + Hkv) * D;
+  for (int u = threadIdx.x; u < Hkv * D / 8; u += blockDim.x) {
+    const int h = (u * 8) / D, d = (u * 8) % D;
+    *reinterpret_cast<uint4*>(vc + ((blk * Hkv + h) * bs + off) * D + d) =
+        *reinterpret_cast<const uint4*>(vrow + h * D + d);
+  }
+}
+
+__global__ void argmax_reduce_kernel(const float* __restrict__ pv, const int32_t* __restrict__ pi, int rows,
+                                     int ntiles, int32_t* out) {
+  const int r = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  const int l = threadIdx.x & 31;
+  if (r >= rows) return;
+  float best = -INFINITY;
+  int bi = 0x7fffffff;
+  for (int j = l; j < ntiles; j += 32) {
+    const float v = pv[(int64_t)r * ntiles + j];
+    const int i = pi[(int64_t)r * ntiles + j];
+    if (v > best || (v == best && i < bi)) {
+      best = v;
+      bi = i;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const float v2 = __shfl_xor_sync(0xffffffffu, best, o);
+    const int i2 = __shfl_xor_sync(0xffffffffu, bi, o);
+    if (v2 > best || (v2 == best && i2 < bi)) {
+      best = v2;
+      bi = i2;
+    }
+  }
+  if (l == 0) out[r] = bi;
+}
+
+int grid_for(int64_t n, int threads) {
+  int64_t g = (n + threads - 1) / threads;
+  return (int)(g < 148 * 32 ? (g < 1 ? 1 : g) : 148 * 32);
+}
+
+}  // namespace
+
+void launch_init_bf16(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid, float scale,
+                      int mode, int64_t row_offset, cudaStream_t s) {
+  init_bf16_kernel<<<grid_for(rows * cols, 256), 256, 0, s>>>(dst, rows, cols, seed, tid, scale, mode, row_offset);
+}
+void launch_init_f32(float* dst, int64_t n, uint64_t seed, uint64_t tid, float scale, cudaStream_t s) {
+  init_f32_kernel<<<grid_for(n, 256), 256, 0, s>>>(dst, n, seed, tid, scale);
+}
+void launch_fill_f32(float* dst, int64_t n, float v, cudaStream_t s) {
+  fill_f32_kernel<<<grid_for(n, 256), 256, 0, s>>>(dst, n, v);
+}
+void launch_fill_kv(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, uint64_t seed, uint64_t tid, cudaStream_t s) {
+  fill_kv_kernel<<<grid_for(n, 256), 256, 0, s>>>(kc, vc, n, seed, tid);
+}
+void launch_prep(const int32_t* positions, const int32_t* cu_q, const int32_t* block_table, int T, int S,
+                 int maxblk, int block_size, int32_t* slots, float2* rope_cs, int head_dim, float rope_theta,
+                 cudaStream_t s) {
+  if (T <= 0) return;
+  prep_kernel<<<T, 64, 0, s>>>(positions, cu_q, block_table, T, S, maxblk, block_size, slots, rope_cs,
+                               head_dim / 2, log2((double)rope_theta));
+}
+void launch_embed(const __nv_bfloat16* E, const int32_t* ids, float* x, int T, int H, cudaStream_t s) {
+  if (T <= 0) return;
+  embed_kernel<<<T, 128, 0, s>>>(E, ids, x, H);
+}
+void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int32_t* rows, int n, int H, float eps,
+                    cudaStream_t s) {
+  if (n <= 0) return;
+  rmsnorm_kernel<<<n, 256, 0, s>>>(x, g, y, rows, H, eps);
+}
+void launch_rope_kv_append(__nv_bfloat16* qkv, int T, int Hq, int Hkv, int D, const float2* rope_cs,
+                           const int32_t* slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int block_size,
+                           cudaStream_t s) {
+  if (T <= 0) return;
+  rope_kv_kernel<<<T, 256, 0, s>>>(qkv, Hq, Hkv, D, rope_cs, slots, kc, vc, block_size);
+}
+void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,
+                          cudaStream_t s) {
+  if (rows <= 0) return;
+  argmax_reduce_kernel<<<(rows + 3) / 4, 128, 0, s>>>(part_val, part_idx, rows, ntiles, out);
+}
+
+}  // namespace gllm

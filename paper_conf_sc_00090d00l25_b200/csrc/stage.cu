@@ -1,0 +1,752 @@
+// gllm_stage: one pipeline stage's layers on one B200 (P1) and
+// the per-stage forward over one Token-Throttled mixed batch (steps a2-a12).
+//
+// Per forward (all on the caller's stream, nothing synchronises with the host):
+//   host: validate + pack the batch metadata and the attention work lists into a pinned
+//         ring slot (input prep), one H2D copy
+//   prep (slot mapping O2 + RoPE table) -> [stage 0: embedding] -> per layer:
+//     RMSNorm -> QKV GEMM(+bias) -> RoPE + KV append -> prefill attention | decode attention
+//     -> O GEMM (+= residual) -> RMSNorm -> gate_up GEMM (SiLU*up) -> down GEMM (+= residual)
+//   [last stage: final RMSNorm on sampled rows -> LM-head GEMM with argmax epilogue -> reduce]
+#include <cuda_bf16.h>
+#include <nccl.h>
+
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "attention.cuh"
+#include "common.h"
+#include "gemm.cuh"
+#include "kernels.cuh"
+
+using bf16 = __nv_bfloat16;
+
+namespace {
+
+#define CK(expr)                                                                                   \
+  do {                                                                                             \
+    cudaError_t e__ = (expr);                                                                      \
+    if (e__ != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "%s: %s", #expr, cudaGetErrorString(e__)); \
+  } while (0)
+#define RC(expr)            \
+  do {                      \
+    int r__ = (expr);       \
+    if (r__ < 0) return r__; \
+  } while (0)
+
+constexpr uint64_t T_EMBED = 0xFFFFF0ull, T_LMHEAD = 0xFFFFF1ull;
+enum Kind { K_WQ = 0, K_WK, K_WV, K_WO, K_WG, K_WU, K_WD, K_BQ, K_BK, K_BV };
+inline uint64_t layer_tid(int l, int kind) { return 1 + 16 * (uint64_t)l + kind; }
+
+// profiling categories (gllm_stage_last_timing)
+enum Cat { C_TOTAL = 0, C_QKV, C_O, C_GU, C_DOWN, C_PREFILL, C_DECODE, C_ROPE, C_NORM, C_LMHEAD, C_OTHER, C_N };
+
+struct LayerW {
+  bf16 *wqkv = nullptr, *wo = nullptr, *wgu = nullptr, *wd = nullptr;
+  float *bqkv = nullptr, *g1 = nullptr, *g2 = nullptr;
+  bf16 *kc = nullptr, *vc = nullptr;
+  CUtensorMap tm_qkv, tm_o, tm_gu, tm_d;
+};
+
+constexpr int RING = 4;
+
+// NCCL is resolved lazily with dlopen at the first communicator call, so the library never
+// drags its own libnccl.so.2 into a process ahead of torch's (same soname, different version).
+struct NcclApi {
+  decltype(&ncclGetUniqueId) get_unique_id = nullptr;
+  decltype(&ncclCommInitRank) comm_init_rank = nullptr;
+  decltype(&ncclCommDestroy) comm_destroy = nullptr;
+  decltype(&ncclSend) send = nullptr;
+  decltype(&ncclRecv) recv = nullptr;
+  decltype(&ncclGetErrorString) error_string = nullptr;
+  bool ok = false;
+};
+NcclApi& nccl() {
+  static NcclApi api = [] {
+    NcclApi a;
+    void* h = nullptr;
+    if (const char* p = std::getenv("GLLM_NCCL_PATH")) h = dlopen(p, RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);  // torch's, if loaded
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return a;
+    a.get_unique_id = reinterpret_cast<decltype(a.get_unique_id)>(dlsym(h, "ncclGetUniqueId"));
+    a.comm_init_rank = reinterpret_cast<decltype(a.comm_init_rank)>(dlsym(h, "ncclCommInitRank"));
+    a.comm_destroy = reinterpret_cast<decltype(a.comm_destroy)>(dlsym(h, "ncclCommDestroy"));
+    a.send = reinterpret_cast<decltype(a.send)>(dlsym(h, "ncclSend"));
+    a.recv = reinterpret_cast<decltype(a.recv)>(dlsym(h, "ncclRecv"));
+    a.error_string = reinterpret_cast<decltype(a.error_string)>(dlsym(h, "ncclGetErrorString"));
+    a.ok = a.get_unique_id && a.comm_init_rank && a.comm_destroy && a.send && a.recv && a.error_string;
+    return a;
+  }();
+  return api;
+}
+
+size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
+
+}  // namespace
+
+struct gllm_stage {
+  gllm_model_cfg cfg{};
+  int lb = 0, le = 0, kv_blocks = 0, bs = 16, max_tokens = 0, max_seqs = 0, device = 0, num_sms = 148;
+  int rows_alloc = 0, seqs_alloc = 0;
+  std::vector<LayerW> layers;
+  bf16* embed = nullptr;
+  bf16* lm_head = nullptr;
+  float* final_norm = nullptr;
+  CUtensorMap tm_lm;
+  float* xbuf = nullptr;
+  bf16 *y = nullptr, *qkv = nullptr, *attn = nullptr, *act = nullptr, *ys = nullptr;
+  CUtensorMap tm_y, tm_attn, tm_act, tm_ys;
+  float2* rope_cs = nullptr;
+  int32_t* slots = nullptr;
+  int32_t* sampled_tmp = nullptr;
+  float* part_val = nullptr;
+  int32_t* part_idx = nullptr;
+  float *part_o = nullptr, *part_ml = nullptr;
+  int parts_cap = 0;
+  uint8_t* pinned[RING] = {};
+  uint8_t* meta_dev[RING] = {};
+  size_t meta_cap = 0;
+  cudaEvent_t ring_ev[RING] = {};
+  int ring_i = 0;
+  std::vector<void*> allocs;
+  ncclComm_t comm = nullptr;
+  int last_T = 0, last_launches = 0;
+  bool profiling = false;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> prof_ev;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  float last_timing[C_N] = {};
+  bool timing_pending = false;
+
+  bool is_first() const { return lb == 0; }
+  bool is_last() const { return le == cfg.n_layers; }
+  int qd() const { return cfg.n_heads * cfg.head_dim; }
+  int kd() const { return cfg.n_kv_heads * cfg.head_dim; }
+
+  template <class T>
+  int dalloc(T** p, size_t n) {
+    void* q = nullptr;
+    cudaError_t e = cudaMalloc(&q, std::max<size_t>(n, 1) * sizeof(T));
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return gllm::set_error(GLLM_ENOMEM, "cudaMalloc(%zu bytes): %s", n * sizeof(T), cudaGetErrorString(e));
+    }
+    allocs.push_back(q);
+    *p = static_cast<T*>(q);
+    return GLLM_OK;
+  }
+  cudaEvent_t next_ev() {
+    if (ev_used == ev_pool.size()) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      ev_pool.push_back(e);
+    }
+    return ev_pool[ev_used++];
+  }
+};
+
+namespace {
+
+struct Prof {
+  gllm_stage* st;
+  cudaStream_t s;
+  int cat;
+  cudaEvent_t a{};
+  Prof(gllm_stage* st_, cudaStream_t s_, int cat_) : st(st_), s(s_), cat(cat_) {
+    if (st->profiling) {
+      a = st->next_ev();
+      cudaEventRecord(a, s);
+    }
+  }
+  ~Prof() {
+    if (st->profiling) {
+      cudaEvent_t b = st->next_ev();
+      cudaEventRecord(b, s);
+      st->prof_ev.push_back({cat, {a, b}});
+    }
+  }
+};
+
+int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmEpi epi, int M, int N, int K,
+         void* out, int ldo, const float* bias, cudaStream_t s) {
+  gllm::GemmArgs g{};
+  g.M = M;
+  g.N = N;
+  g.K = K;
+  g.out = out;
+  g.ldo = ldo;
+  g.bias = bias;
+  g.part_val = st->part_val;
+  g.part_idx = st->part_idx;
+  st->last_launches += 1;
+  return gllm::launch_gemm(a, b, epi, g, s, st->num_sms);
+}
+
+int check_model(const gllm_model_cfg* c) {
+  if (!c) return gllm::set_error(GLLM_EINVAL, "null model cfg");
+  if (c->n_layers < 1 || c->hidden < 256 || c->n_heads < 1 || c->n_kv_heads < 1 || c->vocab < 256)
+    return gllm::set_error(GLLM_EINVAL, "model cfg: bad sizes");
+  if (c->head_dim != 64 && c->head_dim != 128) return gllm::set_error(GLLM_EINVAL, "head_dim must be 64 or 128");
+  if (c->n_heads % c->n_kv_heads) return gllm::set_error(GLLM_EINVAL, "n_heads %% n_kv_heads != 0");
+  const int g = c->n_heads / c->n_kv_heads;
+  if (g != 1 && g != 2 && g != 4 && g != 5 && g != 8) return gllm::set_error(GLLM_EINVAL, "GQA group %d unsupported", g);
+  if (c->hidden % 256) return gllm::set_error(GLLM_EINVAL, "hidden %% 256 != 0");
+  if (c->intermediate % 128) return gllm::set_error(GLLM_EINVAL, "intermediate %% 128 != 0");
+  if ((c->n_heads * c->head_dim) % 64 || ((c->n_heads + 2 * c->n_kv_heads) * c->head_dim) % 32)
+    return gllm::set_error(GLLM_EINVAL, "q/kv dims must be multiples of 64");
+  if (!(c->rms_eps > 0) || !(c->rope_theta > 1)) return gllm::set_error(GLLM_EINVAL, "bad eps/theta");
+  return GLLM_OK;
+}
+
+void destroy(gllm_stage* st) {
+  if (!st) return;
+  cudaSetDevice(st->device);
+  cudaDeviceSynchronize();
+  for (void* p : st->allocs) cudaFree(p);
+  for (int i = 0; i < RING; ++i) {
+    if (st->pinned[i]) cudaFreeHost(st->pinned[i]);
+    if (st->meta_dev[i]) cudaFree(st->meta_dev[i]);
+    if (st->ring_ev[i]) cudaEventDestroy(st->ring_ev[i]);
+  }
+  for (auto e : st->ev_pool) cudaEventDestroy(e);
+  if (st->comm && nccl().ok) nccl().comm_destroy(st->comm);
+  cudaGetLastError();
+  delete st;
+}
+
+int ensure_meta(gllm_stage* st, size_t bytes) {
+  if (bytes <= st->meta_cap) return GLLM_OK;
+  size_t cap = std::max<size_t>(bytes * 2, 1 << 20);
+  for (int i = 0; i < RING; ++i) {
+    if (st->ring_ev[i]) CK(cudaEventSynchronize(st->ring_ev[i]));
+  }
+  CK(cudaDeviceSynchronize());
+  for (int i = 0; i < RING; ++i) {
+    if (st->pinned[i]) cudaFreeHost(st->pinned[i]);
+    if (st->meta_dev[i]) cudaFree(st->meta_dev[i]);
+    st->pinned[i] = nullptr;
+    st->meta_dev[i] = nullptr;
+    CK(cudaMallocHost(&st->pinned[i], cap));
+    CK(cudaMalloc(&st->meta_dev[i], cap));
+  }
+  st->meta_cap = cap;
+  return GLLM_OK;
+}
+
+int ensure_parts(gllm_stage* st, int parts) {
+  if (parts <= st->parts_cap) return GLLM_OK;
+  CK(cudaDeviceSynchronize());
+  const int cap = std::max(parts * 2, 1024);
+  const size_t G = st->cfg.n_heads / st->cfg.n_kv_heads;
+  float *po = nullptr, *pm = nullptr;
+  CK(cudaMalloc(&po, (size_t)cap * st->cfg.n_kv_heads * G * st->cfg.head_dim * sizeof(float)));
+  CK(cudaMalloc(&pm, (size_t)cap * st->cfg.n_kv_heads * G * 2 * sizeof(float)));
+  if (st->part_o) cudaFree(st->part_o);
+  if (st->part_ml) cudaFree(st->part_ml);
+  st->part_o = po;
+  st->part_ml = pm;
+  st->parts_cap = cap;
+  return GLLM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t layer_end, int32_t kv_blocks,
+                    int32_t block_size, int32_t max_tokens, int32_t max_seqs, int32_t device, gllm_stage** out) {
+  GLLM_TRY_BEGIN
+  RC(check_model(cfg));
+  if (!out) return gllm::set_error(GLLM_EINVAL, "null out");
+  if (layer_begin < 0 || layer_end > cfg->n_layers || layer_begin >= layer_end)
+    return gllm::set_error(GLLM_EINVAL, "bad layer range [%d, %d)", layer_begin, layer_end);
+  if (block_size != 16) return gllm::set_error(GLLM_EINVAL, "block_size must be 16");
+  if (kv_blocks < 1 || max_tokens < 1 || max_seqs < 1 || max_seqs > max_tokens)
+    return gllm::set_error(GLLM_EINVAL, "bad kv_blocks/max_tokens/max_seqs");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return gllm::set_error(GLLM_ECUDA, "no CUDA device %d", device);
+  }
+  CK(cudaSetDevice(device));
+  auto* st = new gllm_stage();
+  st->cfg = *cfg;
+  st->lb = layer_begin;
+  st->le = layer_end;
+  st->kv_blocks = kv_blocks;
+  st->bs = block_size;
+  st->max_tokens = max_tokens;
+  st->max_seqs = max_seqs;
+  st->device = device;
+  st->num_sms = gllm::num_sms_of_current_device();
+  st->rows_alloc = std::max(128, (max_tokens + 127) / 128 * 128);
+  st->seqs_alloc = std::max(128, (max_seqs + 127) / 128 * 128);
+  auto fail = [&](int rc) {
+    destroy(st);
+    return rc;
+  };
+  const int H = cfg->hidden, D = cfg->head_dim, Hkv = cfg->n_kv_heads, I = cfg->intermediate, V = cfg->vocab;
+  const int qd = st->qd(), kd = st->kd(), nqkv = qd + 2 * kd;
+  const uint64_t seed = cfg->weight_seed;
+  const float s_h = (float)std::sqrt(3.0 / H), s_q = (float)std::sqrt(3.0 / qd), s_i = (float)std::sqrt(3.0 / I);
+  const float s_bias = (float)(std::sqrt(3.0) * 0.02), s_emb = (float)std::sqrt(3.0);
+  cudaStream_t s0 = 0;
+  const size_t kv_elems = (size_t)kv_blocks * Hkv * block_size * D;
+  int rc;
+  for (int l = layer_begin; l < layer_end; ++l) {
+    LayerW w;
+    if ((rc = st->dalloc(&w.wqkv, (size_t)nqkv * H)) || (rc = st->dalloc(&w.wo, (size_t)H * qd)) ||
+        (rc = st->dalloc(&w.wgu, (size_t)2 * I * H)) || (rc = st->dalloc(&w.wd, (size_t)H * I)) ||
+        (rc = st->dalloc(&w.g1, H)) || (rc = st->dalloc(&w.g2, H)) || (rc = st->dalloc(&w.kc, kv_elems)) ||
+        (rc = st->dalloc(&w.vc, kv_elems)))
+      return fail(rc);
+    if (cfg->qkv_bias && (rc = st->dalloc(&w.bqkv, nqkv))) return fail(rc);
+    gllm::launch_init_bf16(w.wqkv, qd, H, seed, layer_tid(l, K_WQ), s_h, 0, 0, s0);
+    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WK), s_h, 0, qd, s0);
+    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WV), s_h, 0, qd + kd, s0);
+    gllm::launch_init_bf16(w.wo, H, qd, seed, layer_tid(l, K_WO), s_q, 0, 0, s0);
+    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WG), s_h, 1, 0, s0);
+    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WU), s_h, 2, 0, s0);
+    gllm::launch_init_bf16(w.wd, H, I, seed, layer_tid(l, K_WD), s_i, 0, 0, s0);
+    gllm::launch_fill_f32(w.g1, H, 1.0f, s0);
+    gllm::launch_fill_f32(w.g2, H, 1.0f, s0);
+    if (w.bqkv) {
+      gllm::launch_init_f32(w.bqkv, qd, seed, layer_tid(l, K_BQ), s_bias, s0);
+      gllm::launch_init_f32(w.bqkv + qd, kd, seed, layer_tid(l, K_BK), s_bias, s0);
+      gllm::launch_init_f32(w.bqkv + qd + kd, kd, seed, layer_tid(l, K_BV), s_bias, s0);
+    }
+    CK(cudaMemsetAsync(w.kc, 0, kv_elems * sizeof(bf16), s0));
+    CK(cudaMemsetAsync(w.vc, 0, kv_elems * sizeof(bf16), s0));
+    if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_BN)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_BN)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_BN)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_BN)))
+      return fail(rc);
+    st->layers.push_back(w);
+  }
+  if (st->is_first()) {
+    if ((rc = st->dalloc(&st->embed, (size_t)V * H))) return fail(rc);
+    gllm::launch_init_bf16(st->embed, V, H, seed, T_EMBED, s_emb, 0, 0, s0);
+  }
+  if (st->is_last()) {
+    if ((rc = st->dalloc(&st->lm_head, (size_t)V * H)) || (rc = st->dalloc(&st->final_norm, H))) return fail(rc);
+    gllm::launch_init_bf16(st->lm_head, V, H, seed, T_LMHEAD, s_h, 0, 0, s0);
+    gllm::launch_fill_f32(st->final_norm, H, 1.0f, s0);
+    if ((rc = gllm::make_tmap_bf16(&st->tm_lm, st->lm_head, V, H, gllm::GEMM_BN))) return fail(rc);
+    const int ntn = (V + gllm::GEMM_BN - 1) / gllm::GEMM_BN;
+    if ((rc = st->dalloc(&st->ys, (size_t)st->seqs_alloc * H)) ||
+        (rc = st->dalloc(&st->part_val, (size_t)st->seqs_alloc * ntn)) ||
+        (rc = st->dalloc(&st->part_idx, (size_t)st->seqs_alloc * ntn)) ||
+        (rc = st->dalloc(&st->sampled_tmp, st->seqs_alloc)))
+      return fail(rc);
+    if ((rc = gllm::make_tmap_bf16(&st->tm_ys, st->ys, st->seqs_alloc, H, gllm::GEMM_BM))) return fail(rc);
+  }
+  const size_t R = st->rows_alloc;
+  if ((rc = st->dalloc(&st->xbuf, R * H)) || (rc = st->dalloc(&st->y, R * H)) ||
+      (rc = st->dalloc(&st->qkv, R * nqkv)) || (rc = st->dalloc(&st->attn, R * qd)) ||
+      (rc = st->dalloc(&st->act, R * I)) || (rc = st->dalloc(&st->rope_cs, R * (D / 2))) ||
+      (rc = st->dalloc(&st->slots, R)))
+    return fail(rc);
+  CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
+  CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
+  CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
+  if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
+      (rc = gllm::make_tmap_bf16(&st->tm_attn, st->attn, R, qd, gllm::GEMM_BM)) ||
+      (rc = gllm::make_tmap_bf16(&st->tm_act, st->act, R, I, gllm::GEMM_BM)))
+    return fail(rc);
+  for (int i = 0; i < RING; ++i) {
+    cudaError_t e = cudaEventCreateWithFlags(&st->ring_ev[i], cudaEventDisableTiming);
+    if (e != cudaSuccess) return fail(gllm::set_error(GLLM_ECUDA, "event: %s", cudaGetErrorString(e)));
+  }
+  if ((rc = ensure_meta(st, 1 << 20)) < 0) return fail(rc);
+  if ((rc = ensure_parts(st, 1024)) < 0) return fail(rc);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return fail(gllm::set_error(GLLM_ECUDA, "init: %s", cudaGetErrorString(e)));
+  *out = st;
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_free_stage(gllm_stage* st) {
+  destroy(st);
+  return GLLM_OK;
+}
+
+int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hidden_in, void* hidden_out,
+                       int32_t* sampled_out, void* stream) {
+  GLLM_TRY_BEGIN
+  if (!st || !d) return gllm::set_error(GLLM_EINVAL, "null argument");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const gllm_model_cfg& c = st->cfg;
+  const int T = d->num_tokens, S = d->num_seqs, NP = d->num_prefill_seqs, maxblk = d->max_blocks_per_seq;
+  const int ns = d->num_samples;
+  const int bs = st->bs;
+  // ---------------- validation (EINVAL, never UB)
+  if (T < 0 || T > st->max_tokens) return gllm::set_error(GLLM_EINVAL, "num_tokens %d > max_tokens %d", T, st->max_tokens);
+  if (S < 0 || S > st->max_seqs) return gllm::set_error(GLLM_EINVAL, "num_seqs %d > max_seqs %d", S, st->max_seqs);
+  if (NP < 0 || NP > S || ns < 0 || ns > S || maxblk < 0) return gllm::set_error(GLLM_EINVAL, "bad batch counts");
+  if (T == 0) {
+    st->last_T = 0;
+    st->last_launches = 0;
+    return GLLM_OK;
+  }
+  if (!d->token_ids || !d->positions || !d->cu_q || !d->kv_len || !d->block_table || (ns && !d->sample_token_idx))
+    return gllm::set_error(GLLM_EINVAL, "null batch array");
+  if (!st->is_first() && !hidden_in) return gllm::set_error(GLLM_EINVAL, "hidden_in required on stage > 0");
+  if (!st->is_last() && !hidden_out) return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
+  if (d->cu_q[0] != 0 || d->cu_q[S] != T) return gllm::set_error(GLLM_EINVAL, "cu_q must span [0, num_tokens]");
+  const int G = c.n_heads / c.n_kv_heads;
+  int64_t total_pages = 0;
+  for (int i = 0; i < S; ++i) {
+    const int q0 = d->cu_q[i], q1 = d->cu_q[i + 1], L = d->kv_len[i], n = q1 - q0;
+    if (n < 1 || (i >= NP && n != 1)) return gllm::set_error(GLLM_EINVAL, "seq %d: bad token count %d", i, n);
+    if (L < n || (int64_t)(L + bs - 1) / bs > maxblk) return gllm::set_error(GLLM_EINVAL, "seq %d: bad kv_len %d", i, L);
+    for (int j = 0; j < n; ++j)
+      if (d->positions[q0 + j] != L - n + j) return gllm::set_error(GLLM_EINVAL, "seq %d: positions must be kv_len-n..kv_len-1", i);
+    const int nb = (L + bs - 1) / bs;
+    for (int j = 0; j < nb; ++j) {
+      const int b = d->block_table[(size_t)i * maxblk + j];
+      if (b < 0 || b >= st->kv_blocks) return gllm::set_error(GLLM_EINVAL, "seq %d: block id %d out of range", i, b);
+    }
+    if (i >= NP) total_pages += nb;
+  }
+  for (int t = 0; t < T; ++t)
+    if (d->token_ids[t] < 0 || d->token_ids[t] >= c.vocab) return gllm::set_error(GLLM_EINVAL, "token id out of range");
+  for (int k = 0; k < ns; ++k)
+    if (d->sample_token_idx[k] < 0 || d->sample_token_idx[k] >= T) return gllm::set_error(GLLM_EINVAL, "bad sample idx");
+  // ---------------- attention work lists (host, O(S))
+  std::vector<gllm::PrefillItem> pitems;
+  for (int i = 0; i < NP; ++i) {
+    const int rows = (d->cu_q[i + 1] - d->cu_q[i]) * G;
+    for (int r0 = 0; r0 < rows; r0 += 64) pitems.push_back({i, r0});
+  }
+  const int ND = S - NP;
+  int split_pages = 1 << 30;
+  if (ND > 0) {
+    const int64_t target = 4LL * st->num_sms;  // CTAs
+    int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
+    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(8, per));
+  }
+  std::vector<gllm::DecodeItem> ditems;
+  std::vector<gllm::MergeItem> merges;
+  int nparts = 0;
+  for (int i = NP; i < S; ++i) {
+    const int nb = (d->kv_len[i] + bs - 1) / bs;
+    const int nsplit = (nb + split_pages - 1) / split_pages;
+    if (nsplit == 1) {
+      ditems.push_back({i, 0, -1, 1});
+    } else {
+      merges.push_back({i, nparts, nsplit, 0});
+      for (int k = 0; k < nsplit; ++k) ditems.push_back({i, k, nparts + k, nsplit});
+      nparts += nsplit;
+    }
+  }
+  RC(ensure_parts(st, nparts));
+  // ---------------- pack metadata into a pinned ring slot; one H2D copy (K9)
+  size_t off = 0;
+  auto sect = [&](size_t bytes) {
+    size_t o = off;
+    off = align16(off + bytes);
+    return o;
+  };
+  const size_t o_ids = sect(T * 4), o_pos = sect(T * 4), o_cu = sect((S + 1) * 4), o_kvl = sect(S * 4),
+               o_bt = sect((size_t)S * maxblk * 4), o_samp = sect(ns * 4),
+               o_pi = sect(pitems.size() * sizeof(gllm::PrefillItem)),
+               o_di = sect(ditems.size() * sizeof(gllm::DecodeItem)),
+               o_mi = sect(merges.size() * sizeof(gllm::MergeItem));
+  RC(ensure_meta(st, off));
+  CK(cudaSetDevice(st->device));
+  const int slot = st->ring_i;
+  st->ring_i = (st->ring_i + 1) % RING;
+  CK(cudaEventSynchronize(st->ring_ev[slot]));  // previous use of this slot has been copied
+  uint8_t* h = st->pinned[slot];
+  std::memcpy(h + o_ids, d->token_ids, T * 4);
+  std::memcpy(h + o_pos, d->positions, T * 4);
+  std::memcpy(h + o_cu, d->cu_q, (S + 1) * 4);
+  std::memcpy(h + o_kvl, d->kv_len, S * 4);
+  std::memcpy(h + o_bt, d->block_table, (size_t)S * maxblk * 4);
+  if (ns) std::memcpy(h + o_samp, d->sample_token_idx, ns * 4);
+  if (!pitems.empty()) std::memcpy(h + o_pi, pitems.data(), pitems.size() * sizeof(gllm::PrefillItem));
+  if (!ditems.empty()) std::memcpy(h + o_di, ditems.data(), ditems.size() * sizeof(gllm::DecodeItem));
+  if (!merges.empty()) std::memcpy(h + o_mi, merges.data(), merges.size() * sizeof(gllm::MergeItem));
+  uint8_t* m = st->meta_dev[slot];
+  if (st->timing_pending) st->timing_pending = false;
+  st->prof_ev.clear();
+  st->ev_used = 0;
+  st->last_launches = 0;
+  Prof p_total(st, s, C_TOTAL);
+  CK(cudaMemcpyAsync(m, h, off, cudaMemcpyHostToDevice, s));
+  CK(cudaEventRecord(st->ring_ev[slot], s));
+  const int32_t* d_ids = reinterpret_cast<const int32_t*>(m + o_ids);
+  const int32_t* d_pos = reinterpret_cast<const int32_t*>(m + o_pos);
+  const int32_t* d_cu = reinterpret_cast<const int32_t*>(m + o_cu);
+  const int32_t* d_kvl = reinterpret_cast<const int32_t*>(m + o_kvl);
+  const int32_t* d_bt = reinterpret_cast<const int32_t*>(m + o_bt);
+  const int32_t* d_samp = reinterpret_cast<const int32_t*>(m + o_samp);
+  const auto* d_pi = reinterpret_cast<const gllm::PrefillItem*>(m + o_pi);
+  const auto* d_di = reinterpret_cast<const gllm::DecodeItem*>(m + o_di);
+  const auto* d_mi = reinterpret_cast<const gllm::MergeItem*>(m + o_mi);
+
+  const int H = c.hidden, D = c.head_dim, qd = st->qd(), kd = st->kd(), nqkv = qd + 2 * kd, I = c.intermediate;
+  {
+    Prof p(st, s, C_OTHER);
+    gllm::launch_prep(d_pos, d_cu, d_bt, T, S, maxblk, bs, st->slots, st->rope_cs, D, c.rope_theta, s);
+    st->last_launches += 1;
+  }
+  float* x = hidden_out ? static_cast<float*>(hidden_out) : st->xbuf;
+  if (st->is_first()) {
+    Prof p(st, s, C_OTHER);
+    gllm::launch_embed(st->embed, d_ids, x, T, H, s);
+    st->last_launches += 1;
+  } else if (hidden_in != x) {
+    CK(cudaMemcpyAsync(x, hidden_in, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
+  }
+  gllm::AttnArgs aa{};
+  aa.q = st->qkv;
+  aa.q_stride = nqkv;
+  aa.Hq = c.n_heads;
+  aa.Hkv = c.n_kv_heads;
+  aa.D = D;
+  aa.bs = bs;
+  aa.cu_q = d_cu;
+  aa.kv_len = d_kvl;
+  aa.block_table = d_bt;
+  aa.maxblk = maxblk;
+  aa.out = st->attn;
+  aa.part_o = st->part_o;
+  aa.part_ml = st->part_ml;
+  aa.split_len = split_pages * bs;
+  for (size_t li = 0; li < st->layers.size(); ++li) {
+    LayerW& w = st->layers[li];
+    {
+      Prof p(st, s, C_NORM);
+      gllm::launch_rmsnorm(x, w.g1, st->y, nullptr, T, H, c.rms_eps, s);
+      st->last_launches += 1;
+    }
+    {
+      Prof p(st, s, C_QKV);
+      RC(gemm(st, st->tm_y, w.tm_qkv, gllm::EPI_STORE_BF16, T, nqkv, H, st->qkv, nqkv, w.bqkv, s));
+    }
+    {
+      Prof p(st, s, C_ROPE);
+      gllm::launch_rope_kv_append(st->qkv, T, c.n_heads, c.n_kv_heads, D, st->rope_cs, st->slots, w.kc, w.vc, bs, s);
+      st->last_launches += 1;
+    }
+    aa.kc = w.kc;
+    aa.vc = w.vc;
+    if (!pitems.empty()) {
+      Prof p(st, s, C_PREFILL);
+      RC(gllm::launch_prefill_attention(aa, d_pi, (int)pitems.size(), s));
+      st->last_launches += 1;
+    }
+    if (!ditems.empty()) {
+      Prof p(st, s, C_DECODE);
+      RC(gllm::launch_decode_attention(aa, d_di, (int)ditems.size(), d_mi, (int)merges.size(), s));
+      st->last_launches += merges.empty() ? 1 : 2;
+    }
+    {
+      Prof p(st, s, C_O);
+      RC(gemm(st, st->tm_attn, w.tm_o, gllm::EPI_ADD_F32, T, H, qd, x, H, nullptr, s));
+    }
+    {
+      Prof p(st, s, C_NORM);
+      gllm::launch_rmsnorm(x, w.g2, st->y, nullptr, T, H, c.rms_eps, s);
+      st->last_launches += 1;
+    }
+    {
+      Prof p(st, s, C_GU);
+      RC(gemm(st, st->tm_y, w.tm_gu, gllm::EPI_SILU_MUL, T, 2 * I, H, st->act, I, nullptr, s));
+    }
+    {
+      Prof p(st, s, C_DOWN);
+      RC(gemm(st, st->tm_act, w.tm_d, gllm::EPI_ADD_F32, T, H, I, x, H, nullptr, s));
+    }
+  }
+  if (st->is_last() && ns > 0) {
+    Prof p(st, s, C_LMHEAD);
+    gllm::launch_rmsnorm(x, st->final_norm, st->ys, d_samp, ns, H, c.rms_eps, s);
+    RC(gemm(st, st->tm_ys, st->tm_lm, gllm::EPI_ARGMAX, ns, c.vocab, H, nullptr, 0, nullptr, s));
+    const int ntn = (c.vocab + gllm::GEMM_BN - 1) / gllm::GEMM_BN;
+    gllm::launch_argmax_reduce(st->part_val, st->part_idx, ns, ntn, sampled_out ? sampled_out : st->sampled_tmp, s);
+    st->last_launches += 2;
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "stage_forward launch: %s", cudaGetErrorString(e));
+  st->last_T = T;
+  st->timing_pending = st->profiling;
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_stage_sync(gllm_stage* st) {
+  if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
+  cudaSetDevice(st->device);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "device: %s", cudaGetErrorString(e));
+  return GLLM_OK;
+}
+
+int gllm_stage_set_profiling(gllm_stage* st, int32_t on) {
+  if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
+  st->profiling = on != 0;
+  return GLLM_OK;
+}
+
+int gllm_stage_last_timing(gllm_stage* st, float* out, int32_t n) {
+  if (!st || !out) return gllm::set_error(GLLM_EINVAL, "null argument");
+  float acc[C_N] = {};
+  for (auto& pe : st->prof_ev) {
+    CK(cudaEventSynchronize(pe.second.second));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, pe.second.first, pe.second.second));
+    acc[pe.first] += ms;
+  }
+  for (int i = 0; i < n && i < C_N; ++i) out[i] = acc[i];
+  return GLLM_OK;
+}
+
+int gllm_stage_last_launches(gllm_stage* st, int32_t* out) {
+  if (!st || !out) return gllm::set_error(GLLM_EINVAL, "null argument");
+  *out = st->last_launches;
+  return GLLM_OK;
+}
+
+// ---------------------------------------------------------------- NCCL hand-off (a12)
+int gllm_get_unique_id(void* out128) {
+  if (!out128) return gllm::set_error(GLLM_EINVAL, "null out");
+  if (!nccl().ok) return gllm::set_error(GLLM_ENCCL, "libnccl.so.2 not found");
+  ncclUniqueId id;
+  ncclResult_t r = nccl().get_unique_id(&id);
+  if (r != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclGetUniqueId: %s", nccl().error_string(r));
+  std::memcpy(out128, &id, sizeof(id));
+  return GLLM_OK;
+}
+
+int gllm_comm_init(gllm_stage* st, const void* uid, int32_t rank, int32_t world) {
+  if (!st || !uid || rank < 0 || rank >= world) return gllm::set_error(GLLM_EINVAL, "bad comm_init arguments");
+  if (!nccl().ok) return gllm::set_error(GLLM_ENCCL, "libnccl.so.2 not found");
+  cudaSetDevice(st->device);
+  ncclUniqueId id;
+  std::memcpy(&id, uid, sizeof(id));
+  ncclResult_t r = nccl().comm_init_rank(&st->comm, world, id, rank);
+  if (r != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclCommInitRank: %s", nccl().error_string(r));
+  return GLLM_OK;
+}
+
+int gllm_send_hidden(gllm_stage* st, const void* buf, int32_t num_tokens, int32_t dst, void* stream) {
+  if (!st || !st->comm || (!buf && num_tokens)) return gllm::set_error(GLLM_ESTATE, "send_hidden: no communicator");
+  if (num_tokens == 0) return GLLM_OK;
+  ncclResult_t r = nccl().send(buf, (size_t)num_tokens * st->cfg.hidden, ncclFloat32, dst, st->comm,
+                            reinterpret_cast<cudaStream_t>(stream));
+  if (r != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclSend: %s", nccl().error_string(r));
+  return GLLM_OK;
+}
+
+int gllm_recv_hidden(gllm_stage* st, void* buf, int32_t num_tokens, int32_t src, void* stream) {
+  if (!st || !st->comm || (!buf && num_tokens)) return gllm::set_error(GLLM_ESTATE, "recv_hidden: no communicator");
+  if (num_tokens == 0) return GLLM_OK;
+  ncclResult_t r = nccl().recv(buf, (size_t)num_tokens * st->cfg.hidden, ncclFloat32, src, st->comm,
+                            reinterpret_cast<cudaStream_t>(stream));
+  if (r != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclRecv: %s", nccl().error_string(r));
+  return GLLM_OK;
+}
+
+// ---------------------------------------------------------------- introspection
+int gllm_stage_read_weight(gllm_stage* st, int32_t layer, const char* name, int64_t row0, int64_t nrows, float* out) {
+  GLLM_TRY_BEGIN
+  if (!st || !name || !out || row0 < 0 || nrows < 0) return gllm::set_error(GLLM_EINVAL, "bad arguments");
+  const gllm_model_cfg& c = st->cfg;
+  const int H = c.hidden, I = c.intermediate, qd = st->qd(), kd = st->kd();
+  const std::string n(name);
+  cudaSetDevice(st->device);
+  std::vector<bf16> row;
+  auto copy_rows = [&](const bf16* base, int64_t rows, int64_t cols, auto phys) -> int {
+    if (row0 + nrows > rows) return gllm::set_error(GLLM_EINVAL, "row range out of bounds");
+    row.resize(cols);
+    for (int64_t r = 0; r < nrows; ++r) {
+      CK(cudaMemcpy(row.data(), base + (size_t)phys(row0 + r) * cols, cols * sizeof(bf16), cudaMemcpyDeviceToHost));
+      for (int64_t j = 0; j < cols; ++j) out[r * cols + j] = __bfloat162float(row[j]);
+    }
+    return GLLM_OK;
+  };
+  auto ident = [](int64_t r) { return r; };
+  if (n == "embed") {
+    if (!st->embed) return gllm::set_error(GLLM_EINVAL, "no embedding on this stage");
+    return copy_rows(st->embed, c.vocab, H, ident);
+  }
+  if (n == "lm_head") {
+    if (!st->lm_head) return gllm::set_error(GLLM_EINVAL, "no LM head on this stage");
+    return copy_rows(st->lm_head, c.vocab, H, ident);
+  }
+  if (layer < st->lb || layer >= st->le) return gllm::set_error(GLLM_EINVAL, "layer %d not on this stage", layer);
+  LayerW& w = st->layers[layer - st->lb];
+  if (n == "wq") return copy_rows(w.wqkv, qd, H, ident);
+  if (n == "wk") return copy_rows(w.wqkv, kd, H, [&](int64_t r) { return qd + r; });
+  if (n == "wv") return copy_rows(w.wqkv, kd, H, [&](int64_t r) { return qd + kd + r; });
+  if (n == "wo") return copy_rows(w.wo, H, qd, ident);
+  if (n == "wg") return copy_rows(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + r % 128; });
+  if (n == "wu") return copy_rows(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + 128 + r % 128; });
+  if (n == "wd") return copy_rows(w.wd, H, I, ident);
+  if (n == "bq" || n == "bk" || n == "bv") {
+    if (!w.bqkv) return gllm::set_error(GLLM_EINVAL, "model has no qkv bias");
+    const int64_t o = n == "bq" ? 0 : (n == "bk" ? qd : qd + kd), len = n == "bq" ? qd : kd;
+    if (row0 != 0 || nrows != 1) return gllm::set_error(GLLM_EINVAL, "bias: read row 0 only");
+    CK(cudaMemcpy(out, w.bqkv + o, len * sizeof(float), cudaMemcpyDeviceToHost));
+    return GLLM_OK;
+  }
+  return gllm::set_error(GLLM_EINVAL, "unknown weight '%s'", name);
+  GLLM_TRY_END
+}
+
+int gllm_stage_read_kv(gllm_stage* st, int32_t layer, const int32_t* slots, int32_t n, float* k_out, float* v_out) {
+  GLLM_TRY_BEGIN
+  if (!st || (!slots && n) || !k_out || !v_out) return gllm::set_error(GLLM_EINVAL, "bad arguments");
+  if (layer < st->lb || layer >= st->le) return gllm::set_error(GLLM_EINVAL, "layer not on this stage");
+  cudaSetDevice(st->device);
+  LayerW& w = st->layers[layer - st->lb];
+  const int Hkv = st->cfg.n_kv_heads, D = st->cfg.head_dim, bs = st->bs;
+  std::vector<bf16> tmp(D);
+  for (int i = 0; i < n; ++i) {
+    const int64_t sl = slots[i];
+    if (sl < 0 || sl >= (int64_t)st->kv_blocks * bs) return gllm::set_error(GLLM_EINVAL, "slot out of range");
+    const int64_t blk = sl / bs, o = sl % bs;
+    for (int h = 0; h < Hkv; ++h) {
+      const size_t idx = ((blk * Hkv + h) * bs + o) * D;
+      CK(cudaMemcpy(tmp.data(), w.kc + idx, D * sizeof(bf16), cudaMemcpyDeviceToHost));
+      for (int j = 0; j < D; ++j) k_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(tmp[j]);
+      CK(cudaMemcpy(tmp.data(), w.vc + idx, D * sizeof(bf16), cudaMemcpyDeviceToHost));
+      for (int j = 0; j < D; ++j) v_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(tmp[j]);
+    }
+  }
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n) {
+  if (!st || !out || n < 0 || n > st->max_tokens) return gllm::set_error(GLLM_EINVAL, "bad arguments");
+  cudaSetDevice(st->device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(out, st->slots, n * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  return GLLM_OK;
+}
+
+int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed) {
+  if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
+  cudaSetDevice(st->device);
+  const size_t n = (size_t)st->kv_blocks * st->cfg.n_kv_heads * st->bs * st->cfg.head_dim;
+  for (int l = st->lb; l < st->le; ++l) {
+    if (layer >= 0 && l != layer) continue;
+    LayerW& w = st->layers[l - st->lb];
+    gllm::launch_fill_kv(w.kc, w.vc, n, seed, 0xEE0000ull + 2 * (uint64_t)l, 0);
+  }
+  CK(cudaDeviceSynchronize());
+  return GLLM_OK;
+}
+
+}  // extern "C"

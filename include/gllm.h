@@ -174,6 +174,18 @@ GLLM_API int gllm_free_stage(gllm_stage* st);
 GLLM_API int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* desc, const void* hidden_in,
                        void* hidden_out, int32_t* sampled_out, void* stream);
 
+/* Two-phase form of stage_forward, after the paper's dual-phase transmission
+ * (L204): prepare() validates the desc, builds the attention work lists and
+ * copies all metadata to a stage-owned device slot on `stream` as soon as the
+ * schedule is known; forward_prepared() later launches the layers once the
+ * activations arrive (it waits on the slot's copy event, any stream).  The
+ * handle stays valid until gllm_stage_release(); a slot is only reused after
+ * its last forward completed.  Same errors as gllm_stage_forward. */
+GLLM_API int gllm_stage_prepare(gllm_stage* st, const gllm_batch_desc* desc, void* stream, int32_t* handle);
+GLLM_API int gllm_stage_forward_prepared(gllm_stage* st, int32_t handle, const void* hidden_in, void* hidden_out,
+                                         int32_t* sampled_out, void* stream);
+GLLM_API int gllm_stage_release(gllm_stage* st, int32_t handle);
+
 /* Pipeline hand-off (a12; activations over NCCL, L222).  comm_init joins an
  * NCCL communicator of `world` ranks (unique_id: 128 bytes from ncclGetUniqueId,
  * exchanged by the caller).  send/recv move num_tokens x hidden fp32 rows of a
@@ -200,7 +212,7 @@ GLLM_API int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n);
  * tensor id 0xEE0000 + 2*l (+1 for V).  Used by benchmarks for warm decode state. */
 GLLM_API int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed);
 
-/* Timing of the last forward from CUDA events recorded on the forward's own
+/* Timing of the forwards since the previous call, from CUDA events recorded on each forward's own
  * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).
  * out[n] receives milliseconds per category (synchronises on the events):
  *   [0] whole forward  [1] QKV GEMM  [2] O GEMM  [3] gate_up GEMM  [4] down GEMM

@@ -88,6 +88,19 @@ NcclApi& nccl() {
 
 size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 
+// One batch's metadata, packed on the host (pinned) and copied to the device once: token ids,
+// positions, cu_q, kv_len, block table, sample rows and the attention work lists.
+struct Prepared {
+  bool in_use = false;
+  int T = 0, S = 0, NP = 0, maxblk = 0, ns = 0, n_pi = 0, n_di = 0, n_mi = 0, split_len = 16, nparts = 0;
+  size_t o_ids = 0, o_pos = 0, o_cu = 0, o_kvl = 0, o_bt = 0, o_samp = 0, o_pi = 0, o_di = 0, o_mi = 0, bytes = 0;
+  uint8_t* host = nullptr;
+  uint8_t* dev = nullptr;
+  size_t cap = 0;
+  cudaEvent_t copied = nullptr;  // H2D of this slot done
+  cudaEvent_t used = nullptr;    // last forward reading this slot done
+};
+
 }  // namespace
 
 struct gllm_stage {
@@ -109,10 +122,7 @@ struct gllm_stage {
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
   int parts_cap = 0;
-  uint8_t* pinned[RING] = {};
-  uint8_t* meta_dev[RING] = {};
-  size_t meta_cap = 0;
-  cudaEvent_t ring_ev[RING] = {};
+  std::vector<Prepared> prep;  // [0, RING): internal ring of stage_forward; others: gllm_stage_prepare handles
   int ring_i = 0;
   std::vector<void*> allocs;
   ncclComm_t comm = nullptr;
@@ -209,10 +219,11 @@ void destroy(gllm_stage* st) {
   cudaSetDevice(st->device);
   cudaDeviceSynchronize();
   for (void* p : st->allocs) cudaFree(p);
-  for (int i = 0; i < RING; ++i) {
-    if (st->pinned[i]) cudaFreeHost(st->pinned[i]);
-    if (st->meta_dev[i]) cudaFree(st->meta_dev[i]);
-    if (st->ring_ev[i]) cudaEventDestroy(st->ring_ev[i]);
+  for (auto& p : st->prep) {
+    if (p.host) cudaFreeHost(p.host);
+    if (p.dev) cudaFree(p.dev);
+    if (p.copied) cudaEventDestroy(p.copied);
+    if (p.used) cudaEventDestroy(p.used);
   }
   for (auto e : st->ev_pool) cudaEventDestroy(e);
   if (st->comm && nccl().ok) nccl().comm_destroy(st->comm);
@@ -220,22 +231,26 @@ void destroy(gllm_stage* st) {
   delete st;
 }
 
-int ensure_meta(gllm_stage* st, size_t bytes) {
-  if (bytes <= st->meta_cap) return GLLM_OK;
-  size_t cap = std::max<size_t>(bytes * 2, 1 << 20);
-  for (int i = 0; i < RING; ++i) {
-    if (st->ring_ev[i]) CK(cudaEventSynchronize(st->ring_ev[i]));
-  }
-  CK(cudaDeviceSynchronize());
-  for (int i = 0; i < RING; ++i) {
-    if (st->pinned[i]) cudaFreeHost(st->pinned[i]);
-    if (st->meta_dev[i]) cudaFree(st->meta_dev[i]);
-    st->pinned[i] = nullptr;
-    st->meta_dev[i] = nullptr;
-    CK(cudaMallocHost(&st->pinned[i], cap));
-    CK(cudaMalloc(&st->meta_dev[i], cap));
-  }
-  st->meta_cap = cap;
+int new_slot(gllm_stage* st) {
+  Prepared p;
+  CK(cudaEventCreateWithFlags(&p.copied, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&p.used, cudaEventDisableTiming));
+  st->prep.push_back(p);
+  return GLLM_OK;
+}
+
+int ensure_slot_cap(Prepared& p, size_t bytes) {
+  if (bytes <= p.cap) return GLLM_OK;
+  CK(cudaEventSynchronize(p.copied));
+  CK(cudaEventSynchronize(p.used));
+  if (p.host) cudaFreeHost(p.host);
+  if (p.dev) cudaFree(p.dev);
+  p.host = nullptr;
+  p.dev = nullptr;
+  const size_t cap = std::max<size_t>(bytes * 3 / 2, 256 << 10);
+  CK(cudaMallocHost(&p.host, cap));
+  CK(cudaMalloc(&p.dev, cap));
+  p.cap = cap;
   return GLLM_OK;
 }
 
@@ -360,11 +375,8 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = gllm::make_tmap_bf16(&st->tm_attn, st->attn, R, qd, gllm::GEMM_BM)) ||
       (rc = gllm::make_tmap_bf16(&st->tm_act, st->act, R, I, gllm::GEMM_BM)))
     return fail(rc);
-  for (int i = 0; i < RING; ++i) {
-    cudaError_t e = cudaEventCreateWithFlags(&st->ring_ev[i], cudaEventDisableTiming);
-    if (e != cudaSuccess) return fail(gllm::set_error(GLLM_ECUDA, "event: %s", cudaGetErrorString(e)));
-  }
-  if ((rc = ensure_meta(st, 1 << 20)) < 0) return fail(rc);
+  for (int i = 0; i < RING; ++i)
+    if ((rc = new_slot(st)) < 0) return fail(rc);
   if ((rc = ensure_parts(st, 1024)) < 0) return fail(rc);
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return fail(gllm::set_error(GLLM_ECUDA, "init: %s", cudaGetErrorString(e)));
@@ -378,11 +390,14 @@ int gllm_free_stage(gllm_stage* st) {
   return GLLM_OK;
 }
 
-int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hidden_in, void* hidden_out,
-                       int32_t* sampled_out, void* stream) {
-  GLLM_TRY_BEGIN
+}  // extern "C"
+
+namespace {
+
+// Validates the batch, builds the attention work lists and copies everything to the device
+// slot on `s` (the early-metadata phase of the paper's dual-phase transmission, L204).
+int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepared& P) {
   if (!st || !d) return gllm::set_error(GLLM_EINVAL, "null argument");
-  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const gllm_model_cfg& c = st->cfg;
   const int T = d->num_tokens, S = d->num_seqs, NP = d->num_prefill_seqs, maxblk = d->max_blocks_per_seq;
   const int ns = d->num_samples;
@@ -391,15 +406,14 @@ int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hid
   if (T < 0 || T > st->max_tokens) return gllm::set_error(GLLM_EINVAL, "num_tokens %d > max_tokens %d", T, st->max_tokens);
   if (S < 0 || S > st->max_seqs) return gllm::set_error(GLLM_EINVAL, "num_seqs %d > max_seqs %d", S, st->max_seqs);
   if (NP < 0 || NP > S || ns < 0 || ns > S || maxblk < 0) return gllm::set_error(GLLM_EINVAL, "bad batch counts");
-  if (T == 0) {
-    st->last_T = 0;
-    st->last_launches = 0;
-    return GLLM_OK;
-  }
+  P.T = T;
+  P.S = S;
+  P.NP = NP;
+  P.maxblk = maxblk;
+  P.ns = ns;
+  if (T == 0) return GLLM_OK;
   if (!d->token_ids || !d->positions || !d->cu_q || !d->kv_len || !d->block_table || (ns && !d->sample_token_idx))
     return gllm::set_error(GLLM_EINVAL, "null batch array");
-  if (!st->is_first() && !hidden_in) return gllm::set_error(GLLM_EINVAL, "hidden_in required on stage > 0");
-  if (!st->is_last() && !hidden_out) return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
   if (d->cu_q[0] != 0 || d->cu_q[S] != T) return gllm::set_error(GLLM_EINVAL, "cu_q must span [0, num_tokens]");
   const int G = c.n_heads / c.n_kv_heads;
   int64_t total_pages = 0;
@@ -447,52 +461,71 @@ int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hid
       nparts += nsplit;
     }
   }
-  RC(ensure_parts(st, nparts));
-  // ---------------- pack metadata into a pinned ring slot; one H2D copy (K9)
+  // ---------------- pack into the slot's pinned buffer; one H2D copy (K9)
   size_t off = 0;
   auto sect = [&](size_t bytes) {
     size_t o = off;
     off = align16(off + bytes);
     return o;
   };
-  const size_t o_ids = sect(T * 4), o_pos = sect(T * 4), o_cu = sect((S + 1) * 4), o_kvl = sect(S * 4),
-               o_bt = sect((size_t)S * maxblk * 4), o_samp = sect(ns * 4),
-               o_pi = sect(pitems.size() * sizeof(gllm::PrefillItem)),
-               o_di = sect(ditems.size() * sizeof(gllm::DecodeItem)),
-               o_mi = sect(merges.size() * sizeof(gllm::MergeItem));
-  RC(ensure_meta(st, off));
+  P.o_ids = sect(T * 4);
+  P.o_pos = sect(T * 4);
+  P.o_cu = sect((S + 1) * 4);
+  P.o_kvl = sect(S * 4);
+  P.o_bt = sect((size_t)S * maxblk * 4);
+  P.o_samp = sect(ns * 4);
+  P.o_pi = sect(pitems.size() * sizeof(gllm::PrefillItem));
+  P.o_di = sect(ditems.size() * sizeof(gllm::DecodeItem));
+  P.o_mi = sect(merges.size() * sizeof(gllm::MergeItem));
+  P.bytes = off;
+  P.n_pi = (int)pitems.size();
+  P.n_di = (int)ditems.size();
+  P.n_mi = (int)merges.size();
+  P.split_len = split_pages * bs;
+  P.nparts = nparts;
   CK(cudaSetDevice(st->device));
-  const int slot = st->ring_i;
-  st->ring_i = (st->ring_i + 1) % RING;
-  CK(cudaEventSynchronize(st->ring_ev[slot]));  // previous use of this slot has been copied
-  uint8_t* h = st->pinned[slot];
-  std::memcpy(h + o_ids, d->token_ids, T * 4);
-  std::memcpy(h + o_pos, d->positions, T * 4);
-  std::memcpy(h + o_cu, d->cu_q, (S + 1) * 4);
-  std::memcpy(h + o_kvl, d->kv_len, S * 4);
-  std::memcpy(h + o_bt, d->block_table, (size_t)S * maxblk * 4);
-  if (ns) std::memcpy(h + o_samp, d->sample_token_idx, ns * 4);
-  if (!pitems.empty()) std::memcpy(h + o_pi, pitems.data(), pitems.size() * sizeof(gllm::PrefillItem));
-  if (!ditems.empty()) std::memcpy(h + o_di, ditems.data(), ditems.size() * sizeof(gllm::DecodeItem));
-  if (!merges.empty()) std::memcpy(h + o_mi, merges.data(), merges.size() * sizeof(gllm::MergeItem));
-  uint8_t* m = st->meta_dev[slot];
-  if (st->timing_pending) st->timing_pending = false;
-  st->prof_ev.clear();
-  st->ev_used = 0;
-  st->last_launches = 0;
-  Prof p_total(st, s, C_TOTAL);
-  CK(cudaMemcpyAsync(m, h, off, cudaMemcpyHostToDevice, s));
-  CK(cudaEventRecord(st->ring_ev[slot], s));
-  const int32_t* d_ids = reinterpret_cast<const int32_t*>(m + o_ids);
-  const int32_t* d_pos = reinterpret_cast<const int32_t*>(m + o_pos);
-  const int32_t* d_cu = reinterpret_cast<const int32_t*>(m + o_cu);
-  const int32_t* d_kvl = reinterpret_cast<const int32_t*>(m + o_kvl);
-  const int32_t* d_bt = reinterpret_cast<const int32_t*>(m + o_bt);
-  const int32_t* d_samp = reinterpret_cast<const int32_t*>(m + o_samp);
-  const auto* d_pi = reinterpret_cast<const gllm::PrefillItem*>(m + o_pi);
-  const auto* d_di = reinterpret_cast<const gllm::DecodeItem*>(m + o_di);
-  const auto* d_mi = reinterpret_cast<const gllm::MergeItem*>(m + o_mi);
+  RC(ensure_slot_cap(P, off));
+  CK(cudaEventSynchronize(P.copied));      // the previous H2D out of this pinned buffer is done
+  CK(cudaStreamWaitEvent(s, P.used, 0));   // and no queued forward still reads the device copy
+  uint8_t* h = P.host;
+  std::memcpy(h + P.o_ids, d->token_ids, T * 4);
+  std::memcpy(h + P.o_pos, d->positions, T * 4);
+  std::memcpy(h + P.o_cu, d->cu_q, (S + 1) * 4);
+  std::memcpy(h + P.o_kvl, d->kv_len, S * 4);
+  std::memcpy(h + P.o_bt, d->block_table, (size_t)S * maxblk * 4);
+  if (ns) std::memcpy(h + P.o_samp, d->sample_token_idx, ns * 4);
+  if (!pitems.empty()) std::memcpy(h + P.o_pi, pitems.data(), pitems.size() * sizeof(gllm::PrefillItem));
+  if (!ditems.empty()) std::memcpy(h + P.o_di, ditems.data(), ditems.size() * sizeof(gllm::DecodeItem));
+  if (!merges.empty()) std::memcpy(h + P.o_mi, merges.data(), merges.size() * sizeof(gllm::MergeItem));
+  CK(cudaMemcpyAsync(P.dev, h, off, cudaMemcpyHostToDevice, s));
+  CK(cudaEventRecord(P.copied, s));
+  return GLLM_OK;
+}
 
+// Enqueues the stage forward of a prepared batch on `s`.
+int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidden_out, int32_t* sampled_out,
+                 cudaStream_t s) {
+  const gllm_model_cfg& c = st->cfg;
+  const int T = P.T, S = P.S, maxblk = P.maxblk, ns = P.ns, bs = st->bs;
+  st->last_launches = 0;
+  st->last_T = T;
+  if (T == 0) return GLLM_OK;
+  if (!st->is_first() && !hidden_in) return gllm::set_error(GLLM_EINVAL, "hidden_in required on stage > 0");
+  if (!st->is_last() && !hidden_out) return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
+  RC(ensure_parts(st, P.nparts));
+  CK(cudaSetDevice(st->device));
+  CK(cudaStreamWaitEvent(s, P.copied, 0));
+  Prof p_total(st, s, C_TOTAL);
+  uint8_t* m = P.dev;
+  const int32_t* d_ids = reinterpret_cast<const int32_t*>(m + P.o_ids);
+  const int32_t* d_pos = reinterpret_cast<const int32_t*>(m + P.o_pos);
+  const int32_t* d_cu = reinterpret_cast<const int32_t*>(m + P.o_cu);
+  const int32_t* d_kvl = reinterpret_cast<const int32_t*>(m + P.o_kvl);
+  const int32_t* d_bt = reinterpret_cast<const int32_t*>(m + P.o_bt);
+  const int32_t* d_samp = reinterpret_cast<const int32_t*>(m + P.o_samp);
+  const auto* d_pi = reinterpret_cast<const gllm::PrefillItem*>(m + P.o_pi);
+  const auto* d_di = reinterpret_cast<const gllm::DecodeItem*>(m + P.o_di);
+  const auto* d_mi = reinterpret_cast<const gllm::MergeItem*>(m + P.o_mi);
   const int H = c.hidden, D = c.head_dim, qd = st->qd(), kd = st->kd(), nqkv = qd + 2 * kd, I = c.intermediate;
   {
     Prof p(st, s, C_OTHER);
@@ -521,7 +554,7 @@ int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hid
   aa.out = st->attn;
   aa.part_o = st->part_o;
   aa.part_ml = st->part_ml;
-  aa.split_len = split_pages * bs;
+  aa.split_len = P.split_len;
   for (size_t li = 0; li < st->layers.size(); ++li) {
     LayerW& w = st->layers[li];
     {
@@ -540,15 +573,15 @@ int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hid
     }
     aa.kc = w.kc;
     aa.vc = w.vc;
-    if (!pitems.empty()) {
+    if (P.n_pi > 0) {
       Prof p(st, s, C_PREFILL);
-      RC(gllm::launch_prefill_attention(aa, d_pi, (int)pitems.size(), s));
+      RC(gllm::launch_prefill_attention(aa, d_pi, P.n_pi, s));
       st->last_launches += 1;
     }
-    if (!ditems.empty()) {
+    if (P.n_di > 0) {
       Prof p(st, s, C_DECODE);
-      RC(gllm::launch_decode_attention(aa, d_di, (int)ditems.size(), d_mi, (int)merges.size(), s));
-      st->last_launches += merges.empty() ? 1 : 2;
+      RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
+      st->last_launches += P.n_mi ? 2 : 1;
     }
     {
       Prof p(st, s, C_O);
@@ -576,13 +609,59 @@ int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hid
     gllm::launch_argmax_reduce(st->part_val, st->part_idx, ns, ntn, sampled_out ? sampled_out : st->sampled_tmp, s);
     st->last_launches += 2;
   }
+  CK(cudaEventRecord(P.used, s));
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "stage_forward launch: %s", cudaGetErrorString(e));
-  st->last_T = T;
-  st->timing_pending = st->profiling;
+  return GLLM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int gllm_stage_forward(gllm_stage* st, const gllm_batch_desc* d, const void* hidden_in, void* hidden_out,
+                       int32_t* sampled_out, void* stream) {
+  GLLM_TRY_BEGIN
+  if (!st || !d) return gllm::set_error(GLLM_EINVAL, "null argument");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  Prepared& P = st->prep[st->ring_i];
+  st->ring_i = (st->ring_i + 1) % RING;
+  RC(prepare_impl(st, d, s, P));
+  return forward_impl(st, P, hidden_in, hidden_out, sampled_out, s);
+  GLLM_TRY_END
+}
+
+int gllm_stage_prepare(gllm_stage* st, const gllm_batch_desc* d, void* stream, int32_t* handle) {
+  GLLM_TRY_BEGIN
+  if (!st || !d || !handle) return gllm::set_error(GLLM_EINVAL, "null argument");
+  size_t i = RING;
+  while (i < st->prep.size() && st->prep[i].in_use) ++i;
+  if (i == st->prep.size()) RC(new_slot(st));
+  Prepared& P = st->prep[i];
+  RC(prepare_impl(st, d, reinterpret_cast<cudaStream_t>(stream), P));
+  P.in_use = true;
+  *handle = (int32_t)i;
   return GLLM_OK;
   GLLM_TRY_END
 }
+
+int gllm_stage_forward_prepared(gllm_stage* st, int32_t handle, const void* hidden_in, void* hidden_out,
+                                int32_t* sampled_out, void* stream) {
+  GLLM_TRY_BEGIN
+  if (!st || handle < RING || handle >= (int32_t)st->prep.size() || !st->prep[handle].in_use)
+    return gllm::set_error(GLLM_EINVAL, "bad prepared handle %d", handle);
+  return forward_impl(st, st->prep[handle], hidden_in, hidden_out, sampled_out, reinterpret_cast<cudaStream_t>(stream));
+  GLLM_TRY_END
+}
+
+int gllm_stage_release(gllm_stage* st, int32_t handle) {
+  if (!st || handle < RING || handle >= (int32_t)st->prep.size())
+    return gllm::set_error(GLLM_EINVAL, "bad prepared handle %d", handle);
+  st->prep[handle].in_use = false;  // reuse waits on the slot's events
+  return GLLM_OK;
+}
+
+
 
 int gllm_stage_sync(gllm_stage* st) {
   if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
@@ -608,6 +687,8 @@ int gllm_stage_last_timing(gllm_stage* st, float* out, int32_t n) {
     acc[pe.first] += ms;
   }
   for (int i = 0; i < n && i < C_N; ++i) out[i] = acc[i];
+  st->prof_ev.clear();  // timings accumulate over forwards until read
+  st->ev_used = 0;
   return GLLM_OK;
 }
 

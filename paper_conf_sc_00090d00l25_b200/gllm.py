@@ -97,6 +97,9 @@ def lib():
             "gllm_init_stage": ([C.POINTER(ModelCfg), i32, i32, i32, i32, i32, i32, i32, C.POINTER(vp)], C.c_int),
             "gllm_free_stage": ([vp], C.c_int),
             "gllm_stage_forward": ([vp, C.POINTER(BatchDesc), vp, vp, vp, vp], C.c_int),
+            "gllm_stage_prepare": ([vp, C.POINTER(BatchDesc), vp, _P32], C.c_int),
+            "gllm_stage_forward_prepared": ([vp, i32, vp, vp, vp, vp], C.c_int),
+            "gllm_stage_release": ([vp, i32], C.c_int),
             "gllm_get_unique_id": ([vp], C.c_int),
             "gllm_comm_init": ([vp, vp, i32, i32], C.c_int),
             "gllm_send_hidden": ([vp, vp, i32, i32, vp], C.c_int),
@@ -266,6 +269,20 @@ class Stage:
         """Enqueue stage_forward; buffers are raw device pointers (ints), stream a cudaStream_t int."""
         return _check(lib().gllm_stage_forward(self.h, C.byref(desc), hidden_in or None, hidden_out or None,
                                                sampled_out or None, stream or None))
+
+    def prepare(self, desc: BatchDesc, stream=0) -> int:
+        """Phase 1 (metadata): validate + copy the batch metadata to the device; returns a handle."""
+        h = C.c_int32()
+        _check(lib().gllm_stage_prepare(self.h, C.byref(desc), stream or None, C.byref(h)))
+        return h.value
+
+    def forward_prepared(self, handle, hidden_in=0, hidden_out=0, sampled_out=0, stream=0):
+        """Phase 2 (activations): launch the layers of a prepared batch."""
+        return _check(lib().gllm_stage_forward_prepared(self.h, handle, hidden_in or None, hidden_out or None,
+                                                        sampled_out or None, stream or None))
+
+    def release(self, handle):
+        _check(lib().gllm_stage_release(self.h, handle))
 
     def sync(self):
         _check(lib().gllm_stage_sync(self.h))

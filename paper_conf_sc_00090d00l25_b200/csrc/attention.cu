@@ -1,5 +1,6 @@
-// Varlen paged causal attention (a7): prefill chunks on tensor cores, decode rows as
-// bandwidth-bound paged gathers with warp-level softmax reductions.
+// Varlen paged causal attention (a7): prefill chunks and decode rows, both on tensor cores
+// (mma.sync m16n8k16, bf16 in / fp32 accumulate), K/V pages streamed through SMEM with
+// cp.async.
 //
 //   prefill chunk i (c_i tokens at offset s_i): token j attends keys [0, s_i + j]
 //   decode row j (position L_j - 1):           attends keys [0, L_j - 1]
@@ -19,141 +20,185 @@ namespace {
 
 constexpr float LOG2E = 1.4426950408889634f;
 
-__device__ __forceinline__ float dot8(const uint4& a, const uint4& b) {
-  const __nv_bfloat162* x = reinterpret_cast<const __nv_bfloat162*>(&a);
-  const __nv_bfloat162* y = reinterpret_cast<const __nv_bfloat162*>(&b);
-  float s = 0.f;
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const float2 p = __bfloat1622float2(x[i]), q = __bfloat1622float2(y[i]);
-    s = fmaf(p.x, q.x, s);
-    s = fmaf(p.y, q.y, s);
-  }
-  return s;
+// swizzled byte offset of (row, 16-byte chunk) in a row-major tile with D bf16 per row:
+// chunk' = chunk ^ (row % 8) keeps the 8 rows an ldmatrix reads on distinct banks.
+template <int D>
+__device__ __forceinline__ uint32_t swz(int row, int chunk) {
+  return row * (D * 2) + ((chunk ^ (row & 7)) << 4);
 }
 
 // ------------------------------------------------------------------ decode
-// CTA = (decode row, key split) x kv head; 4 warps stride over the split's 16-token pages.
-// Within a warp: LPT lanes cover one token's D dims (8 bf16 per lane), TPI tokens per
-// 16-byte load, so a page is NI loads per lane for K and NI for V.
+// Bandwidth-bound: every decode row reads L x 2 x D x 2 bytes of K/V per kv head once.
+// CTA = (decode row, key split) x kv head, 4 warps; warp w owns pages w, w+4, ... of the split
+// with its own online-softmax state and a private NST-stage cp.async ring (K page + V page per
+// stage), merged across warps at the end.  The G query heads of the kv head are the rows of
+// a 16-row MMA tile (rows >= G are zero), so Q K^T of a 16-token page is 2 n-tiles x D/16
+// k-steps and P V is 1 k-step x D/8 n-tiles -- no shuffles in the dot products.
+template <int D>
+struct DecodeSmem {
+  static constexpr int NST = 3;
+  static constexpr int PAGE = 16 * D * 2;
+  static constexpr int PER_WARP = NST * 2 * PAGE;
+  static constexpr int MERGE = 4 * 16 * D * 4 + 4 * 16 * 2 * 4;
+  static constexpr int BYTES = (4 * PER_WARP > MERGE ? 4 * PER_WARP : MERGE);
+};
+
 template <int D, int G>
 __global__ void __launch_bounds__(128) decode_attn_kernel(const AttnArgs a, const DecodeItem* __restrict__ items) {
-  constexpr int LPT = D / 8;
-  constexpr int TPI = 32 / LPT;
-  constexpr int NI = 16 / TPI;
-  __shared__ float sm_m[4][G], sm_l[4][G];
-  __shared__ float sm_acc[4][G][D];
+  static_assert(G >= 1 && G <= 16, "GQA group must fit one 16-row MMA tile");
+  constexpr int NCH = D / 8;
+  constexpr int NST = DecodeSmem<D>::NST;
+  constexpr int PAGE = DecodeSmem<D>::PAGE;
+  extern __shared__ __align__(128) uint8_t smem[];
 
   const DecodeItem it = items[blockIdx.x];
   const int kvh = blockIdx.y;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = lane >> 2, tq = lane & 3;
   const int t = a.cu_q[it.seq];
   const int L = a.kv_len[it.seq];
   const int k0 = it.split * a.split_len;
   const int k1 = min(L, k0 + a.split_len);
   const int nb0 = k0 / 16, nb1 = (k1 + 15) / 16;
-  const int d0 = (lane % LPT) * 8;
-  const int tk = lane / LPT;
-  const float sl2 = LOG2E * rsqrtf((float)D);
-
-  uint4 qv[G];
-#pragma unroll
-  for (int h = 0; h < G; ++h)
-    qv[h] = *reinterpret_cast<const uint4*>(a.q + (size_t)t * a.q_stride + (size_t)(kvh * G + h) * D + d0);
-  float m[G], l[G], acc[G][8];
-#pragma unroll
-  for (int h = 0; h < G; ++h) {
-    m[h] = -INFINITY;
-    l[h] = 0.f;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) acc[h][j] = 0.f;
-  }
+  const int n_my = nb1 - nb0 > warp ? (nb1 - nb0 - warp + 3) / 4 : 0;
   const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
-  for (int b = nb0 + warp; b < nb1; b += 4) {
-    const size_t page = (size_t)bt[b];
-    const __nv_bfloat16* kb = a.kc + ((page * a.Hkv + kvh) * 16) * D;
-    const __nv_bfloat16* vb = a.vc + ((page * a.Hkv + kvh) * 16) * D;
-    uint4 kr[NI], vr[NI];
+  const float sl2 = LOG2E * rsqrtf((float)D);
+  uint8_t* ws = smem + warp * DecodeSmem<D>::PER_WARP;
+  const uint32_t ws_u32 = ptx::smem_u32(ws);
+
+  auto issue = [&](int i) {
+    if (i < n_my) {
+      const size_t page = (size_t)bt[nb0 + warp + 4 * i];
+      const __nv_bfloat16* kp = a.kc + ((page * a.Hkv + kvh) * 16) * D;
+      const __nv_bfloat16* vp = a.vc + ((page * a.Hkv + kvh) * 16) * D;
+      const uint32_t st = ws_u32 + (i % NST) * 2 * PAGE;
 #pragma unroll
-    for (int i = 0; i < NI; ++i) kr[i] = ptx::ld_nc_v4(kb + (tk + i * TPI) * D + d0);
-#pragma unroll
-    for (int i = 0; i < NI; ++i) vr[i] = ptx::ld_nc_v4(vb + (tk + i * TPI) * D + d0);
-    float s[NI][G];
-#pragma unroll
-    for (int i = 0; i < NI; ++i)
-#pragma unroll
-      for (int h = 0; h < G; ++h) s[i][h] = dot8(qv[h], kr[i]);
-#pragma unroll
-    for (int o = 1; o < LPT; o <<= 1)
-#pragma unroll
-      for (int i = 0; i < NI; ++i)
-#pragma unroll
-        for (int h = 0; h < G; ++h) s[i][h] += __shfl_xor_sync(0xffffffffu, s[i][h], o);
-#pragma unroll
-    for (int i = 0; i < NI; ++i) {
-      const bool ok = b * 16 + tk + i * TPI < k1;
-#pragma unroll
-      for (int h = 0; h < G; ++h) s[i][h] = ok ? s[i][h] * sl2 : -INFINITY;
-    }
-#pragma unroll
-    for (int h = 0; h < G; ++h) {
-      float mx = s[0][h];
-#pragma unroll
-      for (int i = 1; i < NI; ++i) mx = fmaxf(mx, s[i][h]);
-#pragma unroll
-      for (int o = LPT; o < 32; o <<= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-      const float mn = fmaxf(m[h], mx);
-      const float corr = exp2f(m[h] - mn);
-      m[h] = mn;
-      l[h] *= corr;
-#pragma unroll
-      for (int j = 0; j < 8; ++j) acc[h][j] *= corr;
-#pragma unroll
-      for (int i = 0; i < NI; ++i) {
-        const float p = exp2f(s[i][h] - mn);
-        l[h] += p;
-        const __nv_bfloat162* v2 = reinterpret_cast<const __nv_bfloat162*>(&vr[i]);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const float2 vf = __bfloat1622float2(v2[j]);
-          acc[h][2 * j] = fmaf(p, vf.x, acc[h][2 * j]);
-          acc[h][2 * j + 1] = fmaf(p, vf.y, acc[h][2 * j + 1]);
-        }
+      for (int j = 0; j < 16 * NCH / 32; ++j) {
+        const int c = lane + 32 * j;
+        const int r = c / NCH, ch = c % NCH;
+        ptx::cp_async16(st + swz<D>(r, ch), kp + r * D + ch * 8, true);
+        ptx::cp_async16(st + PAGE + swz<D>(r, ch), vp + r * D + ch * 8, true);
       }
     }
-  }
-  // combine the TPI token groups of the warp (m is warp-uniform)
+    ptx::cp_async_commit();  // always commit (possibly empty) so group counting stays uniform
+  };
 #pragma unroll
-  for (int o = LPT; o < 32; o <<= 1)
+  for (int i = 0; i < NST - 1; ++i) issue(i);
+
+  // Q fragments (rows = the G heads of this kv head; rows >= G are zero)
+  uint32_t qa[D / 16][4];
+  {
+    const __nv_bfloat16* qrow = a.q + (size_t)t * a.q_stride + (size_t)kvh * G * D;
 #pragma unroll
-    for (int h = 0; h < G; ++h) {
-      l[h] += __shfl_xor_sync(0xffffffffu, l[h], o);
-#pragma unroll
-      for (int j = 0; j < 8; ++j) acc[h][j] += __shfl_xor_sync(0xffffffffu, acc[h][j], o);
+    for (int ks = 0; ks < D / 16; ++ks) {
+      const int c0 = ks * 16 + 2 * tq;
+      qa[ks][0] = g < G ? *reinterpret_cast<const uint32_t*>(qrow + g * D + c0) : 0u;
+      qa[ks][1] = g + 8 < G ? *reinterpret_cast<const uint32_t*>(qrow + (g + 8) * D + c0) : 0u;
+      qa[ks][2] = g < G ? *reinterpret_cast<const uint32_t*>(qrow + g * D + c0 + 8) : 0u;
+      qa[ks][3] = g + 8 < G ? *reinterpret_cast<const uint32_t*>(qrow + (g + 8) * D + c0 + 8) : 0u;
     }
-  if (tk == 0) {
+  }
+  float o[D / 8][4];
 #pragma unroll
-    for (int h = 0; h < G; ++h) {
+  for (int n = 0; n < D / 8; ++n) o[n][0] = o[n][1] = o[n][2] = o[n][3] = 0.f;
+  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
+
+  for (int i = 0; i < n_my; ++i) {
+    issue(i + NST - 1);
+    ptx::cp_async_wait<NST - 1>();
+    __syncwarp();
+    const uint32_t kst = ws_u32 + (i % NST) * 2 * PAGE;
+    const uint32_t vst = kst + PAGE;
+    float s[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
 #pragma unroll
-      for (int j = 0; j < 8; ++j) sm_acc[warp][h][d0 + j] = acc[h][j];
-      if (lane == 0) {
-        sm_m[warp][h] = m[h];
-        sm_l[warp][h] = l[h];
+    for (int ks = 0; ks < D / 16; ++ks) {
+      uint32_t b0, b1, b2, b3;
+      ptx::ldsm_x4(kst + swz<D>(((lane >> 4) << 3) + (lane & 7), ks * 2 + ((lane >> 3) & 1)), b0, b1, b2, b3);
+      ptx::mma_bf16_16816(s[0], qa[ks], b0, b1);
+      ptx::mma_bf16_16816(s[1], qa[ks], b2, b3);
+    }
+    const int kbase = (nb0 + warp + 4 * i) * 16;
+#pragma unroll
+    for (int n = 0; n < 2; ++n)
+#pragma unroll
+      for (int e = 0; e < 4; ++e) s[n][e] = (kbase + n * 8 + 2 * tq + (e & 1) < k1) ? s[n][e] * sl2 : -INFINITY;
+    float corr[2];
+#pragma unroll
+    for (int hr = 0; hr < 2; ++hr) {
+      float mx = fmaxf(fmaxf(s[0][2 * hr], s[0][2 * hr + 1]), fmaxf(s[1][2 * hr], s[1][2 * hr + 1]));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
+      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
+      const float mn = fmaxf(mrow[hr], mx);
+      corr[hr] = exp2f(mrow[hr] - mn);
+      mrow[hr] = mn;
+      float sum = 0.f;
+#pragma unroll
+      for (int n = 0; n < 2; ++n) {
+        s[n][2 * hr] = exp2f(s[n][2 * hr] - mn);
+        s[n][2 * hr + 1] = exp2f(s[n][2 * hr + 1] - mn);
+        sum += s[n][2 * hr] + s[n][2 * hr + 1];
+      }
+      lrow[hr] = lrow[hr] * corr[hr] + sum;
+    }
+    uint32_t pa[4];
+    pa[0] = ptx::pack_bf16(s[0][0], s[0][1]);
+    pa[1] = ptx::pack_bf16(s[0][2], s[0][3]);
+    pa[2] = ptx::pack_bf16(s[1][0], s[1][1]);
+    pa[3] = ptx::pack_bf16(s[1][2], s[1][3]);
+#pragma unroll
+    for (int dp = 0; dp < D / 16; ++dp) {
+      o[2 * dp][0] *= corr[0];
+      o[2 * dp][1] *= corr[0];
+      o[2 * dp][2] *= corr[1];
+      o[2 * dp][3] *= corr[1];
+      o[2 * dp + 1][0] *= corr[0];
+      o[2 * dp + 1][1] *= corr[0];
+      o[2 * dp + 1][2] *= corr[1];
+      o[2 * dp + 1][3] *= corr[1];
+      uint32_t b0, b1, b2, b3;
+      ptx::ldsm_x4_t(vst + swz<D>((lane & 7) + (((lane >> 3) & 1) << 3), dp * 2 + (lane >> 4)), b0, b1, b2, b3);
+      ptx::mma_bf16_16816(o[2 * dp], pa, b0, b1);
+      ptx::mma_bf16_16816(o[2 * dp + 1], pa, b2, b3);
+    }
+    __syncwarp();  // everyone done reading this stage before it is refilled
+  }
+  ptx::cp_async_wait<0>();
+#pragma unroll
+  for (int hr = 0; hr < 2; ++hr) {
+    lrow[hr] += __shfl_xor_sync(0xffffffffu, lrow[hr], 1);
+    lrow[hr] += __shfl_xor_sync(0xffffffffu, lrow[hr], 2);
+  }
+  // ---- merge the 4 warps (SMEM reused)
+  __syncthreads();
+  float* sm_o = reinterpret_cast<float*>(smem);         // [4][16][D]
+  float* sm_ml = sm_o + 4 * 16 * D;                      // [4][16][2]
+#pragma unroll
+  for (int hr = 0; hr < 2; ++hr) {
+    const int r = g + 8 * hr;
+    if (r < G) {
+#pragma unroll
+      for (int n = 0; n < D / 8; ++n) {
+        sm_o[(warp * 16 + r) * D + n * 8 + 2 * tq] = o[n][2 * hr];
+        sm_o[(warp * 16 + r) * D + n * 8 + 2 * tq + 1] = o[n][2 * hr + 1];
+      }
+      if (tq == 0) {
+        sm_ml[(warp * 16 + r) * 2] = mrow[hr];
+        sm_ml[(warp * 16 + r) * 2 + 1] = lrow[hr];
       }
     }
   }
   __syncthreads();
   for (int idx = threadIdx.x; idx < G * D; idx += blockDim.x) {
     const int h = idx / D, d = idx % D;
-    float M = sm_m[0][h];
+    float M = -INFINITY;
 #pragma unroll
-    for (int w = 1; w < 4; ++w) M = fmaxf(M, sm_m[w][h]);
+    for (int w = 0; w < 4; ++w) M = fmaxf(M, sm_ml[(w * 16 + h) * 2]);
     float Ls = 0.f, A = 0.f;
 #pragma unroll
     for (int w = 0; w < 4; ++w) {
-      const float f = exp2f(sm_m[w][h] - M);
-      Ls += sm_l[w][h] * f;
-      A += sm_acc[w][h][d] * f;
+      const float f = exp2f(sm_ml[(w * 16 + h) * 2] - M);
+      Ls += sm_ml[(w * 16 + h) * 2 + 1] * f;
+      A += sm_o[(w * 16 + h) * D + d] * f;
     }
     if (it.part < 0) {
       a.out[(size_t)t * a.Hq * D + (size_t)(kvh * G + h) * D + d] = __float2bfloat16_rn(A / Ls);
@@ -200,19 +245,13 @@ struct PrefillSmem {
   static constexpr int BYTES = 5 * TILE_BYTES;  // Q + 2 x (K, V)
 };
 
-// swizzled byte offset of (row, 16-byte chunk) in a [64][D] bf16 tile
-template <int D>
-__device__ __forceinline__ uint32_t swz(int row, int chunk) {
-  return row * (D * 2) + ((chunk ^ (row & 7)) << 4);
-}
-
 template <int D>
 __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
   constexpr int NCH = D / 8;  // 16-byte chunks per row
+  constexpr int TB = PrefillSmem<D>::TILE_BYTES;
   extern __shared__ __align__(128) uint8_t smem[];
-  uint8_t* sQ = smem;
-  uint8_t* sK[2] = {smem + PrefillSmem<D>::TILE_BYTES, smem + 2 * PrefillSmem<D>::TILE_BYTES};
-  uint8_t* sV[2] = {smem + 3 * PrefillSmem<D>::TILE_BYTES, smem + 4 * PrefillSmem<D>::TILE_BYTES};
+  const uint32_t sQ = ptx::smem_u32(smem);
+  // buffer b: K at sQ + (1 + 2b) TB, V at sQ + (2 + 2b) TB
 
   const PrefillItem it = items[blockIdx.x];
   const int kvh = blockIdx.y;
@@ -235,9 +274,10 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
     const int rr = min(it.row0 + r, nrows - 1);
     const int tok = rr / G, h = kvh * G + rr % G;
     const __nv_bfloat16* src = a.q + (size_t)(t0 + tok) * a.q_stride + (size_t)h * D + ch * 8;
-    ptx::cp_async16(ptx::smem_u32(sQ) + swz<D>(r, ch), src, true);
+    ptx::cp_async16(sQ + swz<D>(r, ch), src, true);
   }
   auto load_kv = [&](int kt, int buf) {
+    const uint32_t kb = sQ + (1 + 2 * buf) * TB, vb = kb + TB;
     for (int idx = threadIdx.x; idx < 64 * NCH; idx += 128) {
       const int r = idx / NCH, ch = idx % NCH;
       const int key = kt * 64 + r;
@@ -245,8 +285,8 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
       const bool ok = blk < nblk_seq;
       const size_t page = ok ? (size_t)bt[blk] : 0;
       const size_t off = ((page * a.Hkv + kvh) * 16 + (key & 15)) * D + ch * 8;
-      ptx::cp_async16(ptx::smem_u32(sK[buf]) + swz<D>(r, ch), a.kc + off, ok);
-      ptx::cp_async16(ptx::smem_u32(sV[buf]) + swz<D>(r, ch), a.vc + off, ok);
+      ptx::cp_async16(kb + swz<D>(r, ch), a.kc + off, ok);
+      ptx::cp_async16(vb + swz<D>(r, ch), a.vc + off, ok);
     }
   };
   load_kv(0, 0);
@@ -278,10 +318,10 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
       for (int ks = 0; ks < D / 16; ++ks) {
         const int r = warp * 16 + (lane & 15);
         const int ch = ks * 2 + (lane >> 4);
-        ptx::ldsm_x4(ptx::smem_u32(sQ) + swz<D>(r, ch), qa[ks][0], qa[ks][1], qa[ks][2], qa[ks][3]);
+        ptx::ldsm_x4(sQ + swz<D>(r, ch), qa[ks][0], qa[ks][1], qa[ks][2], qa[ks][3]);
       }
     }
-    const int buf = kt & 1;
+    const uint32_t kb = sQ + (1 + 2 * (kt & 1)) * TB, vb = kb + TB;
     // ---- S = Q K^T  (16 rows x 64 keys per warp)
     float s[8][4];
 #pragma unroll
@@ -293,7 +333,7 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
         const int r = np * 16 + ((lane >> 4) << 3) + (lane & 7);
         const int ch = ks * 2 + ((lane >> 3) & 1);
         uint32_t b0, b1, b2, b3;
-        ptx::ldsm_x4(ptx::smem_u32(sK[buf]) + swz<D>(r, ch), b0, b1, b2, b3);
+        ptx::ldsm_x4(kb + swz<D>(r, ch), b0, b1, b2, b3);
         ptx::mma_bf16_16816(s[2 * np], qa[ks], b0, b1);
         ptx::mma_bf16_16816(s[2 * np + 1], qa[ks], b2, b3);
       }
@@ -348,7 +388,7 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
         const int r = kk * 16 + (lane & 7) + (((lane >> 3) & 1) << 3);
         const int ch = dp * 2 + (lane >> 4);
         uint32_t b0, b1, b2, b3;
-        ptx::ldsm_x4_t(ptx::smem_u32(sV[buf]) + swz<D>(r, ch), b0, b1, b2, b3);
+        ptx::ldsm_x4_t(vb + swz<D>(r, ch), b0, b1, b2, b3);
         ptx::mma_bf16_16816(o[2 * dp], pa, b0, b1);
         ptx::mma_bf16_16816(o[2 * dp + 1], pa, b2, b3);
       }
@@ -376,7 +416,13 @@ __global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, con
 template <int D, int G>
 int launch_decode_t(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges,
                     cudaStream_t s) {
-  if (n_items > 0) decode_attn_kernel<D, G><<<dim3(n_items, a.Hkv), 128, 0, s>>>(a, items);
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(decode_attn_kernel<D, G>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         DecodeSmem<D>::BYTES);
+    set = true;
+  }
+  if (n_items > 0) decode_attn_kernel<D, G><<<dim3(n_items, a.Hkv), 128, DecodeSmem<D>::BYTES, s>>>(a, items);
   if (n_merges > 0) decode_merge_kernel<D, G><<<dim3(n_merges, a.Hkv), 128, 0, s>>>(a, merges);
   return GLLM_OK;
 }

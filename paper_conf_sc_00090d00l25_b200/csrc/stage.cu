@@ -443,9 +443,11 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   const int ND = S - NP;
   int split_pages = 1 << 30;
   if (ND > 0) {
-    const int64_t target = 4LL * st->num_sms;  // CTAs
+    // split long contexts so that the decode grid has >= ~8 CTAs per SM of work; a split is
+    // at least 32 pages (512 keys) so the merge pass stays negligible
+    const int64_t target = 8LL * st->num_sms;  // CTAs
     int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
-    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(8, per));
+    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(32, per));
   }
   std::vector<gllm::DecodeItem> ditems;
   std::vector<gllm::MergeItem> merges;

@@ -212,6 +212,79 @@ __global__ void __launch_bounds__(256, 1)
             }
           }
         }
+      } else if constexpr (EPI == EPI_QKV_ROPE) {
+        // The 256 columns of a tile are whole heads (D | 256); rotate-half partners (i, i + D/2)
+        // are 32-column chunks c and c + D/64 of the same head.
+        const int D = p.head_dim, half = D / 2, per_head = D / 32;
+        const int slot = row_ok ? __ldg(p.slots + row) : 0;
+        const int64_t blk = slot / p.block_size, off = slot % p.block_size;
+        uint32_t u[32];
+#pragma unroll 1
+        for (int c = 0; c < GEMM_BN / 32; ++c) {
+          const int hpos = c % per_head;  // chunk index within its head
+          if (hpos >= per_head / 2) continue;
+          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+          ptx::tmem_ld_32x32b_x32(tbase + (c + per_head / 2) * 32, u);
+          ptx::tmem_ld_wait();
+          const int col1 = n_blk * GEMM_BN + c * 32;  // first-half column of this chunk
+          if (!row_ok || col1 >= p.N) continue;
+          const int col2 = col1 + half;
+          const int i0 = hpos * 32;                   // rotation index of element 0
+          float x1[32], x2[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            x1[j] = __uint_as_float(r[j]);
+            x2[j] = __uint_as_float(u[j]);
+          }
+          if (p.bias) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {
+              x1[j] += __ldg(p.bias + col1 + j);
+              x2[j] += __ldg(p.bias + col2 + j);
+            }
+          }
+          __nv_bfloat16 *dst1, *dst2;
+          if (col1 < p.q_dim + p.kv_dim) {  // q or k: rotate
+            const float4* cs = reinterpret_cast<const float4*>(p.rope_cs + (size_t)row * half + i0);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              const float4 v = __ldg(cs + j);  // (cos, sin) of elements 2j, 2j+1
+              const float a1 = x1[2 * j], a2 = x2[2 * j], b1 = x1[2 * j + 1], b2 = x2[2 * j + 1];
+              x1[2 * j] = a1 * v.x - a2 * v.y;
+              x2[2 * j] = a2 * v.x + a1 * v.y;
+              x1[2 * j + 1] = b1 * v.z - b2 * v.w;
+              x2[2 * j + 1] = b2 * v.z + b1 * v.w;
+            }
+          }
+          if (col1 < p.q_dim) {
+            __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo;
+            dst1 = out + col1;
+            dst2 = out + col2;
+          } else {
+            const bool is_k = col1 < p.q_dim + p.kv_dim;
+            const int cc = col1 - p.q_dim - (is_k ? 0 : p.kv_dim);
+            const int h = cc / D;
+            __nv_bfloat16* base = (is_k ? p.kc : p.vc) + ((blk * p.n_kv_heads + h) * p.block_size + off) * D;
+            dst1 = base + i0;
+            dst2 = base + i0 + half;
+          }
+          uint4* d1 = reinterpret_cast<uint4*>(dst1);
+          uint4* d2 = reinterpret_cast<uint4*>(dst2);
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            uint4 w1, w2;
+            w1.x = ptx::pack_bf16(x1[q * 8 + 0], x1[q * 8 + 1]);
+            w1.y = ptx::pack_bf16(x1[q * 8 + 2], x1[q * 8 + 3]);
+            w1.z = ptx::pack_bf16(x1[q * 8 + 4], x1[q * 8 + 5]);
+            w1.w = ptx::pack_bf16(x1[q * 8 + 6], x1[q * 8 + 7]);
+            w2.x = ptx::pack_bf16(x2[q * 8 + 0], x2[q * 8 + 1]);
+            w2.y = ptx::pack_bf16(x2[q * 8 + 2], x2[q * 8 + 3]);
+            w2.z = ptx::pack_bf16(x2[q * 8 + 4], x2[q * 8 + 5]);
+            w2.w = ptx::pack_bf16(x2[q * 8 + 6], x2[q * 8 + 7]);
+            d1[q] = w1;
+            d2[q] = w2;
+          }
+        }
       } else {  // EPI_ARGMAX
         float best = -INFINITY;
         int best_i = 0x7fffffff;
@@ -313,6 +386,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
     case EPI_ADD_F32: return launch_t<EPI_ADD_F32>(a, b, args, stream, num_sms);
     case EPI_SILU_MUL: return launch_t<EPI_SILU_MUL>(a, b, args, stream, num_sms);
     case EPI_ARGMAX: return launch_t<EPI_ARGMAX>(a, b, args, stream, num_sms);
+    case EPI_QKV_ROPE: return launch_t<EPI_QKV_ROPE>(a, b, args, stream, num_sms);
   }
   return set_error(GLLM_EINVAL, "gemm: unknown epilogue");
 }

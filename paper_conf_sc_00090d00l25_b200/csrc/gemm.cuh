@@ -1,6 +1,7 @@
 // tcgen05 GEMM  Y[M,N] = X[M,K] . W[N,K]^T  with fused epilogues (internal interface).
 #pragma once
 #include <cuda.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -11,6 +12,7 @@ enum GemmEpi : int {
   EPI_ADD_F32 = 1,     // out fp32 [M, ldo] += acc          (residual add, a8 / a10)
   EPI_SILU_MUL = 2,    // out bf16 [M, ldo] = silu(gate) * up; W rows interleaved per 128 (a9)
   EPI_ARGMAX = 3,      // per (row, n-tile) max & argmax of acc -> partial buffers (a11)
+  EPI_QKV_ROPE = 4,    // fused QKV epilogue (a5+a6): (+bias) RoPE on q -> out, RoPE on k and v -> paged cache
 };
 
 struct GemmArgs {
@@ -21,6 +23,12 @@ struct GemmArgs {
   float* part_val;   // EPI_ARGMAX: [M, num_n_tiles]
   int32_t* part_idx; // EPI_ARGMAX: [M, num_n_tiles]
   int num_m_tiles, num_n_tiles;
+  // EPI_QKV_ROPE
+  const float2* rope_cs;  // [M, head_dim/2] (cos, sin) of each row's position
+  const int32_t* slots;   // [M] cache slot of each row
+  __nv_bfloat16* kc;      // [kv_blocks][n_kv_heads][block_size][head_dim]
+  __nv_bfloat16* vc;
+  int q_dim, kv_dim, head_dim, n_kv_heads, block_size;
 };
 
 constexpr int GEMM_BM = 128, GEMM_BN = 256, GEMM_BK = 64, GEMM_STAGES = 4;

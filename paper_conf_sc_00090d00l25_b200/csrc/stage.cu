@@ -436,9 +436,21 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
     if (d->sample_token_idx[k] < 0 || d->sample_token_idx[k] >= T) return gllm::set_error(GLLM_EINVAL, "bad sample idx");
   // ---------------- attention work lists (host, O(S))
   std::vector<gllm::PrefillItem> pitems;
+  std::vector<std::pair<int, int>> pcost;  // (key tiles, item index): longest CTAs first (causal tail)
   for (int i = 0; i < NP; ++i) {
-    const int rows = (d->cu_q[i + 1] - d->cu_q[i]) * G;
-    for (int r0 = 0; r0 < rows; r0 += 64) pitems.push_back({i, r0});
+    const int n = d->cu_q[i + 1] - d->cu_q[i];
+    const int rows = n * G, s0 = d->kv_len[i] - n;
+    for (int r0 = 0; r0 < rows; r0 += 64) {
+      const int last = std::min(r0 + 63, rows - 1) / G;
+      pcost.push_back({(s0 + last + 64) / 64, (int)pitems.size()});
+      pitems.push_back({i, r0});
+    }
+  }
+  std::stable_sort(pcost.begin(), pcost.end(), [](const auto& a, const auto& b) { return a.first > b.first; });
+  {
+    std::vector<gllm::PrefillItem> sorted(pitems.size());
+    for (size_t j = 0; j < pcost.size(); ++j) sorted[j] = pitems[pcost[j].second];
+    pitems.swap(sorted);
   }
   const int ND = S - NP;
   int split_pages = 1 << 30;
@@ -565,13 +577,26 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       st->last_launches += 1;
     }
     {
+      // QKV projection with RoPE and the paged KV append fused into the epilogue (a5 + a6)
       Prof p(st, s, C_QKV);
-      RC(gemm(st, st->tm_y, w.tm_qkv, gllm::EPI_STORE_BF16, T, nqkv, H, st->qkv, nqkv, w.bqkv, s));
-    }
-    {
-      Prof p(st, s, C_ROPE);
-      gllm::launch_rope_kv_append(st->qkv, T, c.n_heads, c.n_kv_heads, D, st->rope_cs, st->slots, w.kc, w.vc, bs, s);
+      gllm::GemmArgs g{};
+      g.M = T;
+      g.N = nqkv;
+      g.K = H;
+      g.out = st->qkv;
+      g.ldo = nqkv;
+      g.bias = w.bqkv;
+      g.rope_cs = st->rope_cs;
+      g.slots = st->slots;
+      g.kc = w.kc;
+      g.vc = w.vc;
+      g.q_dim = qd;
+      g.kv_dim = kd;
+      g.head_dim = D;
+      g.n_kv_heads = c.n_kv_heads;
+      g.block_size = bs;
       st->last_launches += 1;
+      RC(gllm::launch_gemm(st->tm_y, w.tm_qkv, gllm::EPI_QKV_ROPE, g, s, st->num_sms));
     }
     aa.kc = w.kc;
     aa.vc = w.vc;

@@ -68,11 +68,14 @@ class OracleRun:
         self.W = Weights(shape, dtype=dtype)
         self.cache = om.PagedCache(shape, sched_cfg.block_size, dtype)
 
-    def step(self, hidden_in=None):
+    def step(self, hidden_in=None, hin_fn=None):
         b = self.sched.build_batch()
         out = dict(batch=b)
         if b.num_tokens == 0:
             return out
+        if hin_fn is not None:
+            hidden_in = hin_fn(b)
+        out["hidden_in"] = hidden_in
         r = om.stage_forward(self.shape, self.W, self.cache, b, self.lb, self.le, hidden_in)
         out.update(r)
         return out

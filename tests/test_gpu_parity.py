@@ -23,8 +23,9 @@ def _run_pair(shape, cfg, stream, lb=0, le=None, max_ticks=None, kv_blocks=None,
     n_rows, errs, greedy = 0, [], []
     ticks = 0
     while not o.sched.done() and (max_ticks is None or ticks < max_ticks):
-        ob = o.step()
-        gb = g.step(None)
+        # stage-local parity for lb > 0: any fp32 input works; both sides get the batch's embedding rows
+        ob = o.step(hin_fn=(lambda b: o.W.embed_rows(b.token_ids)) if lb > 0 else None)
+        gb = g.step(ob.get("hidden_in"))
         ticks += 1
         b = ob["batch"]
         d = gb["desc"]
@@ -119,6 +120,17 @@ def test_c1_full_width_first_stage_layer():
     n, errs, _ = _run_pair(m, cfg, st, lb=0, le=1, max_ticks=40, kv_blocks=4000, check_kv=False)
     assert n > 1000
     assert errs.max() <= TOL_HIDDEN, errs.max()
+
+
+def test_c1_last_stage_full_vocab_lm_head():
+    # last stage of a 2-layer Llama-3-8B-shaped model: layer 1 + final norm + 128256-wide LM head with the
+    # fused argmax epilogue (501 N tiles) -> greedy ids tolerance-aware vs the oracle's fp32 logits
+    m = MODELS["C1"].with_layers(2)
+    st = make_stream("C1", m.vocab, n=40)
+    cfg = SCHED["C1"].with_(num_blocks=2000, pp_depth=1)
+    n, errs, greedy = _run_pair(m, cfg, st, lb=1, le=2, max_ticks=12, kv_blocks=2000, check_kv=False)
+    assert errs.max() <= TOL_HIDDEN, errs.max()
+    assert len(greedy) > 50 and greedy.mean() >= 0.99, (len(greedy), greedy.mean())
 
 
 def test_invalid_batch_is_einval_not_ub():

@@ -47,9 +47,28 @@ def peaks():
     return FALLBACK_PEAKS, "fallback"
 
 
-def kv_blocks_for(n_gpus):
-    # C1 uses 100000 blocks at PP=2 (~105 GB/stage); at PP=1 all 32 layers share one GPU -> 60000
-    return 60000 if n_gpus == 1 else 100000
+def kv_blocks_for(config, pp):
+    # C1 uses 100000 blocks at PP=2 (~105 GB/stage); at PP=1 all 32 layers share one GPU -> 60000.
+    # C2-C4 keep SURVEY §8(d)'s pools (their stages hold 8-12 layers).
+    if config == "C1":
+        return 60000 if pp == 1 else 100000
+    return SCHED[config].num_blocks
+
+
+def pp_of(args):
+    return args.pp or args.gpus
+
+
+def workload_config(args, sp):
+    m = MODELS[args.config]
+    PP = pp_of(args)
+    emulated = args.gpus == 1 and PP > 1
+    w = f"{args.config}: {m.name}-shaped random-init (O4), {args.config} stream, PP={PP}"
+    if emulated:
+        w += f", stage {args.stage} of {PP} run alone on 1 GPU (synthetic hidden_in)"
+    return {"workload": w, "model": f"{m.name}-shape", "pp": PP, "parallelism": f"pp{PP}",
+            "seq_len": f"mixed (stream {args.config})", "kv_blocks": sp.num_blocks,
+            "emulated_stage": args.stage if emulated else None}
 
 
 class Clocks:
@@ -170,11 +189,20 @@ def run_ours(args):
         dist.init_process_group("gloo", rank=rank, world_size=world)
         meta = dist.group.WORLD
     m = MODELS[args.config]
-    sp = SCHED[args.config].with_(pp_depth=N, num_blocks=args.kv_blocks or kv_blocks_for(N))
-    lb, le = split_layers(m.n_layers, N)[rank]
-    max_tokens = sp.maxp + -(-sp.max_seqs // N) + 64
+    PP = pp_of(args)
+    emulate = world == 1 and PP > 1          # one stage of a PP-stage deployment on this GPU
+    assert emulate or PP == N, "--pp must equal --gpus unless emulating one stage on one GPU"
+    sidx = args.stage if emulate else rank
+    sp = SCHED[args.config].with_(pp_depth=PP, num_blocks=args.kv_blocks or kv_blocks_for(args.config, PP))
+    lb, le = split_layers(m.n_layers, PP)[sidx]
+    max_tokens = sp.maxp + -(-sp.max_seqs // PP) + 64
     stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=local)
     ex = GpuExecutor(stage, dev, max_tokens, m.hidden)
+    if emulate and sidx > 0:
+        for b in ex.hin:
+            b.normal_()                       # synthetic activations arriving from stage sidx-1
+    if args.config == "C4":
+        stage.fill_kv(0xC4)                   # warm-start decode set: cache pages hold O4 values
     tr = None
     if world > 1:
         uid = [gllm.get_unique_id() if rank == 0 else None]
@@ -186,7 +214,7 @@ def run_ours(args):
     if rank == 0:
         sched = gllm.Sched(sp)
         sched.add_stream(stream)
-    pipe = Pipeline(rank, world, ex, tr, sched, meta, pp=N)
+    pipe = Pipeline(rank, world, ex, tr, sched, meta, pp=PP, stage=sidx if emulate else None)
 
     def barrier():
         torch.cuda.synchronize(dev)
@@ -292,18 +320,18 @@ def run_ours(args):
     e2e_value = e2e_tokens / (float(te[0]) * 1e-3)
 
     if rank == 0:
-        cpu = cpu_baseline(args, m, timed[0]) if (N == 1 and not args.no_cpu_baseline) else None
+        cpu = (cpu_baseline(args, m, timed[0], le - lb, le == m.n_layers)
+               if (N == 1 and not args.no_cpu_baseline) else None)
         clocks = clk.summary()
         out = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": N, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 3), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-            "config": {"workload": f"{args.config}: Llama-3-8B-shaped random-init (O4), C1 stream, PP={N}",
-                       "model": "llama3-8b-shape", "pp": N, "layers_per_stage": le - lb,
-                       "global_batch": round(tokens / args.steps, 1), "seq_len": "mixed (stream C1)",
-                       "parallelism": f"pp{N}", "token_budget": sp.maxp, "kv_blocks": sp.num_blocks,
-                       "preroll_ticks": args.preroll, "window_ticks": [int(timed[0]["tick"]), int(timed[-1]["tick"])],
-                       "l2": "inputs > L2: every step streams all stage weights (~16 GB at PP=1 >> 126 MB L2)"},
+            "config": {**workload_config(args, sp), "layers_per_stage": le - lb,
+                       "global_batch": round(tokens / args.steps, 1),
+                       "token_budget": sp.maxp, "preroll_ticks": args.preroll,
+                       "window_ticks": [int(timed[0]["tick"]), int(timed[-1]["tick"])],
+                       "l2": f"inputs > L2: every step streams all {le - lb} layers' weights (GBs >> 126 MB L2)"},
             "e2e": {"value": round(e2e_value, 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d / args.steps),
                     "d2h_bytes_per_step": int(d2h / args.steps)},
             "gpu_launches": int(launches),
@@ -355,22 +383,24 @@ def _oracle_layer_time(m, a, W, layers=1):
     return time.perf_counter() - t0
 
 
-def cpu_baseline(args, m, a):
+def cpu_baseline(args, m, a, n_layers=None, with_lm_head=True):
+    """The oracle on a bounded sample: 1 decoder layer of the batch, scaled to the stage's layers."""
     from oracle.weights import Weights
     try:
         from threadpoolctl import threadpool_info
         threads = max((p.get("num_threads", 1) for p in threadpool_info()), default=os.cpu_count())
     except Exception:
         threads = os.cpu_count()
+    n_layers = n_layers or m.n_layers
     W = Weights(m)
     sec = _oracle_layer_time(m, a, W, 1)
     T = int(a["num_tokens"])
     layer_flops = 2.0 * T * (m.hidden * (m.q_dim + 2 * m.kv_dim) + m.q_dim * m.hidden + 3 * m.hidden * m.intermediate)
-    lm_flops = 2.0 * int(np.asarray(a["sample_idx"]).shape[0]) * m.hidden * m.vocab
-    est = sec * (m.n_layers + lm_flops / layer_flops)
+    lm_flops = 2.0 * int(np.asarray(a["sample_idx"]).shape[0]) * m.hidden * m.vocab if with_lm_head else 0.0
+    est = sec * (n_layers + lm_flops / layer_flops)
     return {"value": round(T / est, 2), "unit": UNIT, "cores": int(threads), "kind": "oracle",
-            "sample": f"oracle fp32 forward of 1 of {m.n_layers} decoder layers on the first timed tick "
-                      f"(T={T}), {sec:.2f} s, scaled by layers + LM-head FLOP share",
+            "sample": f"oracle fp32 forward of 1 of {n_layers} decoder layers on the first timed tick "
+                      f"(T={T}), {sec:.2f} s, scaled by layers" + (" + LM-head FLOP share" if with_lm_head else ""),
             "host_cpus": os.cpu_count()}
 
 
@@ -383,7 +413,7 @@ def run_reference(args):
     from oracle.weights import Weights
     m = MODELS[args.config]
     N = args.gpus
-    sp = SCHED[args.config].with_(pp_depth=N, num_blocks=args.kv_blocks or kv_blocks_for(N))
+    sp = SCHED[args.config].with_(pp_depth=pp_of(args), num_blocks=args.kv_blocks or kv_blocks_for(args.config, pp_of(args)))
     st = make_stream(args.config, m.vocab)
     s = Scheduler(sp, st.requests, st.warm)
     for _ in range(args.preroll):
@@ -418,8 +448,7 @@ def run_reference(args):
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 2), "unit": UNIT, "n_gpus": N,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_sec / max(args.steps, 1) * 1e3, 1),
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-           "config": {"workload": f"{args.config}: Llama-3-8B-shaped random-init (O4), C1 stream, PP={N}",
-                      "model": "llama3-8b-shape", "pp": N, "parallelism": f"pp{N}", "kv_blocks": sp.num_blocks},
+           "config": workload_config(args, sp),
            "cpu_baseline": {"value": round(v, 2), "unit": UNIT, "cores": int(threads), "kind": "oracle",
                             "sample": sample_desc},
            "e2e": {"value": round(v, 2), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -433,10 +462,16 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C1")
-    ap.add_argument("--preroll", type=int, default=400)
+    ap.add_argument("--preroll", type=int, default=None,
+                    help="ticks run before the window (default: the config's window start)")
+    ap.add_argument("--pp", type=int, default=0, help="pipeline depth (default --gpus)")
+    ap.add_argument("--stage", type=int, default=0, help="with --gpus 1 --pp N: which stage to run")
     ap.add_argument("--kv-blocks", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
+    if args.preroll is None:
+        from workloads.configs import STREAMS
+        args.preroll = int(STREAMS[args.config].get("window", (400, None))[0])
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":

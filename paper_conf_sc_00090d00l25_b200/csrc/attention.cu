@@ -234,185 +234,6 @@ __global__ void __launch_bounds__(128) decode_merge_kernel(const AttnArgs a, con
   }
 }
 
-// ------------------------------------------------------------------ prefill
-// CTA = 64 flattened (token, group head) rows of one chunk x one kv head; 4 warps x 16 rows.
-// K/V tiles of 64 keys (4 pages) double-buffered in SMEM with cp.async; S = Q K^T and
-// O += P V on mma.sync m16n8k16 (bf16 in, fp32 accumulate); online softmax in registers.
-template <int D>
-struct PrefillSmem {
-  static constexpr int ROW_BYTES = D * 2;
-  static constexpr int TILE_BYTES = 64 * ROW_BYTES;
-  static constexpr int BYTES = 5 * TILE_BYTES;  // Q + 2 x (K, V)
-};
-
-template <int D>
-__global__ void __launch_bounds__(128) prefill_attn_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
-  constexpr int NCH = D / 8;  // 16-byte chunks per row
-  constexpr int TB = PrefillSmem<D>::TILE_BYTES;
-  extern __shared__ __align__(128) uint8_t smem[];
-  const uint32_t sQ = ptx::smem_u32(smem);
-  // buffer b: K at sQ + (1 + 2b) TB, V at sQ + (2 + 2b) TB
-
-  const PrefillItem it = items[blockIdx.x];
-  const int kvh = blockIdx.y;
-  const int G = a.Hq / a.Hkv;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int t0 = a.cu_q[it.seq];
-  const int c = a.cu_q[it.seq + 1] - t0;
-  const int s0 = a.kv_len[it.seq] - c;  // chunk offset
-  const int nrows = c * G;
-  const int row_last = min(it.row0 + 63, nrows - 1);
-  const int max_pos = s0 + row_last / G;
-  const int n_kt = (max_pos + 64) / 64;  // key tiles covering [0, max_pos]
-  const int nblk_seq = (a.kv_len[it.seq] + 15) / 16;
-  const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
-  const float sl2 = LOG2E * rsqrtf((float)D);
-
-  // ---- Q tile -> SMEM (rows beyond the chunk are clamped to the last row; never stored)
-  for (int idx = threadIdx.x; idx < 64 * NCH; idx += 128) {
-    const int r = idx / NCH, ch = idx % NCH;
-    const int rr = min(it.row0 + r, nrows - 1);
-    const int tok = rr / G, h = kvh * G + rr % G;
-    const __nv_bfloat16* src = a.q + (size_t)(t0 + tok) * a.q_stride + (size_t)h * D + ch * 8;
-    ptx::cp_async16(sQ + swz<D>(r, ch), src, true);
-  }
-  auto load_kv = [&](int kt, int buf) {
-    const uint32_t kb = sQ + (1 + 2 * buf) * TB, vb = kb + TB;
-    for (int idx = threadIdx.x; idx < 64 * NCH; idx += 128) {
-      const int r = idx / NCH, ch = idx % NCH;
-      const int key = kt * 64 + r;
-      const int blk = key >> 4;
-      const bool ok = blk < nblk_seq;
-      const size_t page = ok ? (size_t)bt[blk] : 0;
-      const size_t off = ((page * a.Hkv + kvh) * 16 + (key & 15)) * D + ch * 8;
-      ptx::cp_async16(kb + swz<D>(r, ch), a.kc + off, ok);
-      ptx::cp_async16(vb + swz<D>(r, ch), a.vc + off, ok);
-    }
-  };
-  load_kv(0, 0);
-  ptx::cp_async_commit();
-
-  // per-thread rows of the m16n8 fragments: g and g + 8 of this warp's 16 rows
-  const int g = lane >> 2, tq = lane & 3;
-  int pos_r[2];
-#pragma unroll
-  for (int hr = 0; hr < 2; ++hr) {
-    const int rr = min(it.row0 + warp * 16 + g + hr * 8, nrows - 1);
-    pos_r[hr] = s0 + rr / G;
-  }
-  const int pos_min_warp = s0 + min(it.row0 + warp * 16, nrows - 1) / G;
-
-  uint32_t qa[D / 16][4];
-  float o[D / 8][4];
-#pragma unroll
-  for (int n = 0; n < D / 8; ++n) o[n][0] = o[n][1] = o[n][2] = o[n][3] = 0.f;
-  float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
-
-  for (int kt = 0; kt < n_kt; ++kt) {
-    if (kt + 1 < n_kt) load_kv(kt + 1, (kt + 1) & 1);
-    ptx::cp_async_commit();
-    ptx::cp_async_wait<1>();
-    __syncthreads();
-    if (kt == 0) {
-#pragma unroll
-      for (int ks = 0; ks < D / 16; ++ks) {
-        const int r = warp * 16 + (lane & 15);
-        const int ch = ks * 2 + (lane >> 4);
-        ptx::ldsm_x4(sQ + swz<D>(r, ch), qa[ks][0], qa[ks][1], qa[ks][2], qa[ks][3]);
-      }
-    }
-    const uint32_t kb = sQ + (1 + 2 * (kt & 1)) * TB, vb = kb + TB;
-    // ---- S = Q K^T  (16 rows x 64 keys per warp)
-    float s[8][4];
-#pragma unroll
-    for (int n = 0; n < 8; ++n) s[n][0] = s[n][1] = s[n][2] = s[n][3] = 0.f;
-#pragma unroll
-    for (int ks = 0; ks < D / 16; ++ks) {
-#pragma unroll
-      for (int np = 0; np < 4; ++np) {
-        const int r = np * 16 + ((lane >> 4) << 3) + (lane & 7);
-        const int ch = ks * 2 + ((lane >> 3) & 1);
-        uint32_t b0, b1, b2, b3;
-        ptx::ldsm_x4(kb + swz<D>(r, ch), b0, b1, b2, b3);
-        ptx::mma_bf16_16816(s[2 * np], qa[ks], b0, b1);
-        ptx::mma_bf16_16816(s[2 * np + 1], qa[ks], b2, b3);
-      }
-    }
-    // ---- scale, causal mask, online softmax
-    const bool need_mask = kt * 64 + 63 > pos_min_warp;
-#pragma unroll
-    for (int n = 0; n < 8; ++n)
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int key = kt * 64 + n * 8 + 2 * tq + (e & 1);
-        const int hr = e >> 1;
-        s[n][e] = (need_mask && key > pos_r[hr]) ? -INFINITY : s[n][e] * sl2;
-      }
-    float corr[2];
-#pragma unroll
-    for (int hr = 0; hr < 2; ++hr) {
-      float mx = -INFINITY;
-#pragma unroll
-      for (int n = 0; n < 8; ++n) mx = fmaxf(mx, fmaxf(s[n][2 * hr], s[n][2 * hr + 1]));
-      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
-      mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-      const float mn = fmaxf(mrow[hr], mx);
-      corr[hr] = exp2f(mrow[hr] - mn);
-      mrow[hr] = mn;
-      float sum = 0.f;
-#pragma unroll
-      for (int n = 0; n < 8; ++n) {
-        s[n][2 * hr] = exp2f(s[n][2 * hr] - mn);
-        s[n][2 * hr + 1] = exp2f(s[n][2 * hr + 1] - mn);
-        sum += s[n][2 * hr] + s[n][2 * hr + 1];
-      }
-      lrow[hr] = lrow[hr] * corr[hr] + sum;
-    }
-#pragma unroll
-    for (int n = 0; n < D / 8; ++n) {
-      o[n][0] *= corr[0];
-      o[n][1] *= corr[0];
-      o[n][2] *= corr[1];
-      o[n][3] *= corr[1];
-    }
-    // ---- O += P V
-#pragma unroll
-    for (int kk = 0; kk < 4; ++kk) {
-      uint32_t pa[4];
-      pa[0] = ptx::pack_bf16(s[2 * kk][0], s[2 * kk][1]);
-      pa[1] = ptx::pack_bf16(s[2 * kk][2], s[2 * kk][3]);
-      pa[2] = ptx::pack_bf16(s[2 * kk + 1][0], s[2 * kk + 1][1]);
-      pa[3] = ptx::pack_bf16(s[2 * kk + 1][2], s[2 * kk + 1][3]);
-#pragma unroll
-      for (int dp = 0; dp < D / 16; ++dp) {
-        const int r = kk * 16 + (lane & 7) + (((lane >> 3) & 1) << 3);
-        const int ch = dp * 2 + (lane >> 4);
-        uint32_t b0, b1, b2, b3;
-        ptx::ldsm_x4_t(vb + swz<D>(r, ch), b0, b1, b2, b3);
-        ptx::mma_bf16_16816(o[2 * dp], pa, b0, b1);
-        ptx::mma_bf16_16816(o[2 * dp + 1], pa, b2, b3);
-      }
-    }
-    __syncthreads();
-  }
-  // ---- normalise and store
-#pragma unroll
-  for (int hr = 0; hr < 2; ++hr) {
-    float lt = lrow[hr];
-    lt += __shfl_xor_sync(0xffffffffu, lt, 1);
-    lt += __shfl_xor_sync(0xffffffffu, lt, 2);
-    const float inv = 1.f / lt;
-    const int rr = it.row0 + warp * 16 + g + hr * 8;
-    if (rr < nrows) {
-      const int tok = rr / G, h = kvh * G + rr % G;
-      __nv_bfloat16* dst = a.out + (size_t)(t0 + tok) * a.Hq * D + (size_t)h * D;
-#pragma unroll
-      for (int n = 0; n < D / 8; ++n)
-        *reinterpret_cast<uint32_t*>(dst + n * 8 + 2 * tq) = ptx::pack_bf16(o[n][2 * hr] * inv, o[n][2 * hr + 1] * inv);
-    }
-  }
-}
-
 template <int D, int G>
 int launch_decode_t(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges,
                     cudaStream_t s) {
@@ -441,25 +262,6 @@ int launch_decode_d(const AttnArgs& a, const DecodeItem* items, int n_items, con
 }
 
 }  // namespace
-
-int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
-  if (n_items <= 0) return GLLM_OK;
-  if (a.D == 128) {
-    static bool set = false;
-    if (!set) {
-      cudaFuncSetAttribute(prefill_attn_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           PrefillSmem<128>::BYTES);
-      set = true;
-    }
-    prefill_attn_kernel<128><<<dim3(n_items, a.Hkv), 128, PrefillSmem<128>::BYTES, s>>>(a, items);
-  } else if (a.D == 64) {
-    prefill_attn_kernel<64><<<dim3(n_items, a.Hkv), 128, PrefillSmem<64>::BYTES, s>>>(a, items);
-  } else {
-    return set_error(GLLM_EINVAL, "prefill attention: head_dim %d unsupported", a.D);
-  }
-  cudaError_t e = cudaGetLastError();
-  return e == cudaSuccess ? GLLM_OK : set_error(GLLM_ECUDA, "prefill attention launch: %s", cudaGetErrorString(e));
-}
 
 int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
                             int n_merges, cudaStream_t s) {

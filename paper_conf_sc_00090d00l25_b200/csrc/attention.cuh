@@ -6,7 +6,7 @@
 
 namespace gllm {
 
-// work item of the prefill kernel: chunk `seq`, flattened (token, group-head) rows [row0, row0+64)
+// work item of the prefill kernel: chunk `seq`, flattened (token, group-head) rows [row0, row0+rows_per_item)
 struct PrefillItem {
   int32_t seq, row0;
 };
@@ -35,6 +35,8 @@ struct AttnArgs {
   int split_len;       // decode keys per split (multiple of 16)
 };
 
+// flattened (token, group-head) rows per prefill work item
+int prefill_rows_per_item();
 int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
 int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
                             int n_merges, cudaStream_t s);

@@ -440,8 +440,9 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   for (int i = 0; i < NP; ++i) {
     const int n = d->cu_q[i + 1] - d->cu_q[i];
     const int rows = n * G, s0 = d->kv_len[i] - n;
-    for (int r0 = 0; r0 < rows; r0 += 64) {
-      const int last = std::min(r0 + 63, rows - 1) / G;
+    const int rpi = gllm::prefill_rows_per_item();
+    for (int r0 = 0; r0 < rows; r0 += rpi) {
+      const int last = std::min(r0 + rpi - 1, rows - 1) / G;
       pcost.push_back({(s0 + last + 64) / 64, (int)pitems.size()});
       pitems.push_back({i, r0});
     }

@@ -141,15 +141,30 @@ class NcclTransport:
         ex.send_ev[i].record(ex.comm)
 
 
+class _NullTransport:
+    """Stage emulation on one GPU: the hidden input buffers keep synthetic data, nothing is sent."""
+
+    def recv(self, k, T):
+        pass
+
+    def send(self, k, T):
+        pass
+
+
 class Pipeline:
     """The per-rank tick loop.  `meta` is a torch.distributed group (gloo) for metadata and
     sampled ids; None when world == 1."""
 
-    def __init__(self, rank, world, executor, transport=None, sched=None, meta=None, pp=None):
+    def __init__(self, rank, world, executor, transport=None, sched=None, meta=None, pp=None, stage=None):
+        """`stage` (emulation, world == 1): run only pipeline stage `stage` of `pp` on this GPU, with
+        synthetic hidden inputs -- the per-stage work of a PP=pp deployment measured on one GPU."""
         self.rank, self.world = rank, world
         self.ex, self.tr, self.sched, self.meta = executor, transport, sched, meta
         self.pp = pp or world
-        self.is_first, self.is_last = rank == 0, rank == world - 1
+        s, n = (rank, world) if stage is None else (stage, self.pp)
+        self.is_first, self.is_last = s == 0, s == n - 1
+        if self.tr is None and not (self.is_first and self.is_last) and world == 1:
+            self.tr = _NullTransport()
         self.pending_samples = {}   # tick -> ns (last stage)
         self._expect = {}           # tick -> ns (driver): sampled ids owed by the last stage
         self.tokens = 0
@@ -185,7 +200,7 @@ class Pipeline:
         if ns == 0:
             return np.zeros(0, np.int32)
         if self.world == 1:
-            return self.ex.sampled(j, ns)
+            return self.ex.sampled(j, ns) if self.is_last else None
         import torch
         import torch.distributed as dist
         t = torch.empty(ns, dtype=torch.int32)

@@ -122,6 +122,19 @@ def test_c1_full_width_first_stage_layer():
     assert errs.max() <= TOL_HIDDEN, errs.max()
 
 
+@pytest.mark.parametrize("cfg_name,n_req,ticks,kvb", [("C2", 60, 14, 3000), ("C4", 30, 10, 3000)])
+def test_full_width_other_shapes_stage_local(cfg_name, n_req, ticks, kvb):
+    # C2 = Qwen2.5-14B shapes (H 5120, GQA group 5, q/k/v bias, theta 1e6); C4 = Llama-3-70B shapes
+    # (H 8192, I 28672, GQA group 8): one middle-stage layer fed the batch's embedding rows
+    # (stage-local parity), on a stream prefix of the config.
+    m = MODELS[cfg_name].with_layers(4)
+    st = make_stream("C1", m.vocab, n=n_req)          # cold stream of C1 lengths (C4's warm set is separate)
+    cfg = SCHED[cfg_name].with_(num_blocks=kvb, pp_depth=2)
+    n, errs, _ = _run_pair(m, cfg, st, lb=1, le=2, max_ticks=ticks, kv_blocks=kvb, check_kv=False)
+    assert n > 300
+    assert errs.max() <= TOL_HIDDEN, errs.max()
+
+
 def test_c1_last_stage_full_vocab_lm_head():
     # last stage of a 2-layer Llama-3-8B-shaped model: layer 1 + final norm + 128256-wide LM head with the
     # fused argmax epilogue (501 N tiles) -> greedy ids tolerance-aware vs the oracle's fp32 logits

@@ -117,7 +117,10 @@ class Clocks:
 
 # ---------------------------------------------------------------------------- work model
 def batch_work(m, a, n_layers, is_last):
-    """Algorithmic FLOPs / bytes of one micro-batch per kernel category."""
+    """Algorithmic (FLOPs, bytes) of one micro-batch per kernel category.
+
+    GEMM bytes = weights read once + activations in + outputs out; whichever of FLOPs / Pi
+    and bytes / beta is larger decides the bound (T below the ridge ~205 tokens -> HBM)."""
     T = int(a["num_tokens"])
     H, qd, kd, I, V = m.hidden, m.q_dim, m.kv_dim, m.intermediate, m.vocab
     ns = int(np.asarray(a["sample_idx"]).shape[0])
@@ -131,37 +134,41 @@ def batch_work(m, a, n_layers, is_last):
         pairs += c * s + c * (c + 1) // 2
     dec_keys = int(kvl[NP:].sum()) if kvl.shape[0] > NP else 0
     nd = kvl.shape[0] - NP
+    L = n_layers
+
+    def gemm(M, N, K, out_bytes):
+        return (2.0 * M * N * K * L, float((N * K * 2 + M * K * 2 + M * N * out_bytes) * L))
     w = {
-        "qkv_gemm": ("tensor", 2.0 * T * H * (qd + 2 * kd) * n_layers),
-        "o_gemm": ("tensor", 2.0 * T * qd * H * n_layers),
-        "gate_up_gemm": ("tensor", 2.0 * T * H * 2 * I * n_layers),
-        "down_gemm": ("tensor", 2.0 * T * I * H * n_layers),
-        "prefill_attn": ("tensor", 4.0 * m.n_heads * m.head_dim * pairs * n_layers),
-        "decode_attn": ("hbm", float((dec_keys * kvb + nd * qd * 2 * 2) * n_layers)),
-        "rope_kv_append": ("hbm", float(T * ((qd + 2 * kd) * 2 + qd * 2 + kvb) * n_layers)),
-        "rmsnorm": ("hbm", float(2 * T * H * (4 + 2) * n_layers)),
+        "qkv_gemm": gemm(T, qd + 2 * kd, H, 2),
+        "o_gemm": gemm(T, H, qd, 8),            # fp32 residual read + write
+        "gate_up_gemm": gemm(T, 2 * I, H, 1),   # bf16 SiLU*up output is half the columns
+        "down_gemm": gemm(T, H, I, 8),
+        "prefill_attn": (4.0 * m.n_heads * m.head_dim * pairs * L, float(T * qd * 4 * L)),
+        "decode_attn": (4.0 * m.n_heads * m.head_dim * dec_keys * L, float((dec_keys * kvb + nd * qd * 2 * 2) * L)),
+        "rope_kv_append": (0.0, float(T * ((qd + 2 * kd) * 2 + qd * 2 + kvb) * L)),
+        "rmsnorm": (0.0, float(2 * T * H * (4 + 2) * L)),
     }
     if is_last:
-        w["lm_head"] = ("tensor", 2.0 * ns * H * V)
+        w["lm_head"] = (2.0 * ns * H * V, float(V * H * 2 + ns * H * 2))
     return w
 
 
 def roofline_report(timing_ms, work, launches, pk):
-    """Per category achieved/peak; the dominant (largest-time) kernel is the headline."""
+    """Per category: roofline time = max(FLOPs / Pi, bytes / beta) decides the bound; achieved is
+    in the bound's unit.  The dominant (largest-time) kernel is the headline."""
     kern = {}
+    pi = float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"])) * 1e12
+    beta = float(pk["hbm_gbs"]) * 1e9
     for name, ms in timing_ms.items():
         if name in ("total", "other") or name not in work or ms <= 0:
             continue
-        bound, amount = work[name]
-        if bound == "tensor":
-            ach = amount / (ms * 1e-3) / 1e12
-            peak = float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"]))
-            unit = "TFLOP/s"
+        flops, nbytes = work[name]
+        sec = ms * 1e-3
+        if flops / pi >= nbytes / beta:
+            bound, ach, peak, unit = "tensor", flops / sec / 1e12, pi / 1e12, "TFLOP/s"
         else:
-            ach = amount / (ms * 1e-3) / 1e9
-            peak = float(pk["hbm_gbs"])
-            unit = "GB/s"
-        kern[name] = {"bound": bound, "achieved": round(ach, 1), "peak": peak, "unit": unit,
+            bound, ach, peak, unit = "hbm", nbytes / sec / 1e9, beta / 1e9, "GB/s"
+        kern[name] = {"bound": bound, "achieved": round(ach, 1), "peak": round(peak, 1), "unit": unit,
                       "frac": round(ach / peak, 4), "ms": round(ms, 3),
                       "share": round(ms / max(timing_ms.get("total", ms), 1e-9), 4)}
     dom = max(kern, key=lambda k: kern[k]["ms"]) if kern else None
@@ -285,8 +292,9 @@ def run_ours(args):
     # roofline of this rank's dominant kernel (rank 0 reports its own stage)
     work = {}
     for a in timed:
-        for kname, (bound, amt) in batch_work(m, a, le - lb, le == m.n_layers).items():
-            work[kname] = (bound, work.get(kname, (bound, 0.0))[1] + amt)
+        for kname, (fl, by) in batch_work(m, a, le - lb, le == m.n_layers).items():
+            f0, b0 = work.get(kname, (0.0, 0.0))
+            work[kname] = (f0 + fl, b0 + by)
     pk, pk_src = peaks()
     dom, kern = roofline_report(timing, work, launches, pk)
     traffic = None

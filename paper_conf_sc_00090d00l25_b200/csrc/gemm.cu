@@ -2,11 +2,18 @@
 //
 //   Y[M,N] = X[M,K] . W[N,K]^T      X = activations (bf16, K-major), W = weights (bf16, K-major)
 //
-// Tile 128 x 256 x 64, 4-stage TMA -> SMEM ring (128-byte swizzle), one
-// elected thread issues tcgen05.mma (M=128, N=256, K=16) into a double-
-// buffered fp32 TMEM accumulator (2 x 256 columns), 4 epilogue warps drain
-// TMEM with tcgen05.ld and apply the fused epilogue (bias, fp32 residual add,
-// SiLU*up, or a row-wise argmax for the greedy LM head).  Warp roles:
+// Two variants of one kernel template:
+//   CG = 2 (default for >= ~1 wave of work): a CTA pair (cluster of 2 on one TPC) computes a
+//          256 x 256 tile with tcgen05.mma.cta_group::2 (M=256, N=256, K=16); each CTA loads its
+//          128 rows of A and 128 of the 256 rows of B (halving SMEM/L2 operand traffic per
+//          FLOP), 6-stage TMA ring of 32 KB stages, the leader CTA issues the MMAs and commits
+//          to both CTAs' barriers (multicast); each CTA drains its own 128 x 256 TMEM accumulator.
+//   CG = 1: one CTA per 128 x 256 tile (tcgen05.mma.cta_group::1, M=128), 4-stage ring of 48 KB
+//          stages; used for small T, where it also supports stream-K (equal k-block ranges per
+//          CTA, partial tiles combined with fp32 vector reductions or through a workspace).
+// Both: single-thread MMA issue, double-buffered fp32 TMEM accumulator (2 x 256 columns), 4
+// epilogue warps (tcgen05.ld) with the fused epilogues: bias, fp32 residual add, SiLU*up,
+// RoPE + paged KV append, row argmax for the greedy LM head.
 //   warp 0: TMA producer      warp 1: MMA issuer      warp 2: TMEM allocator
 //   warps 4-7: epilogue (warp 4+i reads TMEM lanes 32i..32i+31)
 #include <cudaTypedefs.h>
@@ -20,73 +27,394 @@
 
 namespace gllm {
 
+int g_force_cg = 0;
+
 namespace {
 
-constexpr int A_BYTES = GEMM_BM * GEMM_BK * 2;
-constexpr int B_BYTES = GEMM_BN * GEMM_BK * 2;
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int SMEM_BYTES = GEMM_STAGES * STAGE_BYTES + 1024 + 256;
 constexpr int TMEM_COLS = 2 * GEMM_BN;
+
+template <int CG>
+struct Cfg {
+  static constexpr int B_ROWS = GEMM_BN / CG;  // rows of the B tile loaded by each CTA
+  static constexpr int A_BYTES = GEMM_BM * GEMM_BK * 2;
+  static constexpr int B_BYTES = B_ROWS * GEMM_BK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = CG == 2 ? 6 : GEMM_STAGES;
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int TILE_M = GEMM_BM * CG;  // rows of one (cluster) tile
+};
 
 __device__ __forceinline__ float silu_f(float x) { return x / (1.0f + __expf(-x)); }
 
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// TMA 2-D load of this CTA's half of a 2-CTA tile; completion bytes land on the LEADER's barrier
+// (peer bit of the shared::cluster address cleared).
+__device__ __forceinline__ void tma_load_2d_cg2(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int32_t c0,
+                                                int32_t c1) {
+  const uint32_t mbar = ptx::smem_u32(bar) & 0xFEFFFFFFu;
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
+      "%4}], [%2];" ::"r"(ptx::smem_u32(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(mbar), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void umma_bf16_cg2(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                              uint32_t accumulate) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// commit of the leader's MMAs, arriving on the barrier at the same offset in both CTAs
+__device__ __forceinline__ void umma_commit_cg2(uint64_t* bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          ptx::smem_u32(bar)),
+      "h"((uint16_t)3)
+      : "memory");
+}
+// arrive on the leader CTA's copy of a barrier (from either CTA of the pair)
+__device__ __forceinline__ void mbar_arrive_leader(uint64_t* bar) {
+  asm volatile(
+      "{\n"
+      ".reg .b32 ra;\n"
+      "mapa.shared::cluster.u32 ra, %0, 0;\n"
+      "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n"
+      "}\n" ::"r"(ptx::smem_u32(bar))
+      : "memory");
+}
+template <int CG>
+__device__ __forceinline__ void tmem_alloc_cg(uint32_t* dst, uint32_t ncols) {
+  if constexpr (CG == 1) {
+    ptx::tmem_alloc(dst, ncols);
+    ptx::tmem_relinquish();
+  } else {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(ptx::smem_u32(dst)),
+                 "r"(ncols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+}
+template <int CG>
+__device__ __forceinline__ void tmem_dealloc_cg(uint32_t taddr, uint32_t ncols) {
+  if constexpr (CG == 1)
+    ptx::tmem_dealloc(taddr, ncols);
+  else
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+
+// Job iterator shared by the three warp roles (each role walks the same sequence).  `unit` is
+// the CTA (CG=1) or the cluster (CG=2) index, `nunits` their count.
+struct Jobs {
+  int mode, ntiles, nk, per, total, unit, nunits;
+  int it, u, u1;
+  __device__ void init(const GemmArgs& p, int unit_, int nunits_, int num_m) {
+    mode = p.streamk;
+    ntiles = num_m * p.num_n_tiles;
+    nk = p.K / GEMM_BK;
+    per = p.units_per_cta;
+    total = ntiles * nk;
+    unit = unit_;
+    nunits = nunits_;
+    it = 0;
+    u = unit * per;
+    u1 = min(total, u + per);
+  }
+  __device__ bool next(int& tile, int& kb0, int& kb1) {
+    if (mode == 0) {
+      tile = unit + it * nunits;
+      ++it;
+      kb0 = 0;
+      kb1 = nk;
+      return tile < ntiles;
+    }
+    if (u >= u1) return false;
+    tile = u / nk;
+    kb0 = u - tile * nk;
+    kb1 = min(nk, kb0 + (u1 - u));
+    u += kb1 - kb0;
+    return true;
+  }
+};
+
+__device__ __forceinline__ void store_bf16x32(__nv_bfloat16* dst, const float* v) {
+  uint4* d = reinterpret_cast<uint4*>(dst);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint4 w;
+    w.x = ptx::pack_bf16(v[q * 8 + 0], v[q * 8 + 1]);
+    w.y = ptx::pack_bf16(v[q * 8 + 2], v[q * 8 + 3]);
+    w.z = ptx::pack_bf16(v[q * 8 + 4], v[q * 8 + 5]);
+    w.w = ptx::pack_bf16(v[q * 8 + 6], v[q * 8 + 7]);
+    d[q] = w;
+  }
+}
+
+// 32 consecutive fp32 reductions as 8 vector reductions (red.global.add.v4.f32, sm_90+)
+__device__ __forceinline__ void atomic_add_f32x32(float* dst, const uint32_t (&r)[32]) {
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(dst + 4 * q), "r"(r[q * 4 + 0]),
+                 "r"(r[q * 4 + 1]), "r"(r[q * 4 + 2]), "r"(r[q * 4 + 3])
+                 : "memory");
+}
+
+// RoPE (rotate-half) of a 32-element chunk pair (x1 = dims i0.., x2 = dims i0+D/2..) with the
+// row's (cos, sin) table, then stores to q (row of `out`), or to the paged K / V cache.
+__device__ __forceinline__ void qkv_rope_store(const GemmArgs& p, int row, int col1, int i0, float* x1, float* x2,
+                                               int64_t blk, int64_t off) {
+  const int D = p.head_dim, half = D / 2;
+  if (col1 < p.q_dim + p.kv_dim) {
+    const float4* cs = reinterpret_cast<const float4*>(p.rope_cs + (size_t)row * half + i0);
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+      const float4 v = __ldg(cs + j);  // (cos, sin) of elements 2j, 2j+1
+      const float a1 = x1[2 * j], a2 = x2[2 * j], b1 = x1[2 * j + 1], b2 = x2[2 * j + 1];
+      x1[2 * j] = a1 * v.x - a2 * v.y;
+      x2[2 * j] = a2 * v.x + a1 * v.y;
+      x1[2 * j + 1] = b1 * v.z - b2 * v.w;
+      x2[2 * j + 1] = b2 * v.z + b1 * v.w;
+    }
+  }
+  __nv_bfloat16 *dst1, *dst2;
+  if (col1 < p.q_dim) {
+    __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo;
+    dst1 = out + col1;
+    dst2 = out + col1 + half;
+  } else {
+    const bool is_k = col1 < p.q_dim + p.kv_dim;
+    const int cc = col1 - p.q_dim - (is_k ? 0 : p.kv_dim);
+    const int h = cc / D;
+    __nv_bfloat16* base = (is_k ? p.kc : p.vc) + ((blk * p.n_kv_heads + h) * p.block_size + off) * D;
+    dst1 = base + i0;
+    dst2 = base + i0 + half;
+  }
+  store_bf16x32(dst1, x1);
+  store_bf16x32(dst2, x2);
+}
+
+// One warp's 32 rows of one 256-column accumulator tile: wait for the MMAs (tfull), drain TMEM,
+// apply the fused epilogue.  `partial`: stream-K segment, combine atomically.
 template <int EPI>
+__device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
+                                              uint64_t* tfull_bar, uint32_t parity) {
+  const bool row_ok = row < p.M;
+  uint32_t r[32];
+  auto wait_acc = [&]() {
+    ptx::mbar_wait(tfull_bar, parity);
+    ptx::tc_fence_after();
+  };
+  if (p.ws != nullptr) {
+    // workspace mode (stream-K for non-additive epilogues): every segment adds into ws
+    wait_acc();
+#pragma unroll 1
+    for (int c = 0; c < GEMM_BN / 32; ++c) {
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+      ptx::tmem_ld_wait();
+      const int col0 = n_blk * GEMM_BN + c * 32;
+      if (row_ok && col0 < p.N) atomic_add_f32x32(p.ws + (size_t)row * p.N + col0, r);
+    }
+  } else if constexpr (EPI == EPI_STORE_BF16) {
+    wait_acc();
+    __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
+#pragma unroll 1
+    for (int c = 0; c < GEMM_BN / 32; ++c) {
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+      ptx::tmem_ld_wait();
+      const int col0 = n_blk * GEMM_BN + c * 32;
+      if (row_ok && col0 < p.N) {
+        float v[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]) + (p.bias ? __ldg(p.bias + col0 + j) : 0.f);
+        store_bf16x32(out + (size_t)row * p.ldo + col0, v);
+      }
+    }
+  } else if constexpr (EPI == EPI_ADD_F32) {
+    float* rowp = reinterpret_cast<float*>(p.out) + (size_t)row * p.ldo + n_blk * GEMM_BN;
+    const bool ok = row_ok && n_blk * GEMM_BN < p.N;
+    // residual chunks are double-buffered in registers: chunk c+1 is loaded while chunk c is
+    // added, and chunk 0 is in flight while the MMAs finish
+    float4 xa[8], xb[8];
+    if (ok && !partial) {
+#pragma unroll
+      for (int q = 0; q < 8; ++q) xa[q] = reinterpret_cast<const float4*>(rowp)[q];
+    }
+    wait_acc();
+#pragma unroll
+    for (int c = 0; c < GEMM_BN / 32; ++c) {
+      if (ok && !partial && c + 1 < GEMM_BN / 32) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) xb[q] = reinterpret_cast<const float4*>(rowp + (c + 1) * 32)[q];
+      }
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+      ptx::tmem_ld_wait();
+      if (ok) {
+        if (partial) {
+          atomic_add_f32x32(rowp + c * 32, r);
+        } else {
+          float4* dst = reinterpret_cast<float4*>(rowp + c * 32);
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            float4 x = xa[q];
+            x.x += __uint_as_float(r[q * 4 + 0]);
+            x.y += __uint_as_float(r[q * 4 + 1]);
+            x.z += __uint_as_float(r[q * 4 + 2]);
+            x.w += __uint_as_float(r[q * 4 + 3]);
+            dst[q] = x;
+            xa[q] = xb[q];
+          }
+        }
+      }
+    }
+  } else if constexpr (EPI == EPI_SILU_MUL) {
+    wait_acc();
+    __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
+    uint32_t u[32];
+#pragma unroll 1
+    for (int c = 0; c < GEMM_BN / 64; ++c) {
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);                // gate columns
+      ptx::tmem_ld_32x32b_x32(tbase + GEMM_BN / 2 + c * 32, u);  // up columns
+      ptx::tmem_ld_wait();
+      const int col0 = n_blk * (GEMM_BN / 2) + c * 32;
+      if (row_ok && col0 < p.N / 2) {
+        float h[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) h[j] = silu_f(__uint_as_float(r[j])) * __uint_as_float(u[j]);
+        store_bf16x32(out + (size_t)row * p.ldo + col0, h);
+      }
+    }
+  } else if constexpr (EPI == EPI_QKV_ROPE) {
+    // The 256 columns of a tile are whole heads (D | 256); rotate-half partners (i, i + D/2)
+    // are 32-column chunks c and c + D/64 of the same head.
+    const int per_head = p.head_dim / 32;
+    const int slot = row_ok ? __ldg(p.slots + row) : 0;
+    const int64_t blk = slot / p.block_size, off = slot % p.block_size;
+    uint32_t u[32];
+    wait_acc();
+#pragma unroll 1
+    for (int c = 0; c < GEMM_BN / 32; ++c) {
+      const int hpos = c % per_head;
+      if (hpos >= per_head / 2) continue;
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+      ptx::tmem_ld_32x32b_x32(tbase + (c + per_head / 2) * 32, u);
+      ptx::tmem_ld_wait();
+      const int col1 = n_blk * GEMM_BN + c * 32;
+      if (!row_ok || col1 >= p.N) continue;
+      float x1[32], x2[32];
+#pragma unroll
+      for (int j = 0; j < 32; ++j) {
+        x1[j] = __uint_as_float(r[j]) + (p.bias ? __ldg(p.bias + col1 + j) : 0.f);
+        x2[j] = __uint_as_float(u[j]) + (p.bias ? __ldg(p.bias + col1 + p.head_dim / 2 + j) : 0.f);
+      }
+      qkv_rope_store(p, row, col1, hpos * 32, x1, x2, blk, off);
+    }
+  } else {  // EPI_ARGMAX
+    wait_acc();
+    float best = -INFINITY;
+    int best_i = 0x7fffffff;
+#pragma unroll 1
+    for (int c = 0; c < GEMM_BN / 32; ++c) {
+      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+      ptx::tmem_ld_wait();
+      const int col0 = n_blk * GEMM_BN + c * 32;
+#pragma unroll
+      for (int j = 0; j < 32; ++j) {
+        const float v = __uint_as_float(r[j]);
+        if (col0 + j < p.N && v > best) {  // strict: lowest column wins ties (R18)
+          best = v;
+          best_i = col0 + j;
+        }
+      }
+    }
+    if (row_ok) {
+      p.part_val[(size_t)row * p.num_n_tiles + n_blk] = best;
+      p.part_idx[(size_t)row * p.num_n_tiles + n_blk] = best_i;
+    }
+  }
+}
+
+template <int EPI, int CG>
 __global__ void __launch_bounds__(256, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
                    const GemmArgs p) {
+  using C = Cfg<CG>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
-  uint8_t* sB = smem + GEMM_STAGES * A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(sB + GEMM_STAGES * B_BYTES);
-  uint64_t* empty = full + GEMM_STAGES;
-  uint64_t* tfull = empty + GEMM_STAGES;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(tempty + 2);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const uint32_t rank = CG == 2 ? cluster_rank() : 0;
+  const bool leader = rank == 0;
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tma_a);
     ptx::tma_prefetch(&tma_b);
   }
   if (warp == 1 && lane == 0) {
-    for (int s = 0; s < GEMM_STAGES; ++s) {
+    for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
     }
     for (int s = 0; s < 2; ++s) {
       ptx::mbar_init(&tfull[s], 1);
-      ptx::mbar_init(&tempty[s], 4);
+      ptx::mbar_init(&tempty[s], 4 * CG);  // every epilogue warp of the pair releases the leader's buffer
     }
     ptx::fence_barrier_init();
   }
-  if (warp == 2) {
-    ptx::tmem_alloc(tmem_ptr, TMEM_COLS);
-    ptx::tmem_relinquish();
-  }
+  if (warp == 2) tmem_alloc_cg<CG>(tmem_ptr, TMEM_COLS);
   ptx::tc_fence_before();
-  __syncthreads();
+  if constexpr (CG == 2)
+    cluster_sync_all();
+  else
+    __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_ptr;
 
-  const int num_m = p.num_m_tiles;
-  const int ntiles = num_m * p.num_n_tiles;
-  const int nk = p.K / GEMM_BK;
+  const int num_m = (p.M + C::TILE_M - 1) / C::TILE_M;
+  Jobs jobs;
+  jobs.init(p, blockIdx.x / CG, gridDim.x / CG, num_m);
+  int tile, kb0, kb1;
 
   if (warp == 0) {
     if (lane == 0) {
-      // ---------------- TMA producer
+      // ---------------- TMA producer (both CTAs of a pair load their halves)
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+      while (jobs.next(tile, kb0, kb1)) {
         const int m_blk = tile % num_m, n_blk = tile / num_m;
-        for (int kb = 0; kb < nk; ++kb) {
+        const int a_row = m_blk * C::TILE_M + rank * GEMM_BM;
+        const int b_row = n_blk * GEMM_BN + rank * C::B_ROWS;
+        for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&empty[stage], phase ^ 1);
-          ptx::mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
-          ptx::tma_load_2d(sA + stage * A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, m_blk * GEMM_BM);
-          ptx::tma_load_2d(sB + stage * B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, n_blk * GEMM_BN);
-          if (++stage == GEMM_STAGES) {
+          if constexpr (CG == 1) {
+            ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+            ptx::tma_load_2d(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
+            ptx::tma_load_2d(sB + stage * C::B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, b_row);
+            ptx::tma_load_2d(sB + stage * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[stage], kb * GEMM_BK,
+                             b_row + GEMM_B_BOX);
+          } else {
+            if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+            tma_load_2d_cg2(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
+            tma_load_2d_cg2(sB + stage * C::B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, b_row);
+          }
+          if (++stage == C::STAGES) {
             stage = 0;
             phase ^= 1;
           }
@@ -94,237 +422,156 @@ __global__ void __launch_bounds__(256, 1)
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      // ---------------- MMA issuer (single thread)
-      constexpr uint32_t idesc = ptx::umma_idesc_bf16(GEMM_BM, GEMM_BN);
+    if (lane == 0 && leader) {
+      // ---------------- MMA issuer (single thread of the leader CTA)
+      constexpr uint32_t idesc = ptx::umma_idesc_bf16(C::TILE_M, GEMM_BN);
       int stage = 0;
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+      while (jobs.next(tile, kb0, kb1)) {
         ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * GEMM_BN;
-        for (int kb = 0; kb < nk; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
-          const uint32_t a_addr = ptx::smem_u32(sA + stage * A_BYTES);
-          const uint32_t b_addr = ptx::smem_u32(sB + stage * B_BYTES);
+          const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+          const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
           for (int k = 0; k < GEMM_BK / 16; ++k) {
-            ptx::umma_bf16(d_tmem, ptx::umma_desc_sw128(a_addr + k * 32), ptx::umma_desc_sw128(b_addr + k * 32),
-                           idesc, (kb | k) != 0);
+            const uint64_t ad = ptx::umma_desc_sw128(a_addr + k * 32), bd = ptx::umma_desc_sw128(b_addr + k * 32);
+            const uint32_t accum = (kb > kb0 || k > 0) ? 1u : 0u;
+            if constexpr (CG == 1)
+              ptx::umma_bf16(d_tmem, ad, bd, idesc, accum);
+            else
+              umma_bf16_cg2(d_tmem, ad, bd, idesc, accum);
           }
-          ptx::umma_commit(&empty[stage]);  // frees the SMEM slot once these MMAs retire
-          if (++stage == GEMM_STAGES) {
+          if constexpr (CG == 1)
+            ptx::umma_commit(&empty[stage]);  // frees the SMEM slot once these MMAs retire
+          else
+            umma_commit_cg2(&empty[stage]);   // ... in both CTAs
+          if (++stage == C::STAGES) {
             stage = 0;
             phase ^= 1;
           }
         }
-        ptx::umma_commit(&tfull[acc]);  // accumulator ready for the epilogue
+        if constexpr (CG == 1)
+          ptx::umma_commit(&tfull[acc]);  // accumulator ready for the epilogue
+        else
+          umma_commit_cg2(&tfull[acc]);
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
       }
     }
   } else if (warp >= 4) {
-    // ---------------- epilogue warps
+    // ---------------- epilogue warps (each CTA drains its own 128 rows)
     const int ew = warp - 4;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int nk = p.K / GEMM_BK;
+    while (jobs.next(tile, kb0, kb1)) {
       const int m_blk = tile % num_m, n_blk = tile / num_m;
-      ptx::mbar_wait(&tfull[acc], acc_phase);
-      ptx::tc_fence_after();
-      const int row = m_blk * GEMM_BM + ew * 32 + lane;
-      const bool row_ok = row < p.M;
+      const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
-      uint32_t r[32];
-      if constexpr (EPI == EPI_STORE_BF16) {
-        __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
-#pragma unroll 1
-        for (int c = 0; c < GEMM_BN / 32; ++c) {
-          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-          ptx::tmem_ld_wait();
-          const int col0 = n_blk * GEMM_BN + c * 32;
-          if (row_ok && col0 < p.N) {
-            float v[32];
-#pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
-            if (p.bias) {
-#pragma unroll
-              for (int j = 0; j < 32; ++j) v[j] += __ldg(p.bias + col0 + j);
-            }
-            uint4* dst = reinterpret_cast<uint4*>(out + (size_t)row * p.ldo + col0);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              uint4 w;
-              w.x = ptx::pack_bf16(v[q * 8 + 0], v[q * 8 + 1]);
-              w.y = ptx::pack_bf16(v[q * 8 + 2], v[q * 8 + 3]);
-              w.z = ptx::pack_bf16(v[q * 8 + 4], v[q * 8 + 5]);
-              w.w = ptx::pack_bf16(v[q * 8 + 6], v[q * 8 + 7]);
-              dst[q] = w;
-            }
-          }
-        }
-      } else if constexpr (EPI == EPI_ADD_F32) {
-        float* out = reinterpret_cast<float*>(p.out);
-#pragma unroll 1
-        for (int c = 0; c < GEMM_BN / 32; ++c) {
-          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-          ptx::tmem_ld_wait();
-          const int col0 = n_blk * GEMM_BN + c * 32;
-          if (row_ok && col0 < p.N) {
-            float4* dst = reinterpret_cast<float4*>(out + (size_t)row * p.ldo + col0);
-#pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              float4 x = dst[q];
-              x.x += __uint_as_float(r[q * 4 + 0]);
-              x.y += __uint_as_float(r[q * 4 + 1]);
-              x.z += __uint_as_float(r[q * 4 + 2]);
-              x.w += __uint_as_float(r[q * 4 + 3]);
-              dst[q] = x;
-            }
-          }
-        }
-      } else if constexpr (EPI == EPI_SILU_MUL) {
-        __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
-        uint32_t u[32];
-#pragma unroll 1
-        for (int c = 0; c < GEMM_BN / 64; ++c) {
-          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);                  // gate columns
-          ptx::tmem_ld_32x32b_x32(tbase + GEMM_BN / 2 + c * 32, u);    // up columns
-          ptx::tmem_ld_wait();
-          const int col0 = n_blk * (GEMM_BN / 2) + c * 32;
-          if (row_ok && col0 < p.N / 2) {
-            uint4* dst = reinterpret_cast<uint4*>(out + (size_t)row * p.ldo + col0);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              float h[8];
-#pragma unroll
-              for (int j = 0; j < 8; ++j)
-                h[j] = silu_f(__uint_as_float(r[q * 8 + j])) * __uint_as_float(u[q * 8 + j]);
-              uint4 w;
-              w.x = ptx::pack_bf16(h[0], h[1]);
-              w.y = ptx::pack_bf16(h[2], h[3]);
-              w.z = ptx::pack_bf16(h[4], h[5]);
-              w.w = ptx::pack_bf16(h[6], h[7]);
-              dst[q] = w;
-            }
-          }
-        }
-      } else if constexpr (EPI == EPI_QKV_ROPE) {
-        // The 256 columns of a tile are whole heads (D | 256); rotate-half partners (i, i + D/2)
-        // are 32-column chunks c and c + D/64 of the same head.
-        const int D = p.head_dim, half = D / 2, per_head = D / 32;
-        const int slot = row_ok ? __ldg(p.slots + row) : 0;
-        const int64_t blk = slot / p.block_size, off = slot % p.block_size;
-        uint32_t u[32];
-#pragma unroll 1
-        for (int c = 0; c < GEMM_BN / 32; ++c) {
-          const int hpos = c % per_head;  // chunk index within its head
-          if (hpos >= per_head / 2) continue;
-          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-          ptx::tmem_ld_32x32b_x32(tbase + (c + per_head / 2) * 32, u);
-          ptx::tmem_ld_wait();
-          const int col1 = n_blk * GEMM_BN + c * 32;  // first-half column of this chunk
-          if (!row_ok || col1 >= p.N) continue;
-          const int col2 = col1 + half;
-          const int i0 = hpos * 32;                   // rotation index of element 0
-          float x1[32], x2[32];
-#pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            x1[j] = __uint_as_float(r[j]);
-            x2[j] = __uint_as_float(u[j]);
-          }
-          if (p.bias) {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              x1[j] += __ldg(p.bias + col1 + j);
-              x2[j] += __ldg(p.bias + col2 + j);
-            }
-          }
-          __nv_bfloat16 *dst1, *dst2;
-          if (col1 < p.q_dim + p.kv_dim) {  // q or k: rotate
-            const float4* cs = reinterpret_cast<const float4*>(p.rope_cs + (size_t)row * half + i0);
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-              const float4 v = __ldg(cs + j);  // (cos, sin) of elements 2j, 2j+1
-              const float a1 = x1[2 * j], a2 = x2[2 * j], b1 = x1[2 * j + 1], b2 = x2[2 * j + 1];
-              x1[2 * j] = a1 * v.x - a2 * v.y;
-              x2[2 * j] = a2 * v.x + a1 * v.y;
-              x1[2 * j + 1] = b1 * v.z - b2 * v.w;
-              x2[2 * j + 1] = b2 * v.z + b1 * v.w;
-            }
-          }
-          if (col1 < p.q_dim) {
-            __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo;
-            dst1 = out + col1;
-            dst2 = out + col2;
-          } else {
-            const bool is_k = col1 < p.q_dim + p.kv_dim;
-            const int cc = col1 - p.q_dim - (is_k ? 0 : p.kv_dim);
-            const int h = cc / D;
-            __nv_bfloat16* base = (is_k ? p.kc : p.vc) + ((blk * p.n_kv_heads + h) * p.block_size + off) * D;
-            dst1 = base + i0;
-            dst2 = base + i0 + half;
-          }
-          uint4* d1 = reinterpret_cast<uint4*>(dst1);
-          uint4* d2 = reinterpret_cast<uint4*>(dst2);
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            uint4 w1, w2;
-            w1.x = ptx::pack_bf16(x1[q * 8 + 0], x1[q * 8 + 1]);
-            w1.y = ptx::pack_bf16(x1[q * 8 + 2], x1[q * 8 + 3]);
-            w1.z = ptx::pack_bf16(x1[q * 8 + 4], x1[q * 8 + 5]);
-            w1.w = ptx::pack_bf16(x1[q * 8 + 6], x1[q * 8 + 7]);
-            w2.x = ptx::pack_bf16(x2[q * 8 + 0], x2[q * 8 + 1]);
-            w2.y = ptx::pack_bf16(x2[q * 8 + 2], x2[q * 8 + 3]);
-            w2.z = ptx::pack_bf16(x2[q * 8 + 4], x2[q * 8 + 5]);
-            w2.w = ptx::pack_bf16(x2[q * 8 + 6], x2[q * 8 + 7]);
-            d1[q] = w1;
-            d2[q] = w2;
-          }
-        }
-      } else {  // EPI_ARGMAX
-        float best = -INFINITY;
-        int best_i = 0x7fffffff;
-#pragma unroll 1
-        for (int c = 0; c < GEMM_BN / 32; ++c) {
-          ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-          ptx::tmem_ld_wait();
-          const int col0 = n_blk * GEMM_BN + c * 32;
-#pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const float v = __uint_as_float(r[j]);
-            if (col0 + j < p.N && v > best) {  // strict: lowest column wins ties (R18)
-              best = v;
-              best_i = col0 + j;
-            }
-          }
-        }
-        if (row_ok) {
-          p.part_val[(size_t)row * p.num_n_tiles + n_blk] = best;
-          p.part_idx[(size_t)row * p.num_n_tiles + n_blk] = best_i;
-        }
-      }
+      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase);
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+      if (lane == 0) {
+        if constexpr (CG == 1)
+          ptx::mbar_arrive(&tempty[acc]);
+        else
+          mbar_arrive_leader(&tempty[acc]);
+      }
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
     }
   }
-  __syncthreads();
+  ptx::tc_fence_before();
+  if constexpr (CG == 2)
+    cluster_sync_all();
+  else
+    __syncthreads();
   if (warp == 2) {
     ptx::tc_fence_after();
-    ptx::tmem_dealloc(tmem_base, TMEM_COLS);
+    tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
+  }
+}
+
+// Workspace mode: apply the non-additive epilogue to the fp32 sums in ws [M, N].
+// One thread per (row, 32-column chunk) of the OUTPUT space of the epilogue.
+template <int EPI>
+__global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
+  const int chunks_per_row = (EPI == EPI_SILU_MUL) ? p.N / 64 : p.N / 32;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= p.M * chunks_per_row) return;
+  const int row = idx / chunks_per_row, c = idx % chunks_per_row;
+  const float* w = p.ws + (size_t)row * p.N;
+  if constexpr (EPI == EPI_STORE_BF16) {
+    float v[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] = w[c * 32 + j] + (p.bias ? p.bias[c * 32 + j] : 0.f);
+    store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, v);
+  } else if constexpr (EPI == EPI_SILU_MUL) {
+    const int n_blk = c / 4, cc = c % 4;  // output chunk -> (tile, chunk within the 128 gate columns)
+    const float* g = w + n_blk * GEMM_BN + cc * 32;
+    const float* u = g + GEMM_BN / 2;
+    float h[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) h[j] = silu_f(g[j]) * u[j];
+    store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, h);
+  } else if constexpr (EPI == EPI_QKV_ROPE) {
+    const int per_head = p.head_dim / 32, hpos = c % per_head;
+    if (hpos >= per_head / 2) return;
+    const int col1 = c * 32, half = p.head_dim / 2;
+    float x1[32], x2[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+      x1[j] = w[col1 + j] + (p.bias ? p.bias[col1 + j] : 0.f);
+      x2[j] = w[col1 + half + j] + (p.bias ? p.bias[col1 + half + j] : 0.f);
+    }
+    const int slot = p.slots[row];
+    qkv_rope_store(p, row, col1, hpos * 32, x1, x2, slot / p.block_size, slot % p.block_size);
   }
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_encode_once;
 
+// Scheduling decision (host).  Returns 1 for stream-K (CG=1 only).
+int choose_streamk(int M, int N, int ntiles, int nk, int epi, int num_sms) {
+  if (epi == EPI_ARGMAX || nk < 8) return 0;
+  const int waves = (ntiles + num_sms - 1) / num_sms;
+  const double eff = (double)ntiles / ((double)waves * num_sms);
+  // Measured on B200: with >= one wave of tiles the reductions of partial tiles cost more than
+  // the last-wave imbalance they remove, so stream-K is used only below one wave (small T).
+  if (ntiles >= num_sms) return 0;
+  if (epi == EPI_ADD_F32) return 1;  // partial tiles: fp32 vector reductions into the residual
+  // non-additive epilogues go through the fp32 workspace (memset + reductions + finish pass)
+  return (eff < 0.5 && (size_t)M * N <= GEMM_WS_ELEMS) ? 1 : 0;
+}
+
+// CTA-pair tiles need at least one wave of 256 x 256 tiles.  Measured on B200 (tools/gemm_bench.py,
+// profiles/r01): the pair kernel is +17% on the C1 QKV shape (2094x6144x4096) and +11% on
+// 8192^3, but 3-7% slower on the O / gate_up / down shapes at T ~ 2094, so those keep the
+// 1-CTA kernel unless M is large.
+int choose_cg(int M, int N, int epi, int num_sms) {
+  if (g_force_cg) return g_force_cg;
+  const int tiles2 = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
+  if (M < 256 || tiles2 * 2 < num_sms || epi == EPI_ARGMAX) return 1;
+  if (epi == EPI_STORE_BF16 || epi == EPI_QKV_ROPE) return 2;
+  return M >= 4096 ? 2 : 1;
+}
+
 }  // namespace
+
+size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms) {
+  const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
+  if (epi == EPI_ADD_F32 || choose_cg(M, N, epi, num_sms) == 2 ||
+      !choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms))
+    return 0;
+  return (size_t)M * N;
+}
 
 int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols, uint32_t box_rows) {
   std::call_once(g_encode_once, [] {
@@ -355,38 +602,88 @@ int num_sms_of_current_device() {
   return n > 0 ? n : 148;
 }
 
-template <int EPI>
+template <int EPI, int CG>
 static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args, cudaStream_t stream,
                     int num_sms) {
+  using C = Cfg<CG>;
   static bool attr_set = false;  // per-process; the attribute is per-function
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(gemm_tc_kernel<EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
+    cudaError_t e =
+        cudaFuncSetAttribute(gemm_tc_kernel<EPI, CG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm smem attribute: %s", cudaGetErrorString(e));
     attr_set = true;
   }
-  const int ntiles = args.num_m_tiles * args.num_n_tiles;
-  const int grid = ntiles < num_sms ? ntiles : num_sms;
+  const int num_m = (args.M + C::TILE_M - 1) / C::TILE_M;
+  const int ntiles = num_m * args.num_n_tiles;
+  int grid;
+  if (args.streamk) {
+    const int total = ntiles * (args.K / GEMM_BK);
+    grid = (total + args.units_per_cta - 1) / args.units_per_cta;
+  } else {
+    const int units = num_sms / CG;
+    grid = (ntiles < units ? ntiles : units) * CG;
+  }
   if (grid <= 0) return GLLM_OK;
-  gemm_tc_kernel<EPI><<<grid, 256, SMEM_BYTES, stream>>>(a, b, args);
+  if (args.ws) {
+    cudaError_t e = cudaMemsetAsync(args.ws, 0, (size_t)args.M * args.N * sizeof(float), stream);
+    if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm workspace memset: %s", cudaGetErrorString(e));
+  }
+  if constexpr (CG == 1) {
+    gemm_tc_kernel<EPI, 1><<<grid, 256, C::SMEM_BYTES, stream>>>(a, b, args);
+  } else {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = C::SMEM_BYTES;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_tc_kernel<EPI, 2>, a, b, args);
+    if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (2-CTA) launch: %s", cudaGetErrorString(e));
+  }
+  if (args.ws) {
+    const int chunks = args.M * ((EPI == EPI_SILU_MUL) ? args.N / 64 : args.N / 32);
+    gemm_finish_kernel<EPI><<<(chunks + 255) / 256, 256, 0, stream>>>(args);
+  }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm launch: %s", cudaGetErrorString(e));
   return GLLM_OK;
 }
 
+template <int EPI>
+static int launch_e(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args, cudaStream_t stream,
+                    int num_sms, int cg) {
+  return cg == 2 ? launch_t<EPI, 2>(a, b, args, stream, num_sms) : launch_t<EPI, 1>(a, b, args, stream, num_sms);
+}
+
 int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const GemmArgs& args0, cudaStream_t stream,
                 int num_sms) {
-  if (args0.K % GEMM_BK != 0 || args0.M < 0 || args0.N <= 0)
+  if (args0.K % GEMM_BK != 0 || args0.M < 0 || args0.N <= 0 || args0.N % 32)
     return set_error(GLLM_EINVAL, "gemm: K %% 64 != 0 or bad M/N (M=%d N=%d K=%d)", args0.M, args0.N, args0.K);
   if (args0.M == 0) return GLLM_OK;
   GemmArgs args = args0;
+  const int cg = choose_cg(args.M, args.N, epi, num_sms);
   args.num_m_tiles = (args.M + GEMM_BM - 1) / GEMM_BM;
   args.num_n_tiles = (args.N + GEMM_BN - 1) / GEMM_BN;
+  const int ntiles = args.num_m_tiles * args.num_n_tiles, nk = args.K / GEMM_BK;
+  args.streamk = cg == 1 ? choose_streamk(args.M, args.N, ntiles, nk, epi, num_sms) : 0;
+  args.units_per_cta = args.streamk ? (ntiles * nk + num_sms - 1) / num_sms : 0;
+  if (args.streamk && epi != EPI_ADD_F32) {
+    if (!args0.ws) return set_error(GLLM_EINVAL, "gemm: stream-K workspace required");
+  } else {
+    args.ws = nullptr;
+  }
   switch (epi) {
-    case EPI_STORE_BF16: return launch_t<EPI_STORE_BF16>(a, b, args, stream, num_sms);
-    case EPI_ADD_F32: return launch_t<EPI_ADD_F32>(a, b, args, stream, num_sms);
-    case EPI_SILU_MUL: return launch_t<EPI_SILU_MUL>(a, b, args, stream, num_sms);
-    case EPI_ARGMAX: return launch_t<EPI_ARGMAX>(a, b, args, stream, num_sms);
-    case EPI_QKV_ROPE: return launch_t<EPI_QKV_ROPE>(a, b, args, stream, num_sms);
+    case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, args, stream, num_sms, cg);
+    case EPI_ADD_F32: return launch_e<EPI_ADD_F32>(a, b, args, stream, num_sms, cg);
+    case EPI_SILU_MUL: return launch_e<EPI_SILU_MUL>(a, b, args, stream, num_sms, cg);
+    case EPI_ARGMAX: return launch_e<EPI_ARGMAX>(a, b, args, stream, num_sms, cg);
+    case EPI_QKV_ROPE: return launch_e<EPI_QKV_ROPE>(a, b, args, stream, num_sms, cg);
   }
   return set_error(GLLM_EINVAL, "gemm: unknown epilogue");
 }

@@ -29,9 +29,24 @@ struct GemmArgs {
   __nv_bfloat16* kc;      // [kv_blocks][n_kv_heads][block_size][head_dim]
   __nv_bfloat16* vc;
   int q_dim, kv_dim, head_dim, n_kv_heads, block_size;
+  // scheduling (filled by launch_gemm): 0 = one CTA per 128x256 tile (persistent round robin);
+  // 1 = stream-K: CTA i owns k-block units [i*units_per_cta, (i+1)*units_per_cta) of the
+  // (tile, k-block) space; partial tiles combine with fp32 atomics into `out` (EPI_ADD_F32) or
+  // into the fp32 workspace `ws` [M, N], finished by gemm_finish_kernel.
+  int streamk, units_per_cta;
+  float* ws;
 };
 
+// fp32 workspace (elements) launch_gemm may need for a GEMM of this shape/epilogue (0 = none)
+size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms);
+
 constexpr int GEMM_BM = 128, GEMM_BN = 256, GEMM_BK = 64, GEMM_STAGES = 4;
+constexpr size_t GEMM_WS_ELEMS = size_t(8) << 20;  // stream-K fp32 workspace capacity (32 MB)
+// TMA box rows of the B (weight) tensor maps: one 128-row half of a 256-wide N tile, so the same
+// map serves the 1-CTA kernel (two loads per stage) and the CTA-pair kernel (one per CTA).
+constexpr int GEMM_B_BOX = 128;
+// testing / tuning: force the 1-CTA (1) or CTA-pair (2) kernel; 0 = automatic
+extern int g_force_cg;
 
 // Encodes a 2-D bf16 K-major tensor map (rows x cols, cols contiguous) with a
 // (box_rows x 64) box and 128-byte swizzle.  Returns 0 or a GLLM_* error.

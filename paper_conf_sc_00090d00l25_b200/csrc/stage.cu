@@ -118,6 +118,7 @@ struct gllm_stage {
   float2* rope_cs = nullptr;
   int32_t* slots = nullptr;
   int32_t* sampled_tmp = nullptr;
+  float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T)
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
@@ -126,6 +127,8 @@ struct gllm_stage {
   int ring_i = 0;
   std::vector<void*> allocs;
   ncclComm_t comm = nullptr;
+  cudaStream_t side = nullptr;  // prefill attention runs here, concurrent with decode attention
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int last_T = 0, last_launches = 0;
   bool profiling = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> prof_ev;
@@ -194,6 +197,7 @@ int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmE
   g.bias = bias;
   g.part_val = st->part_val;
   g.part_idx = st->part_idx;
+  g.ws = st->gemm_ws;
   st->last_launches += 1;
   return gllm::launch_gemm(a, b, epi, g, s, st->num_sms);
 }
@@ -227,6 +231,9 @@ void destroy(gllm_stage* st) {
   }
   for (auto e : st->ev_pool) cudaEventDestroy(e);
   if (st->comm && nccl().ok) nccl().comm_destroy(st->comm);
+  if (st->side) cudaStreamDestroy(st->side);
+  if (st->ev_fork) cudaEventDestroy(st->ev_fork);
+  if (st->ev_join) cudaEventDestroy(st->ev_join);
   cudaGetLastError();
   delete st;
 }
@@ -338,10 +345,10 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     }
     CK(cudaMemsetAsync(w.kc, 0, kv_elems * sizeof(bf16), s0));
     CK(cudaMemsetAsync(w.vc, 0, kv_elems * sizeof(bf16), s0));
-    if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_BN)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_BN)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_BN)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_BN)))
+    if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_B_BOX)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_B_BOX)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_B_BOX)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)))
       return fail(rc);
     st->layers.push_back(w);
   }
@@ -353,7 +360,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     if ((rc = st->dalloc(&st->lm_head, (size_t)V * H)) || (rc = st->dalloc(&st->final_norm, H))) return fail(rc);
     gllm::launch_init_bf16(st->lm_head, V, H, seed, T_LMHEAD, s_h, 0, 0, s0);
     gllm::launch_fill_f32(st->final_norm, H, 1.0f, s0);
-    if ((rc = gllm::make_tmap_bf16(&st->tm_lm, st->lm_head, V, H, gllm::GEMM_BN))) return fail(rc);
+    if ((rc = gllm::make_tmap_bf16(&st->tm_lm, st->lm_head, V, H, gllm::GEMM_B_BOX))) return fail(rc);
     const int ntn = (V + gllm::GEMM_BN - 1) / gllm::GEMM_BN;
     if ((rc = st->dalloc(&st->ys, (size_t)st->seqs_alloc * H)) ||
         (rc = st->dalloc(&st->part_val, (size_t)st->seqs_alloc * ntn)) ||
@@ -366,7 +373,9 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   if ((rc = st->dalloc(&st->xbuf, R * H)) || (rc = st->dalloc(&st->y, R * H)) ||
       (rc = st->dalloc(&st->qkv, R * nqkv)) || (rc = st->dalloc(&st->attn, R * qd)) ||
       (rc = st->dalloc(&st->act, R * I)) || (rc = st->dalloc(&st->rope_cs, R * (D / 2))) ||
-      (rc = st->dalloc(&st->slots, R)))
+      (rc = st->dalloc(&st->slots, R)) ||
+      // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
+      (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)))
     return fail(rc);
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
@@ -377,6 +386,10 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     return fail(rc);
   for (int i = 0; i < RING; ++i)
     if ((rc = new_slot(st)) < 0) return fail(rc);
+  if (cudaStreamCreateWithFlags(&st->side, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&st->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&st->ev_join, cudaEventDisableTiming) != cudaSuccess)
+    return fail(gllm::set_error(GLLM_ECUDA, "side stream / events"));
   if ((rc = ensure_parts(st, 1024)) < 0) return fail(rc);
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return fail(gllm::set_error(GLLM_ECUDA, "init: %s", cudaGetErrorString(e)));
@@ -596,17 +609,34 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.head_dim = D;
       g.n_kv_heads = c.n_kv_heads;
       g.block_size = bs;
+      g.ws = st->gemm_ws;
       st->last_launches += 1;
       RC(gllm::launch_gemm(st->tm_y, w.tm_qkv, gllm::EPI_QKV_ROPE, g, s, st->num_sms));
     }
     aa.kc = w.kc;
     aa.vc = w.vc;
+    // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
+    // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
+    const bool overlap = P.n_pi > 0 && P.n_di > 0;
     if (P.n_pi > 0) {
-      Prof p(st, s, C_PREFILL);
-      RC(gllm::launch_prefill_attention(aa, d_pi, P.n_pi, s));
+      cudaStream_t ps = overlap ? st->side : s;
+      if (overlap) {
+        CK(cudaEventRecord(st->ev_fork, s));
+        CK(cudaStreamWaitEvent(ps, st->ev_fork, 0));
+      }
+      {
+        Prof p(st, ps, C_PREFILL);
+        RC(gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps));
+      }
+      if (overlap) CK(cudaEventRecord(st->ev_join, ps));
       st->last_launches += 1;
     }
-    if (P.n_di > 0) {
+    if (overlap) {
+      Prof p(st, s, C_DECODE);
+      RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
+      st->last_launches += P.n_mi ? 2 : 1;
+      CK(cudaStreamWaitEvent(s, st->ev_join, 0));
+    } else if (P.n_di > 0) {
       Prof p(st, s, C_DECODE);
       RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
       st->last_launches += P.n_mi ? 2 : 1;

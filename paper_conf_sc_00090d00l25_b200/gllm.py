@@ -112,6 +112,8 @@ def lib():
             "gllm_stage_set_profiling": ([vp, i32], C.c_int),
             "gllm_stage_last_timing": ([vp, C.POINTER(C.c_float), i32], C.c_int),
             "gllm_stage_last_launches": ([vp, _P32], C.c_int),
+            "gllm_op_gemm": ([vp, vp, i32, i32, i32, i32, vp, vp, vp], C.c_int),
+            "gllm_op_set_gemm_variant": ([i32], C.c_int),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -333,6 +335,16 @@ class Stage:
 
     def recv_hidden(self, ptr, num_tokens, src, stream=0):
         _check(lib().gllm_recv_hidden(self.h, ptr, num_tokens, src, stream or None))
+
+
+def op_gemm(A_ptr, W_ptr, M, N, K, epi, out_ptr, bias_ptr=0, stream=0):
+    """gllm_op_gemm (include/gllm_ops.h): the stage's tcgen05 GEMM on raw device pointers."""
+    _check(lib().gllm_op_gemm(A_ptr, W_ptr, M, N, K, epi, bias_ptr or None, out_ptr, stream or None))
+
+
+def op_set_gemm_variant(cta_group: int):
+    """0 = automatic, 1 = 1-CTA 128x256 kernel, 2 = CTA-pair 256x256 kernel (testing / tuning)."""
+    _check(lib().gllm_op_set_gemm_variant(cta_group))
 
 
 def get_unique_id() -> bytes:

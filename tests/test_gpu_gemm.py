@@ -1,0 +1,97 @@
+"""Kernel-level parity of the tcgen05 GEMM (gllm_op_gemm, include/gllm_ops.h) against the plain
+definition Y = A W^T computed in fp64 with numpy on the same bf16 values, for ragged M (TMA
+out-of-bounds rows, partial tiles), stream-K (few tiles) and every epilogue."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_sc_00090d00l25_b200 import gllm
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(params=[1, 2, 0], ids=["cta1", "cta2", "auto"], autouse=True)
+def variant(request):
+    # every test runs with the 1-CTA kernel, the CTA-pair (cta_group::2) kernel and the automatic choice
+    gllm.op_set_gemm_variant(request.param)
+    yield request.param
+    gllm.op_set_gemm_variant(0)
+
+
+def _bf16(shape, scale, seed):
+    g = torch.Generator().manual_seed(seed)
+    return (torch.randn(shape, generator=g) * scale).to(torch.bfloat16)
+
+
+def _ref(A, W):
+    return A.double().numpy() @ W.double().numpy().T
+
+
+@pytest.mark.parametrize("M", [1, 7, 128, 129, 1000, 2094])
+@pytest.mark.parametrize("N,K", [(768, 256), (4096, 4096), (6144, 4096), (1024, 14336)])
+def test_store_bf16_with_bias(M, N, K):
+    A, W = _bf16((M, K), 1.0, 1), _bf16((N, K), K ** -0.5, 2)
+    bias = torch.randn(N, generator=torch.Generator().manual_seed(3)) * 0.02
+    dA, dW, db = A.cuda(), W.cuda(), bias.cuda()
+    out = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 0, out.data_ptr(), db.data_ptr())
+    torch.cuda.synchronize()
+    ref = _ref(A, W) + bias.double().numpy()
+    got = out.float().cpu().numpy()
+    err = np.abs(got - ref).max(-1) / np.abs(ref).max(-1)
+    assert err.max() < 1e-2, err.max()
+
+
+@pytest.mark.parametrize("M", [1, 33, 300, 2094])
+@pytest.mark.parametrize("N,K", [(4096, 4096), (8192, 28672), (5120, 5120)])
+def test_residual_add_f32(M, N, K):
+    # covers whole-tile and stream-K (below one wave of tiles: fp32 vector reductions) schedules
+    A, W = _bf16((M, K), 1.0, 4), _bf16((N, K), K ** -0.5, 5)
+    x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(6))
+    dA, dW, x = A.cuda(), W.cuda(), x0.clone().cuda()
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 1, x.data_ptr())
+    torch.cuda.synchronize()
+    ref = x0.double().numpy() + _ref(A, W)
+    err = np.abs(x.cpu().double().numpy() - ref).max()
+    assert err < 1e-3, err
+
+
+@pytest.mark.parametrize("M", [5, 128, 700])
+def test_silu_mul_interleaved(M):
+    I, K = 1024, 512
+    A = _bf16((M, K), 1.0, 7)
+    Wg, Wu = _bf16((I, K), K ** -0.5, 8), _bf16((I, K), K ** -0.5, 9)
+    W = torch.empty((2 * I, K), dtype=torch.bfloat16)
+    for j in range(I // 128):      # interleave blocks of 128 gate rows and 128 up rows
+        W[256 * j:256 * j + 128] = Wg[128 * j:128 * j + 128]
+        W[256 * j + 128:256 * j + 256] = Wu[128 * j:128 * j + 128]
+    dA, dW = A.cuda(), W.cuda()
+    out = torch.empty((M, I), dtype=torch.bfloat16, device="cuda")
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, 2 * I, K, 2, out.data_ptr())
+    torch.cuda.synchronize()
+    g, u = _ref(A, Wg), _ref(A, Wu)
+    ref = g / (1 + np.exp(-g)) * u
+    err = np.abs(out.float().cpu().numpy() - ref).max(-1) / np.abs(ref).max(-1)
+    assert err.max() < 1e-2, err.max()
+
+
+@pytest.mark.parametrize("M,N", [(1, 512), (9, 128256), (300, 152064)])
+def test_argmax_epilogue(M, N):
+    K = 1024
+    A, W = _bf16((M, K), 1.0, 10), _bf16((N, K), K ** -0.5, 11)
+    dA, dW = A.cuda(), W.cuda()
+    out = torch.empty((M,), dtype=torch.int32, device="cuda")
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 3, out.data_ptr())
+    torch.cuda.synchronize()
+    ref = _ref(A, W)
+    ids = out.cpu().numpy()
+    # fp32 accumulation vs fp64: the chosen logit must be the max up to accumulation error
+    assert np.all(ref[np.arange(M), ids] >= ref.max(-1) - 1e-4 * np.abs(ref).max(-1))
+    assert np.mean(ids == ref.argmax(-1)) >= 0.9
+
+
+def test_bad_shapes_are_einval():
+    A = torch.zeros((4, 100), dtype=torch.bfloat16, device="cuda")
+    with pytest.raises(gllm.GllmError) as e:
+        gllm.op_gemm(A.data_ptr(), A.data_ptr(), 4, 4, 100, 0, A.data_ptr())
+    assert e.value.code == -1

@@ -1,0 +1,62 @@
+"""Micro-benchmark of the stage GEMM through gllm_op_gemm (CUDA events, L2-flushed between reps).
+
+    python tools/gemm_bench.py [--shapes C1]      # prints one line per (M, N, K, epi)
+"""
+import argparse
+import json
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_sc_00090d00l25_b200 import gllm  # noqa: E402
+
+SHAPES = {
+    # (M, N, K, epi): C1 projections at the PP=1 window mean T ~ 2094, and C4's small-T stage
+    "C1": [(2094, 6144, 4096, 0), (2094, 4096, 4096, 1), (2094, 28672, 4096, 2), (2094, 4096, 14336, 1)],
+    "C4": [(128, 10240, 8192, 0), (128, 8192, 8192, 1), (128, 57344, 8192, 2), (128, 8192, 28672, 1)],
+    "sq": [(8192, 8192, 8192, 0)],
+}
+
+
+def bench(M, N, K, epi, reps=20):
+    A = torch.randn((M, K), device="cuda").to(torch.bfloat16)
+    W = (torch.randn((N, K), device="cuda") * K ** -0.5).to(torch.bfloat16)
+    if epi == 1:
+        out = torch.zeros((M, N), device="cuda")
+    elif epi == 2:
+        out = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+    else:
+        out = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+    flush = torch.empty(256 << 20, dtype=torch.int8, device="cuda")
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(3):
+        gllm.op_gemm(A.data_ptr(), W.data_ptr(), M, N, K, epi, out.data_ptr(), 0, s)
+    ts = []
+    for _ in range(reps):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        gllm.op_gemm(A.data_ptr(), W.data_ptr(), M, N, K, epi, out.data_ptr(), 0, s)
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    ts.sort()
+    ms = ts[len(ts) // 2]
+    tf = 2.0 * M * N * K / (ms * 1e-3) / 1e12
+    gbs = (N * K * 2 + M * K * 2) / (ms * 1e-3) / 1e9
+    return dict(M=M, N=N, K=K, epi=epi, us=round(ms * 1e3, 1), tflops=round(tf, 1), weight_gbs=round(gbs, 1))
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--shapes", default="C1,C4,sq")
+    ap.add_argument("--variants", default="0", help="comma list: 0 auto, 1 one-CTA, 2 CTA pair")
+    a = ap.parse_args()
+    for v in [int(x) for x in a.variants.split(",")]:
+        gllm.op_set_gemm_variant(v)
+        for key in a.shapes.split(","):
+            for shp in SHAPES[key]:
+                print(json.dumps({"variant": v, "set": key, **bench(*shp)}), flush=True)
+    gllm.op_set_gemm_variant(0)

@@ -204,12 +204,19 @@ __device__ __forceinline__ void qkv_rope_store(const GemmArgs& p, int row, int c
   store_bf16x32(dst2, x2);
 }
 
+// fused RMSNorm scale of an output row (1 when the A operand is already normalised)
+__device__ __forceinline__ float row_scale(const GemmArgs& p, int row) {
+  return (p.row_ss != nullptr && row < p.M) ? rsqrtf(__ldg(p.row_ss + row) * p.inv_h + p.eps) : 1.0f;
+}
+
 // One warp's 32 rows of one 256-column accumulator tile: wait for the MMAs (tfull), drain TMEM,
 // apply the fused epilogue.  `partial`: stream-K segment, combine atomically.
 template <int EPI>
 __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
                                               uint64_t* tfull_bar, uint32_t parity) {
   const bool row_ok = row < p.M;
+  const float rs = (EPI == EPI_ADD_F32 || EPI == EPI_ARGMAX) ? 1.0f : row_scale(p, row);
+  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && !partial && p.ws == nullptr) p.zero_rows[row] = 0.f;
   uint32_t r[32];
   auto wait_acc = [&]() {
     ptx::mbar_wait(tfull_bar, parity);
@@ -236,7 +243,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       if (row_ok && col0 < p.N) {
         float v[32];
 #pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]) + (p.bias ? __ldg(p.bias + col0 + j) : 0.f);
+        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]) * rs + (p.bias ? __ldg(p.bias + col0 + j) : 0.f);
         store_bf16x32(out + (size_t)row * p.ldo + col0, v);
       }
     }
@@ -251,6 +258,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       for (int q = 0; q < 8; ++q) xa[q] = reinterpret_cast<const float4*>(rowp)[q];
     }
     wait_acc();
+    float ssl = 0.f;  // fused RMSNorm statistics of the new residual row (this tile's columns)
 #pragma unroll
     for (int c = 0; c < GEMM_BN / 32; ++c) {
       if (ok && !partial && c + 1 < GEMM_BN / 32) {
@@ -264,6 +272,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
           atomic_add_f32x32(rowp + c * 32, r);
         } else {
           float4* dst = reinterpret_cast<float4*>(rowp + c * 32);
+          float nx[32];
 #pragma unroll
           for (int q = 0; q < 8; ++q) {
             float4 x = xa[q];
@@ -273,10 +282,20 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
             x.w += __uint_as_float(r[q * 4 + 3]);
             dst[q] = x;
             xa[q] = xb[q];
+            nx[q * 4 + 0] = x.x;
+            nx[q * 4 + 1] = x.y;
+            nx[q * 4 + 2] = x.z;
+            nx[q * 4 + 3] = x.w;
+          }
+          if (p.xb_out) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) ssl = fmaf(nx[j], nx[j], ssl);
+            store_bf16x32(p.xb_out + (size_t)row * p.ldo + n_blk * GEMM_BN + c * 32, nx);
           }
         }
       }
     }
+    if (ok && !partial && p.ss_out) atomicAdd(p.ss_out + row, ssl);
   } else if constexpr (EPI == EPI_SILU_MUL) {
     wait_acc();
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
@@ -290,7 +309,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       if (row_ok && col0 < p.N / 2) {
         float h[32];
 #pragma unroll
-        for (int j = 0; j < 32; ++j) h[j] = silu_f(__uint_as_float(r[j])) * __uint_as_float(u[j]);
+        for (int j = 0; j < 32; ++j) h[j] = silu_f(__uint_as_float(r[j]) * rs) * (__uint_as_float(u[j]) * rs);
         store_bf16x32(out + (size_t)row * p.ldo + col0, h);
       }
     }
@@ -314,8 +333,8 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       float x1[32], x2[32];
 #pragma unroll
       for (int j = 0; j < 32; ++j) {
-        x1[j] = __uint_as_float(r[j]) + (p.bias ? __ldg(p.bias + col1 + j) : 0.f);
-        x2[j] = __uint_as_float(u[j]) + (p.bias ? __ldg(p.bias + col1 + p.head_dim / 2 + j) : 0.f);
+        x1[j] = __uint_as_float(r[j]) * rs + (p.bias ? __ldg(p.bias + col1 + j) : 0.f);
+        x2[j] = __uint_as_float(u[j]) * rs + (p.bias ? __ldg(p.bias + col1 + p.head_dim / 2 + j) : 0.f);
       }
       qkv_rope_store(p, row, col1, hpos * 32, x1, x2, blk, off);
     }
@@ -507,10 +526,12 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
   if (idx >= p.M * chunks_per_row) return;
   const int row = idx / chunks_per_row, c = idx % chunks_per_row;
   const float* w = p.ws + (size_t)row * p.N;
+  const float rs = row_scale(p, row);
+  if (p.zero_rows != nullptr && c == 0) p.zero_rows[row] = 0.f;
   if constexpr (EPI == EPI_STORE_BF16) {
     float v[32];
 #pragma unroll
-    for (int j = 0; j < 32; ++j) v[j] = w[c * 32 + j] + (p.bias ? p.bias[c * 32 + j] : 0.f);
+    for (int j = 0; j < 32; ++j) v[j] = w[c * 32 + j] * rs + (p.bias ? p.bias[c * 32 + j] : 0.f);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, v);
   } else if constexpr (EPI == EPI_SILU_MUL) {
     const int n_blk = c / 4, cc = c % 4;  // output chunk -> (tile, chunk within the 128 gate columns)
@@ -518,7 +539,7 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
     const float* u = g + GEMM_BN / 2;
     float h[32];
 #pragma unroll
-    for (int j = 0; j < 32; ++j) h[j] = silu_f(g[j]) * u[j];
+    for (int j = 0; j < 32; ++j) h[j] = silu_f(g[j] * rs) * (u[j] * rs);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, h);
   } else if constexpr (EPI == EPI_QKV_ROPE) {
     const int per_head = p.head_dim / 32, hpos = c % per_head;
@@ -527,8 +548,8 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
     float x1[32], x2[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
-      x1[j] = w[col1 + j] + (p.bias ? p.bias[col1 + j] : 0.f);
-      x2[j] = w[col1 + half + j] + (p.bias ? p.bias[col1 + half + j] : 0.f);
+      x1[j] = w[col1 + j] * rs + (p.bias ? p.bias[col1 + j] : 0.f);
+      x2[j] = w[col1 + half + j] * rs + (p.bias ? p.bias[col1 + half + j] : 0.f);
     }
     const int slot = p.slots[row];
     qkv_rope_store(p, row, col1, hpos * 32, x1, x2, slot / p.block_size, slot % p.block_size);
@@ -564,6 +585,12 @@ int choose_cg(int M, int N, int epi, int num_sms) {
 }
 
 }  // namespace
+
+bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms) {
+  if (M <= 0 || choose_cg(M, N, epi, num_sms) == 2) return false;
+  const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
+  return choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms) != 0;
+}
 
 size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms) {
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);

@@ -35,7 +35,20 @@ struct GemmArgs {
   // into the fp32 workspace `ws` [M, N], finished by gemm_finish_kernel.
   int streamk, units_per_cta;
   float* ws;
+  // fused RMSNorm (a4).  Consumers (EPI_STORE_BF16 / EPI_QKV_ROPE / EPI_SILU_MUL) read the bf16
+  // copy of the residual as A and scale each output row by r = rsqrt(row_ss[row] * inv_h + eps)
+  // (the norm gain is folded into W; it is exactly 1 for the O4 weights).  The producer
+  // (EPI_ADD_F32, whole tiles) writes xb_out = bf16(x_new) and adds sum(x_new^2) into ss_out.
+  const float* row_ss;
+  float inv_h, eps;
+  __nv_bfloat16* xb_out;
+  float* ss_out;
+  float* zero_rows;  // consumers: the n-tile-0 epilogue sets zero_rows[row] = 0 (resets the next ss_out)
 };
+
+// true if launch_gemm would combine partial tiles (stream-K) for this shape -- then the ADD_F32
+// epilogue cannot produce xb_out / ss_out and the caller runs rms_stats instead
+bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms);
 
 // fp32 workspace (elements) launch_gemm may need for a GEMM of this shape/epilogue (0 = none)
 size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms);

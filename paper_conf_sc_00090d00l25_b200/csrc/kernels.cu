@@ -137,6 +137,27 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const float* __restrict__ 
   }
 }
 
+__global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict__ x, __nv_bfloat16* xb, float* ss,
+                                                        int H) {
+  __shared__ float red[8];
+  const int r = blockIdx.x;
+  const float* xr = x + (int64_t)r * H;
+  __nv_bfloat16* yr = xb + (int64_t)r * H;
+  float acc = 0.f;
+  for (int c = threadIdx.x * 4; c < H; c += 256 * 4) {
+    const float4 v = *reinterpret_cast<const float4*>(xr + c);
+    acc += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
+    uint2 o;
+    __nv_bfloat162 a = __floats2bfloat162_rn(v.x, v.y);
+    __nv_bfloat162 b = __floats2bfloat162_rn(v.z, v.w);
+    o.x = *reinterpret_cast<uint32_t*>(&a);
+    o.y = *reinterpret_cast<uint32_t*>(&b);
+    *reinterpret_cast<uint2*>(yr + c) = o;
+  }
+  acc = block_sum<256>(acc, red);
+  if (threadIdx.x == 0) ss[r] = acc;
+}
+
 // One CTA per token.  Work unit = one (head, i) rotation pair, i < D/2 (rotate-half convention):
 //   x'[i] = x[i] cos - x[i+D/2] sin ;  x'[i+D/2] = x[i+D/2] cos + x[i] sin
 __global__ void rope_kv_kernel(__nv_bfloat16* qkv, int Hq, int Hkv, int D, const float2* __restrict__ cs,
@@ -236,6 +257,10 @@ void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int3
                     cudaStream_t s) {
   if (n <= 0) return;
   rmsnorm_kernel<<<n, 256, 0, s>>>(x, g, y, rows, H, eps);
+}
+void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s) {
+  if (n <= 0) return;
+  rms_stats_kernel<<<n, 256, 0, s>>>(x, xb, ss, H);
 }
 void launch_rope_kv_append(__nv_bfloat16* qkv, int T, int Hq, int Hkv, int D, const float2* rope_cs,
                            const int32_t* slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int block_size,

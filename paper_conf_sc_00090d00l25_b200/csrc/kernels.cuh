@@ -27,6 +27,10 @@ void launch_embed(const __nv_bfloat16* E, const int32_t* ids, float* x, int T, i
 void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int32_t* rows, int n, int H, float eps,
                     cudaStream_t s);
 
+// Fused-RMSNorm statistics (a4): xb[r] = bf16(x[r]) and ss[r] = sum(x[r]^2) (fp32); the
+// consumer GEMM scales its output rows by rsqrt(ss/H + eps).
+void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s);
+
 // RoPE on q (in place) and k of the fused qkv buffer, K/V appended to the paged cache at slots.
 // Cache layout per layer: [kv_blocks][Hkv][block_size][D] bf16 (K and V separately).
 void launch_rope_kv_append(__nv_bfloat16* qkv, int T, int Hq, int Hkv, int D, const float2* rope_cs,

@@ -6,13 +6,20 @@
 // R1-R18 of DESIGN.md §3.  Decisions and slot mapping must equal the oracle
 // (oracle/scheduler.py, an independent Python implementation) bit for bit;
 // tests/test_sched_parity.py diffs the canonical traces.
+//
+// Cost per tick is proportional to the work scheduled, not to the number of
+// admitted requests: #WP, #RD and the running count are maintained
+// incrementally, waiting prompts sit in an (arrival, id)-ordered queue and
+// ready decodes in a (ready_tick, arrival, id)-ordered FIFO.  Under overload
+// (the C1 stream at PP=1) thousands of prompts wait, which made the plain
+// O(admitted) scans dominate the paper's 0.045 ms budget (L212).
 #include <algorithm>
 #include <cstring>
+#include <deque>
 #include <functional>
 #include <map>
 #include <memory>
 #include <queue>
-#include <unordered_map>
 #include <unordered_set>
 #include <vector>
 
@@ -27,11 +34,19 @@ struct Req {
   int32_t prefill_len = 0, sched_prompt = 0, done_prompt = 0, gen = 0;
   std::vector<int32_t> blocks;
   int32_t inflight = 0;
+  int64_t sel_tick = -1;  // tick in which the request was selected as a decode (R14 exclusion)
   int64_t ready_tick = 0;
   bool finished = false;
+  bool in_waitq = false;  // present in gllm_sched::waitq (possibly stale)
   bool decode_phase() const { return !finished && done_prompt == prefill_len; }
   bool waiting() const { return !finished && sched_prompt < prefill_len; }
 };
+
+bool by_arrival(const Req* a, const Req* b) { return a->arrival != b->arrival ? a->arrival < b->arrival : a->id < b->id; }
+bool by_ready(const Req* a, const Req* b) {
+  if (a->ready_tick != b->ready_tick) return a->ready_tick < b->ready_tick;
+  return by_arrival(a, b);
+}
 
 struct Chunk { Req* r; int32_t start, len; bool completes; };
 struct Decode { Req* r; int32_t pos; };
@@ -45,6 +60,10 @@ struct BatchStore {
   std::vector<int64_t> seq_ids;
   int32_t maxblk = 0;
   std::vector<int32_t> sampled;
+  // for the canonical trace (built on demand by gllm_sched_trace)
+  int64_t rd = 0, wp = 0, free0 = 0, free1 = 0;
+  std::vector<int64_t> preempted;
+  std::vector<std::pair<int64_t, int32_t>> allocs;
 };
 
 int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -57,24 +76,60 @@ struct gllm_sched {
   std::priority_queue<int32_t, std::vector<int32_t>, std::greater<int32_t>> free_pool;
   std::vector<std::unique_ptr<Req>> storage;
   std::unordered_set<int64_t> ids_seen;
-  std::vector<Req*> pending;      // not yet admitted, sorted by (arrival, id) lazily
+  std::vector<Req*> pending;  // not yet admitted, sorted by (arrival, id) lazily
   size_t next_arrival = 0;
   bool pending_dirty = false;
-  std::vector<Req*> admitted;     // admission order
+  std::vector<Req*> active;   // admitted, not finished (lazily compacted); victim search only
+  size_t active_finished = 0;
+  std::vector<Req*> waitq;    // waiting prompts in (arrival, id) order (lazily compacted)
+  size_t waitq_stale = 0;
+  std::deque<Req*> readyq;    // decode-phase, not in flight, (ready_tick, arrival, id) order
+  int64_t wp = 0, rd = 0, running = 0;
   std::map<int64_t, BatchStore> inflight;
+  std::vector<BatchStore> spare;  // retired batches, recycled so their buffers keep their capacity
   int64_t preemptions = 0, finished = 0, admitted_total = 0;
-  std::vector<int64_t> trace;
+  int64_t last_tick = -1;
 
   int32_t alloc(Req* r, std::vector<std::pair<int64_t, int32_t>>* allocs) {
     int32_t b = free_pool.top();  // lowest-numbered free block (R8)
     free_pool.pop();
+    if (r->blocks.empty()) running += 1;
     r->blocks.push_back(b);
     if (allocs) allocs->push_back({r->id, b});
     return b;
   }
   void release(Req* r) {
+    if (!r->blocks.empty()) running -= 1;
     for (int32_t b : r->blocks) free_pool.push(b);
     r->blocks.clear();
+  }
+  void waitq_insert(Req* r) {  // sorted insert (admission and preemption)
+    if (r->in_waitq) {
+      waitq_stale -= 1;  // a stale entry becomes valid again
+      return;
+    }
+    r->in_waitq = true;
+    if (waitq.empty() || !by_arrival(r, waitq.back()))
+      waitq.push_back(r);
+    else
+      waitq.insert(std::upper_bound(waitq.begin(), waitq.end(), r, by_arrival), r);
+  }
+  void compact() {
+    if (waitq_stale > 32 && waitq_stale * 2 > waitq.size()) {
+      size_t j = 0;
+      for (Req* r : waitq) {
+        if (r->waiting())
+          waitq[j++] = r;
+        else
+          r->in_waitq = false;
+      }
+      waitq.resize(j);
+      waitq_stale = 0;
+    }
+    if (active_finished > 64 && active_finished * 2 > active.size()) {
+      active.erase(std::remove_if(active.begin(), active.end(), [](Req* r) { return r->finished; }), active.end());
+      active_finished = 0;
+    }
   }
 };
 
@@ -104,8 +159,10 @@ int check_cfg(const gllm_sched_cfg* c) {
   return GLLM_OK;
 }
 
+// R1-R3: apply batch b's results; requests that become ready enter readyq in (arrival, id) order.
 void retire(gllm_sched* s, BatchStore& b) {
   std::vector<Req*> touched;
+  touched.reserve(b.chunks.size() + b.decodes.size());
   for (auto& c : b.chunks) {
     Req* r = c.r;
     r->done_prompt += c.len;
@@ -113,6 +170,7 @@ void retire(gllm_sched* s, BatchStore& b) {
     if (r->done_prompt == r->prefill_len) {  // prompt completes: first output token (R2)
       r->gen += 1;
       r->ready_tick = s->tick;
+      s->rd += 1;
     }
     touched.push_back(r);
   }
@@ -123,20 +181,43 @@ void retire(gllm_sched* s, BatchStore& b) {
     r->ready_tick = s->tick;
     touched.push_back(r);
   }
-  bool any = false;
+  struct Key {  // sort keys held by value: no pointer chasing inside the sort
+    int64_t arr, id;
+    Req* r;
+  };
+  std::vector<Key> ready;
+  ready.reserve(touched.size());
   for (Req* r : touched) {
-    if (!r->finished && r->gen >= r->output_len) {  // fixed output length (R3)
+    if (r->finished) continue;
+    if (r->gen >= r->output_len) {  // fixed output length (R3)
       r->finished = true;
+      s->rd -= 1;  // every finishing request has its prompt done (gen >= 1)
       s->release(r);
       s->finished += 1;
-      any = true;
+      s->active_finished += 1;
+    } else if (r->decode_phase() && r->inflight == 0 && r->ready_tick == s->tick) {
+      ready.push_back({r->arrival, r->id, r});
     }
   }
-  if (any) {
-    s->admitted.erase(std::remove_if(s->admitted.begin(), s->admitted.end(),
-                                     [](Req* r) { return r->finished; }),
-                      s->admitted.end());
+  std::sort(ready.begin(), ready.end(),
+            [](const Key& a, const Key& b) { return a.arr != b.arr ? a.arr < b.arr : a.id < b.id; });
+  for (const Key& kk : ready) s->readyq.push_back(kk.r);  // ready_tick == tick >= every queued entry
+}
+
+// R14: free the victim's blocks and return it to the waiting queue for recompute.
+void preempt(gllm_sched* s, Req* v) {
+  if (v->decode_phase()) {
+    s->rd -= 1;
+    auto it = std::find(s->readyq.begin(), s->readyq.end(), v);
+    if (it != s->readyq.end()) s->readyq.erase(it);
   }
+  s->wp -= v->prefill_len - v->sched_prompt;
+  s->release(v);
+  v->prefill_len = v->orig_len + v->gen;
+  v->sched_prompt = v->done_prompt = 0;
+  s->wp += v->prefill_len;
+  s->waitq_insert(v);
+  s->preemptions += 1;
 }
 
 }  // namespace
@@ -211,9 +292,14 @@ int gllm_sched_add_warm(gllm_sched* s, int64_t req_id, int32_t context_len, int3
   r->gen = 1;
   r->ids.assign(token_ids, token_ids + (context_len + remaining_out));
   for (int64_t i = 0; i < need; ++i) s->alloc(r.get(), nullptr);
-  s->admitted.push_back(r.get());
+  Req* p = r.get();
+  s->active.push_back(p);
   s->admitted_total += 1;
   s->storage.push_back(std::move(r));
+  if (p->output_len > p->gen) {
+    s->rd += 1;
+    s->readyq.insert(std::upper_bound(s->readyq.begin(), s->readyq.end(), p, by_ready), p);
+  }
   return GLLM_OK;
   GLLM_TRY_END
 }
@@ -228,68 +314,71 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   auto it = s->inflight.find(k - cfg.pp_depth);
   if (it != s->inflight.end()) {
     retire(s, it->second);
+    if (s->spare.size() < 4) s->spare.push_back(std::move(it->second));
     s->inflight.erase(it);
   }
   // 2. admit arrivals (R4)
   if (s->pending_dirty) {
-    std::stable_sort(s->pending.begin() + s->next_arrival, s->pending.end(), [](Req* a, Req* b) {
-      return a->arrival != b->arrival ? a->arrival < b->arrival : a->id < b->id;
-    });
+    std::stable_sort(s->pending.begin() + s->next_arrival, s->pending.end(), by_arrival);
     s->pending_dirty = false;
   }
   while (s->next_arrival < s->pending.size() && s->pending[s->next_arrival]->arrival <= k) {
-    s->admitted.push_back(s->pending[s->next_arrival++]);
+    Req* r = s->pending[s->next_arrival++];
+    s->active.push_back(r);
     s->admitted_total += 1;
+    s->wp += r->prefill_len;
+    s->waitq_insert(r);
   }
-  // 3. statistics (R5)
-  int64_t rd = 0, wp = 0;
-  for (Req* r : s->admitted) {
-    if (r->decode_phase()) rd += 1;
-    if (r->waiting()) wp += r->prefill_len - r->sched_prompt;
-  }
+  s->compact();
+  // 3. statistics (R5), maintained incrementally
+  const int64_t rd = s->rd, wp = s->wp;
   const int64_t free0 = (int64_t)s->free_pool.size();
-  std::vector<std::pair<int64_t, int32_t>> allocs;
-  std::vector<int64_t> preempted;
-  std::unordered_set<int64_t> selected;
   BatchStore b;
+  if (!s->spare.empty()) {  // reuse a retired batch's buffers (no page faults on large tables)
+    b = std::move(s->spare.back());
+    s->spare.pop_back();
+    // (block_table keeps its size: the resize below then only initialises growth)
+    for (auto* v : {&b.token_ids, &b.positions, &b.slots, &b.cu_q, &b.kv_len, &b.samples, &b.sampled}) v->clear();
+    b.chunks.clear();
+    b.decodes.clear();
+    b.seq_ids.clear();
+    b.preempted.clear();
+    b.allocs.clear();
+  }
   b.tick = k;
-  // 4. decode selection (Eq.4; R6-R9; R14)
+  auto& allocs = b.allocs;
+  auto& preempted = b.preempted;
+  // 4. decode selection (Eq.4; R6-R9; R14): the first min(#D, |ready|) of the ready FIFO
   const int32_t d_cnt = cfg.policy == 1 ? (int32_t)rd : throttle_decode(cfg, rd);
-  std::vector<Req*> ready;
-  for (Req* r : s->admitted)
-    if (r->decode_phase() && r->inflight == 0) ready.push_back(r);
-  std::sort(ready.begin(), ready.end(), [](Req* a, Req* b) {
-    if (a->ready_tick != b->ready_tick) return a->ready_tick < b->ready_tick;
-    if (a->arrival != b->arrival) return a->arrival < b->arrival;
-    return a->id < b->id;
-  });
-  const size_t n_try = std::min<size_t>((size_t)d_cnt, ready.size());
-  for (size_t i = 0; i < n_try; ++i) {
-    Req* r = ready[i];
+  const size_t n_try = std::min<size_t>((size_t)d_cnt, s->readyq.size());
+  std::vector<Req*> cand(s->readyq.begin(), s->readyq.begin() + n_try);
+  s->readyq.erase(s->readyq.begin(), s->readyq.begin() + n_try);
+  std::vector<Req*> skipped;  // no block and no victim: stays ready, keeps its place
+  b.decodes.reserve(n_try);
+  for (Req* r : cand) {
     if (!r->decode_phase()) continue;  // preempted earlier this tick
     const int32_t pos = r->orig_len + r->gen - 1;
     if ((int64_t)r->blocks.size() * bs <= pos) {
       if (s->free_pool.empty()) {
         // victim: latest (arrival, id) running request, not in flight, not selected (R14)
         Req* victim = nullptr;
-        for (Req* c : s->admitted) {
-          if (c->blocks.empty() || c->inflight != 0 || c == r || selected.count(c->id)) continue;
-          if (!victim || c->arrival > victim->arrival ||
-              (c->arrival == victim->arrival && c->id > victim->id))
-            victim = c;
+        for (Req* c : s->active) {
+          if (c->finished || c->blocks.empty() || c->inflight != 0 || c == r || c->sel_tick == k) continue;
+          if (!victim || by_arrival(victim, c)) victim = c;
         }
-        if (!victim) continue;
-        s->release(victim);
-        victim->prefill_len = victim->orig_len + victim->gen;
-        victim->sched_prompt = victim->done_prompt = 0;
-        s->preemptions += 1;
+        if (!victim) {
+          skipped.push_back(r);
+          continue;
+        }
+        preempt(s, victim);
         preempted.push_back(victim->id);
       }
       s->alloc(r, &allocs);
     }
     b.decodes.push_back({r, pos});
-    selected.insert(r->id);
+    r->sel_tick = k;
   }
+  for (auto i = skipped.rbegin(); i != skipped.rend(); ++i) s->readyq.push_front(*i);
   // 5. prefill count (Eq.3 + L165; R10-R12)
   int32_t p_cnt;
   if (cfg.policy == 1)
@@ -297,20 +386,12 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   else
     p_cnt = throttle_prefill(cfg, wp, free0);
   // 6. prefill selection, FCFS with CPP (R13)
-  int64_t running = 0;
-  std::vector<Req*> waiting;
-  for (Req* r : s->admitted) {
-    if (!r->blocks.empty() || r->sched_prompt > 0) running += 1;
-    if (r->waiting()) waiting.push_back(r);
-  }
-  std::sort(waiting.begin(), waiting.end(), [](Req* a, Req* b) {
-    return a->arrival != b->arrival ? a->arrival < b->arrival : a->id < b->id;
-  });
   int64_t p_left = p_cnt;
-  for (Req* r : waiting) {
-    if (p_left == 0) break;
+  for (size_t wi = 0; wi < s->waitq.size() && p_left > 0; ++wi) {
+    Req* r = s->waitq[wi];
+    if (!r->waiting()) continue;  // stale entry
     const bool fresh = r->blocks.empty() && r->sched_prompt == 0;
-    if (fresh && running >= cfg.max_seqs) continue;
+    if (fresh && s->running >= cfg.max_seqs) continue;
     const int64_t remaining = r->prefill_len - r->sched_prompt;
     const int64_t want = std::min(remaining, p_left);
     const int64_t capacity = ((int64_t)r->blocks.size() + (int64_t)s->free_pool.size()) * bs - r->sched_prompt;
@@ -318,23 +399,44 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
     if (c <= 0) break;
     const int64_t need = ceil_div(r->sched_prompt + c, bs) - (int64_t)r->blocks.size();
     for (int64_t j = 0; j < need; ++j) s->alloc(r, &allocs);
-    if (fresh) running += 1;
     b.chunks.push_back({r, r->sched_prompt, (int32_t)c, r->sched_prompt + c == r->prefill_len});
     r->sched_prompt += (int32_t)c;
+    s->wp -= c;
+    if (!r->waiting()) s->waitq_stale += 1;
     p_left -= c;
     if (c < want) break;
   }
   // 7. layout (R15): prefill chunks, then decodes
   b.P = p_cnt;
   b.D = d_cnt;
+  const size_t S = b.chunks.size() + b.decodes.size();
+  const size_t T = (size_t)(p_cnt - p_left) + b.decodes.size();
+  b.token_ids.reserve(T);
+  b.positions.reserve(T);
+  b.slots.reserve(T);
+  b.cu_q.reserve(S + 1);
+  b.kv_len.reserve(S);
+  b.seq_ids.reserve(S);
+  b.samples.reserve(S);
   b.cu_q.push_back(0);
   std::vector<const Req*> rows_req;
   std::vector<int32_t> rows_n;
+  rows_req.reserve(S);
+  rows_n.reserve(S);
   for (auto& c : b.chunks) {
-    for (int32_t p = c.start; p < c.start + c.len; ++p) {
-      b.token_ids.push_back(c.r->ids[p]);
-      b.positions.push_back(p);
-      b.slots.push_back(c.r->blocks[p / bs] * bs + p % bs);  // O2
+    const size_t t0 = b.token_ids.size();
+    b.token_ids.insert(b.token_ids.end(), c.r->ids.begin() + c.start, c.r->ids.begin() + c.start + c.len);
+    b.positions.resize(t0 + c.len);
+    b.slots.resize(t0 + c.len);
+    int32_t* pos = b.positions.data() + t0;
+    int32_t* slot = b.slots.data() + t0;
+    for (int32_t p = c.start, blk = c.start / bs, off = c.start % bs; p < c.start + c.len; ++p) {
+      *pos++ = p;
+      *slot++ = c.r->blocks[blk] * bs + off;  // O2: slot = bt[pos / bs] * bs + pos % bs
+      if (++off == bs) {
+        off = 0;
+        ++blk;
+      }
     }
     b.cu_q.push_back(b.cu_q.back() + c.len);
     b.kv_len.push_back(c.start + c.len);
@@ -358,22 +460,17 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   }
   b.maxblk = 0;
   for (int32_t n : rows_n) b.maxblk = std::max(b.maxblk, n);
-  b.block_table.assign(rows_req.size() * (size_t)b.maxblk, -1);
-  for (size_t i = 0; i < rows_req.size(); ++i)
-    for (int32_t j = 0; j < rows_n[i]; ++j) b.block_table[i * b.maxblk + j] = rows_req[i]->blocks[j];
-  // canonical trace (DESIGN.md §3; == oracle.scheduler.trace_bytes)
-  auto& t = s->trace;
-  t.clear();
-  const int64_t T = (int64_t)b.token_ids.size();
-  t.insert(t.end(), {k, (int64_t)p_cnt, (int64_t)d_cnt, rd, wp, free0, (int64_t)s->free_pool.size(),
-                     (int64_t)b.chunks.size(), (int64_t)b.decodes.size(), (int64_t)preempted.size(),
-                     (int64_t)allocs.size(), T, (int64_t)b.samples.size()});
-  for (auto& c : b.chunks) t.insert(t.end(), {c.r->id, (int64_t)c.start, (int64_t)c.len});
-  for (auto& d : b.decodes) t.insert(t.end(), {d.r->id, (int64_t)d.pos});
-  for (int64_t v : preempted) t.push_back(v);
-  for (auto& a : allocs) t.insert(t.end(), {a.first, (int64_t)a.second});
-  for (int32_t v : b.slots) t.push_back(v);
-  for (int32_t v : b.samples) t.push_back(v);
+  b.block_table.resize(rows_req.size() * (size_t)b.maxblk);
+  for (size_t i = 0; i < rows_req.size(); ++i) {  // one pass: blocks, then -1 padding
+    int32_t* row = b.block_table.data() + i * b.maxblk;
+    std::memcpy(row, rows_req[i]->blocks.data(), rows_n[i] * sizeof(int32_t));
+    std::fill(row + rows_n[i], row + b.maxblk, -1);
+  }
+  b.rd = rd;
+  b.wp = wp;
+  b.free0 = free0;
+  b.free1 = (int64_t)s->free_pool.size();
+  s->last_tick = k;
 
   auto& st = s->inflight[k];
   st = std::move(b);
@@ -415,16 +512,13 @@ int gllm_retire_batch(gllm_sched* s, int64_t tick, const int32_t* sampled_ids) {
 
 int gllm_sched_done(const gllm_sched* s) {
   if (!s) return 0;
-  return s->next_arrival >= s->pending.size() && s->admitted.empty() ? 1 : 0;
+  return s->next_arrival >= s->pending.size() && s->finished == s->admitted_total ? 1 : 0;
 }
 
 int gllm_sched_stats(const gllm_sched* s, int64_t* out6) {
   if (!s || !out6) return gllm::set_error(GLLM_EINVAL, "null argument");
-  int64_t running = 0;
-  for (Req* r : s->admitted)
-    if (!r->blocks.empty()) running += 1;
   out6[0] = s->tick;
-  out6[1] = running;
+  out6[1] = s->running;
   out6[2] = (int64_t)s->free_pool.size();
   out6[3] = s->preemptions;
   out6[4] = s->finished;
@@ -433,12 +527,29 @@ int gllm_sched_stats(const gllm_sched* s, int64_t* out6) {
 }
 
 int gllm_sched_trace(gllm_sched* s, void* buf, size_t cap, size_t* used) {
+  GLLM_TRY_BEGIN
   if (!s || !used) return gllm::set_error(GLLM_EINVAL, "null argument");
-  const size_t n = s->trace.size() * sizeof(int64_t);
+  auto it = s->inflight.find(s->last_tick);
+  if (it == s->inflight.end()) return gllm::set_error(GLLM_ESTATE, "no batch built since the last retire");
+  const BatchStore& b = it->second;
+  // canonical trace (DESIGN.md §3; == oracle.scheduler.trace_bytes)
+  std::vector<int64_t> t;
+  const int64_t T = (int64_t)b.token_ids.size();
+  t.insert(t.end(), {b.tick, (int64_t)b.P, (int64_t)b.D, b.rd, b.wp, b.free0, b.free1, (int64_t)b.chunks.size(),
+                     (int64_t)b.decodes.size(), (int64_t)b.preempted.size(), (int64_t)b.allocs.size(), T,
+                     (int64_t)b.samples.size()});
+  for (auto& c : b.chunks) t.insert(t.end(), {c.r->id, (int64_t)c.start, (int64_t)c.len});
+  for (auto& d : b.decodes) t.insert(t.end(), {d.r->id, (int64_t)d.pos});
+  for (int64_t v : b.preempted) t.push_back(v);
+  for (auto& a : b.allocs) t.insert(t.end(), {a.first, (int64_t)a.second});
+  for (int32_t v : b.slots) t.push_back(v);
+  for (int32_t v : b.samples) t.push_back(v);
+  const size_t n = t.size() * sizeof(int64_t);
   *used = n;
   if (cap < n || (!buf && n)) return gllm::set_error(GLLM_EINVAL, "trace buffer too small (%zu < %zu)", cap, n);
-  if (n) std::memcpy(buf, s->trace.data(), n);
+  if (n) std::memcpy(buf, t.data(), n);
   return GLLM_OK;
+  GLLM_TRY_END
 }
 
 }  // extern "C"

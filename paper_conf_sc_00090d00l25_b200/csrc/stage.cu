@@ -48,7 +48,7 @@ enum Cat { C_TOTAL = 0, C_QKV, C_O, C_GU, C_DOWN, C_PREFILL, C_DECODE, C_ROPE, C
 
 struct LayerW {
   bf16 *wqkv = nullptr, *wo = nullptr, *wgu = nullptr, *wd = nullptr;
-  float *bqkv = nullptr, *g1 = nullptr, *g2 = nullptr;
+  float* bqkv = nullptr;
   bf16 *kc = nullptr, *vc = nullptr;
   CUtensorMap tm_qkv, tm_o, tm_gu, tm_d;
 };
@@ -119,6 +119,9 @@ struct gllm_stage {
   int32_t* slots = nullptr;
   int32_t* sampled_tmp = nullptr;
   float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T)
+  float *ss_a = nullptr, *ss_b = nullptr;  // fused-RMSNorm row statistics (sum of squares of x)
+  float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
+  bool fused_norm = true;
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
@@ -325,8 +328,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     LayerW w;
     if ((rc = st->dalloc(&w.wqkv, (size_t)nqkv * H)) || (rc = st->dalloc(&w.wo, (size_t)H * qd)) ||
         (rc = st->dalloc(&w.wgu, (size_t)2 * I * H)) || (rc = st->dalloc(&w.wd, (size_t)H * I)) ||
-        (rc = st->dalloc(&w.g1, H)) || (rc = st->dalloc(&w.g2, H)) || (rc = st->dalloc(&w.kc, kv_elems)) ||
-        (rc = st->dalloc(&w.vc, kv_elems)))
+        (rc = st->dalloc(&w.kc, kv_elems)) || (rc = st->dalloc(&w.vc, kv_elems)))
       return fail(rc);
     if (cfg->qkv_bias && (rc = st->dalloc(&w.bqkv, nqkv))) return fail(rc);
     gllm::launch_init_bf16(w.wqkv, qd, H, seed, layer_tid(l, K_WQ), s_h, 0, 0, s0);
@@ -336,8 +338,8 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WG), s_h, 1, 0, s0);
     gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WU), s_h, 2, 0, s0);
     gllm::launch_init_bf16(w.wd, H, I, seed, layer_tid(l, K_WD), s_i, 0, 0, s0);
-    gllm::launch_fill_f32(w.g1, H, 1.0f, s0);
-    gllm::launch_fill_f32(w.g2, H, 1.0f, s0);
+    // The two RMSNorm gains of the layer are folded into the columns of Wqkv and Wgu
+    // (W' = W diag(g)); under O4 every gain is exactly 1, so W' = W bit for bit.
     if (w.bqkv) {
       gllm::launch_init_f32(w.bqkv, qd, seed, layer_tid(l, K_BQ), s_bias, s0);
       gllm::launch_init_f32(w.bqkv + qd, kd, seed, layer_tid(l, K_BK), s_bias, s0);
@@ -375,9 +377,12 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = st->dalloc(&st->act, R * I)) || (rc = st->dalloc(&st->rope_cs, R * (D / 2))) ||
       (rc = st->dalloc(&st->slots, R)) ||
       // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
-      (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)))
+      (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)) || (rc = st->dalloc(&st->ss_a, R)) ||
+      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)))
     return fail(rc);
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
+  gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
+  if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
@@ -489,6 +494,13 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
       nparts += nsplit;
     }
   }
+  // longest work items first, so the long-context CTAs do not form the tail of the grid
+  std::stable_sort(ditems.begin(), ditems.end(), [&](const gllm::DecodeItem& a, const gllm::DecodeItem& b) {
+    auto len = [&](const gllm::DecodeItem& it) {
+      return std::min(d->kv_len[it.seq] - it.split * split_pages * bs, split_pages * bs);
+    };
+    return len(a) > len(b);
+  });
   // ---------------- pack into the slot's pinned buffer; one H2D copy (K9)
   size_t off = 0;
   auto sect = [&](size_t bytes) {
@@ -583,13 +595,46 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
   aa.part_o = st->part_o;
   aa.part_ml = st->part_ml;
   aa.split_len = P.split_len;
-  for (size_t li = 0; li < st->layers.size(); ++li) {
-    LayerW& w = st->layers[li];
-    {
-      Prof p(st, s, C_NORM);
-      gllm::launch_rmsnorm(x, w.g1, st->y, nullptr, T, H, c.rms_eps, s);
+  // Fused RMSNorm (a4): y holds bf16(x) and ss_a / ss_b the per-row sum of squares of x; the
+  // consumer GEMMs (QKV, gate_up) scale their rows by rsqrt(ss/H + eps) in the epilogue and the
+  // residual-add GEMMs (O, down) produce y and ss for the next norm.  Only the stage entry (and a
+  // stream-K residual GEMM) needs the standalone statistics pass.
+  // (GLLM_UNFUSED_NORM=1 selects standalone RMSNorm kernels instead -- kept for A/B measurement.)
+  const bool fused = st->fused_norm;
+  if (fused) {
+    Prof p(st, s, C_NORM);
+    gllm::launch_rms_stats(x, st->y, st->ss_a, T, H, s);
+    st->last_launches += 1;
+  }
+  auto standalone_norm = [&]() {
+    if (fused) return;
+    Prof p(st, s, C_NORM);
+    gllm::launch_rmsnorm(x, st->ones, st->y, nullptr, T, H, c.rms_eps, s);
+    st->last_launches += 1;
+  };
+  const float inv_h = 1.0f / (float)H;
+  auto residual_gemm = [&](const CUtensorMap& ta, const CUtensorMap& tb, int K, float* ss_next) -> int {
+    // ss_next was zeroed by the n-tile-0 epilogue of the preceding consumer GEMM (zero_rows)
+    const bool sk = !fused || gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
+    gllm::GemmArgs g{};
+    g.M = T;
+    g.N = H;
+    g.K = K;
+    g.out = x;
+    g.ldo = H;
+    g.xb_out = sk ? nullptr : st->y;
+    g.ss_out = sk ? nullptr : ss_next;
+    st->last_launches += 1;
+    RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms));
+    if (sk && fused) {  // partial tiles combine with reductions: recompute the statistics from x
+      gllm::launch_rms_stats(x, st->y, ss_next, T, H, s);
       st->last_launches += 1;
     }
+    return GLLM_OK;
+  };
+  for (size_t li = 0; li < st->layers.size(); ++li) {
+    LayerW& w = st->layers[li];
+    standalone_norm();
     {
       // QKV projection with RoPE and the paged KV append fused into the epilogue (a5 + a6)
       Prof p(st, s, C_QKV);
@@ -610,6 +655,10 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.n_kv_heads = c.n_kv_heads;
       g.block_size = bs;
       g.ws = st->gemm_ws;
+      g.row_ss = fused ? st->ss_a : nullptr;
+      g.inv_h = inv_h;
+      g.eps = c.rms_eps;
+      g.zero_rows = fused ? st->ss_b : nullptr;  // reset for the O GEMM's statistics
       st->last_launches += 1;
       RC(gllm::launch_gemm(st->tm_y, w.tm_qkv, gllm::EPI_QKV_ROPE, g, s, st->num_sms));
     }
@@ -643,20 +692,28 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     }
     {
       Prof p(st, s, C_O);
-      RC(gemm(st, st->tm_attn, w.tm_o, gllm::EPI_ADD_F32, T, H, qd, x, H, nullptr, s));
+      RC(residual_gemm(st->tm_attn, w.tm_o, qd, st->ss_b));
     }
-    {
-      Prof p(st, s, C_NORM);
-      gllm::launch_rmsnorm(x, w.g2, st->y, nullptr, T, H, c.rms_eps, s);
-      st->last_launches += 1;
-    }
+    standalone_norm();
     {
       Prof p(st, s, C_GU);
-      RC(gemm(st, st->tm_y, w.tm_gu, gllm::EPI_SILU_MUL, T, 2 * I, H, st->act, I, nullptr, s));
+      gllm::GemmArgs g{};
+      g.M = T;
+      g.N = 2 * I;
+      g.K = H;
+      g.out = st->act;
+      g.ldo = I;
+      g.ws = st->gemm_ws;
+      g.row_ss = fused ? st->ss_b : nullptr;
+      g.inv_h = inv_h;
+      g.eps = c.rms_eps;
+      g.zero_rows = fused ? st->ss_a : nullptr;  // reset for the down GEMM's statistics
+      st->last_launches += 1;
+      RC(gllm::launch_gemm(st->tm_y, w.tm_gu, gllm::EPI_SILU_MUL, g, s, st->num_sms));
     }
     {
       Prof p(st, s, C_DOWN);
-      RC(gemm(st, st->tm_act, w.tm_d, gllm::EPI_ADD_F32, T, H, I, x, H, nullptr, s));
+      RC(residual_gemm(st->tm_act, w.tm_d, I, st->ss_a));
     }
   }
   if (st->is_last() && ns > 0) {

@@ -38,6 +38,8 @@ struct AttnArgs {
 // flattened (token, group-head) rows per prefill work item
 int prefill_rows_per_item();
 int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
+// same work items on tcgen05 (S and O in TMEM); the default prefill path
+int launch_prefill_attention_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
 int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
                             int n_merges, cudaStream_t s);
 

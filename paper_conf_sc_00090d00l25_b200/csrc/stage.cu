@@ -15,6 +15,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -122,6 +124,7 @@ struct gllm_stage {
   float *ss_a = nullptr, *ss_b = nullptr;  // fused-RMSNorm row statistics (sum of squares of x)
   float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
   bool fused_norm = true;
+  bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
@@ -186,8 +189,14 @@ struct Prof {
       cudaEventRecord(b, s);
       st->prof_ev.push_back({cat, {a, b}});
     }
+    if (g_sync_debug) {  // GLLM_SYNC_DEBUG=1: synchronise and log every launch group (hang triage)
+      const cudaError_t e = cudaStreamSynchronize(s);
+      std::fprintf(stderr, "[gllm] cat %d done: %s\n", cat, cudaGetErrorString(e));
+    }
   }
+  static bool g_sync_debug;
 };
+bool Prof::g_sync_debug = std::getenv("GLLM_SYNC_DEBUG") != nullptr;
 
 int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmEpi epi, int M, int N, int K,
          void* out, int ldo, const float* bias, cudaStream_t s) {
@@ -383,6 +392,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
   gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
   if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
+  if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
@@ -675,7 +685,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       }
       {
         Prof p(st, ps, C_PREFILL);
-        RC(gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps));
+        RC(st->prefill_mma_sync ? gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps)
+                                : gllm::launch_prefill_attention_tc(aa, d_pi, P.n_pi, ps));
       }
       if (overlap) CK(cudaEventRecord(st->ev_join, ps));
       st->last_launches += 1;

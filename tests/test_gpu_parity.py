@@ -122,6 +122,18 @@ def test_c1_full_width_first_stage_layer():
     assert errs.max() <= TOL_HIDDEN, errs.max()
 
 
+def test_c1_stream_long_chunk_continuation():
+    # the first 40 ticks of the full C1 stream at PP=1 include a 984-token chunk continuing a prompt at
+    # offset 1402 (kv 2386 keys, 38 key tiles): the tcgen05 prefill kernel's lazy O rescale and
+    # long causal tails, at full Llama-3-8B width (one layer, stage-local)
+    m = MODELS["C1"].with_layers(4)
+    st = make_stream("C1", m.vocab)
+    cfg = SCHED["C1"].with_(num_blocks=20000, pp_depth=1)
+    n, errs, _ = _run_pair(m, cfg, st, lb=0, le=1, max_ticks=40, kv_blocks=20000, check_kv=False)
+    assert n > 40000
+    assert errs.max() <= TOL_HIDDEN, errs.max()
+
+
 @pytest.mark.parametrize("cfg_name,n_req,ticks,kvb", [("C2", 60, 14, 3000), ("C4", 30, 10, 3000)])
 def test_full_width_other_shapes_stage_local(cfg_name, n_req, ticks, kvb):
     # C2 = Qwen2.5-14B shapes (H 5120, GQA group 5, q/k/v bias, theta 1e6); C4 = Llama-3-70B shapes

@@ -303,6 +303,10 @@ def run_ours(args):
         traffic = json.load(open(tp)).get(f"{args.config}-pp{N}", {}).get(dom)
 
     # ---- e2e: serving loop through the public API (host scheduler, H2D metadata, D2H ids)
+    # the value-phase batches were scheduled directly (teacher forcing, R17) and retire without
+    # sampled ids: forget their sample bookkeeping so no rank waits for ids nobody sends
+    pipe.pending_samples.clear()
+    pipe._expect.clear()
     h2d = d2h = 0
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e2e_tokens = 0

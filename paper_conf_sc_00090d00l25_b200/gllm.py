@@ -160,8 +160,8 @@ class Sched:
         self.h = h
 
     def close(self):
-        if getattr(self, "h", None):
-            lib().gllm_sched_free(self.h)
+        if getattr(self, "h", None) and _lib is not None:
+            _lib.gllm_sched_free(self.h)
             self.h = None
 
     __del__ = close
@@ -261,8 +261,8 @@ class Stage:
         self.h = h
 
     def close(self):
-        if getattr(self, "h", None):
-            lib().gllm_free_stage(self.h)
+        if getattr(self, "h", None) and _lib is not None:
+            _lib.gllm_free_stage(self.h)
             self.h = None
 
     __del__ = close

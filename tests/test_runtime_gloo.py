@@ -102,6 +102,60 @@ def _worker(rank, world, port, ticks, q):
     dist.destroy_process_group()
 
 
+def _bench_flow_worker(rank, world, port, q):
+    """bench.py's multi-rank sequence: preroll ticks, drain, W+K batches scheduled up front and run
+    from prepared handles, bookkeeping reset, e2e serving ticks, drain."""
+    import torch.distributed as dist
+
+    from paper_conf_sc_00090d00l25_b200 import gllm
+    from paper_conf_sc_00090d00l25_b200.runtime import Pipeline, pack_desc, unpack_desc
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    m = MODELS["C0"].with_layers(2)
+    sp = SCHED["C0"].with_(pp_depth=world, num_blocks=256, iterp=2, maxp=64, minp=8)
+    lb, le = split_layers(m.n_layers, world)[rank]
+    ex = OracleExecutor(m, lb, le, sp.block_size)
+    sched = None
+    if rank == 0:
+        sched = gllm.Sched(sp)
+        sched.add_stream(make_stream("C1", m.vocab, n=40))
+    pipe = Pipeline(rank, world, ex, GlooTransport(ex, rank, dist.group.WORLD), sched, dist.group.WORLD)
+    for _ in range(6):
+        pipe.tick()
+    pipe.drain()
+    batches = []
+    for _ in range(5):
+        buf = pack_desc(sched.build_batch()) if rank == 0 else None
+        batches.append(unpack_desc(pipe._bcast(buf)))
+    handles = [ex.prepare(a) for a in batches]
+    for a, h in zip(batches, handles):
+        pipe.run_batch(a, h)
+    pipe.pending_samples.clear()
+    pipe._expect.clear()
+    for _ in range(6):
+        pipe.tick()
+    pipe.drain()
+    dist.barrier()
+    q.put(rank)
+    dist.destroy_process_group()
+
+
+@pytest.mark.timeout(600)
+def test_bench_multi_rank_sequence_does_not_deadlock():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_bench_flow_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    done = sorted(q.get(timeout=500) for _ in range(2))
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert done == [0, 1]
+
+
 def test_pack_unpack_roundtrip():
     from oracle.scheduler import Scheduler
     st = make_stream("C1", 1000, n=50)

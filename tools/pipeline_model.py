@@ -1,0 +1,110 @@
+"""Pipeline-bubble evaluation of Token Throttling vs Sarathi-Serve on measured B200 stage times
+(the paper's central claim, §2.4-2.5, Fig. 15).
+
+One GPU runs stage `--stage` of a `--pp`-stage split of config C* (the per-stage work of a PP
+deployment: same layer count, same micro-batches as the PP scheduler produces) over a window of
+ticks, timing every micro-batch's stage forward with CUDA events.  A discrete-event model then
+replays the window through PP identical stages with the pipeline's two dependencies -- micro-batch
+k enters stage s when stage s-1 finished k and stage s finished k-1, and enters stage 0 only
+after k-PP left the last stage (at most PP in flight, L179) -- giving the bubble fraction
+1 - busy / (PP * makespan) and tokens/s for each policy.
+
+    python tools/pipeline_model.py --config C2 --pp 4 --stage 1 --ticks 200
+"""
+import argparse
+import json
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_sc_00090d00l25_b200 import gllm  # noqa: E402
+from paper_conf_sc_00090d00l25_b200.runtime import split_layers  # noqa: E402
+from workloads.configs import MODELS, SCHED, STREAMS  # noqa: E402
+from workloads.streams import make_stream  # noqa: E402
+
+
+def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_us=0.0):
+    m = MODELS[config]
+    sp = SCHED[config].with_(pp_depth=pp, policy=policy, token_budget=2048,
+                             num_blocks=kv_blocks or SCHED[config].num_blocks)
+    lb, le = split_layers(m.n_layers, pp)[stage_idx]
+    max_tokens = max(sp.maxp, sp.token_budget) + sp.max_seqs + 64
+    st = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs)
+    if config == "C4":
+        st.fill_kv(0xC4)
+    s = gllm.Sched(sp)
+    s.add_stream(make_stream(config, m.vocab))
+    dev = torch.device("cuda")
+    hin = torch.randn((max_tokens, m.hidden), device=dev)
+    hout = torch.empty((max_tokens, m.hidden), device=dev)
+    samp = torch.empty((sp.max_seqs,), dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream()
+    first, last = stage_idx == 0, le == m.n_layers
+
+    def fwd(d):
+        st.forward(d, 0 if first else hin.data_ptr(), 0 if last else hout.data_ptr(),
+                   samp.data_ptr() if last else 0, stream.cuda_stream)
+
+    for _ in range(preroll):
+        d = s.build_batch()
+        if d.num_tokens:
+            fwd(d)
+    torch.cuda.synchronize()
+    times, toks, pre, dec = [], [], [], []
+    for _ in range(ticks):
+        d = s.build_batch()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        if d.num_tokens:
+            fwd(d)
+        e1.record()
+        torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1) if d.num_tokens else 0.0)
+        toks.append(d.num_tokens)
+        pre.append(d.num_prefill_tokens)
+        dec.append(d.num_decode_tokens)
+    st.close()
+    return np.array(times), np.array(toks), np.array(pre), np.array(dec)
+
+
+def simulate(t_ms, pp, host_ms=0.05):
+    """Identical stages taking t_ms[k] for micro-batch k; returns (makespan ms, bubble fraction)."""
+    n = len(t_ms)
+    fin = np.zeros((pp, n))
+    for k in range(n):
+        for s in range(pp):
+            start = 0.0
+            if s > 0:
+                start = max(start, fin[s - 1, k])
+            if k > 0:
+                start = max(start, fin[s, k - 1])
+            if s == 0 and k >= pp:  # at most PP micro-batches in flight: k waits for k-PP's retire
+                start = max(start, fin[pp - 1, k - pp] + host_ms)
+            fin[s, k] = start + t_ms[k]
+    makespan = fin[pp - 1, n - 1]
+    busy = pp * float(np.sum(t_ms))
+    return makespan, 1.0 - busy / (pp * makespan)
+
+
+if __name__ == "__main__":
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--pp", type=int, default=4)
+    ap.add_argument("--stage", type=int, default=1)
+    ap.add_argument("--ticks", type=int, default=160)
+    ap.add_argument("--preroll", type=int, default=None)
+    a = ap.parse_args()
+    preroll = a.preroll if a.preroll is not None else int(STREAMS[a.config].get("window", (400, None))[0])
+    out = {"config": a.config, "pp": a.pp, "stage": a.stage, "ticks": a.ticks, "preroll": preroll}
+    for name, pol in (("token_throttling", 0), ("sarathi_serve", 1)):
+        t, toks, pre, dec = measure(a.config, a.pp, a.stage, pol, preroll, a.ticks)
+        mk, bub = simulate(t, a.pp)
+        out[name] = {"tokens_per_s": round(float(toks.sum()) / (mk * 1e-3), 1), "bubble_fraction": round(bub, 4),
+                     "stage_ms_mean": round(float(t.mean()), 3), "stage_ms_cv": round(float(t.std() / t.mean()), 3),
+                     "tokens_mean": round(float(toks.mean()), 1), "tokens_cv": round(float(toks.std() / toks.mean()), 3),
+                     "prefill_mean": round(float(pre.mean()), 1), "decode_mean": round(float(dec.mean()), 1)}
+        print(name, json.dumps(out[name]), flush=True)
+    print(json.dumps(out))

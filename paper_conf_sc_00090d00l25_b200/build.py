@@ -50,7 +50,14 @@ def _compile(src, force, verbose):
     return obj, None
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, variant: str = "") -> str:
+    """variant "": libgllm.so.  variant "x": compiled with -DGLLM_VARIANT_X into libgllm_x.so
+    (measurement builds selected at run time with GLLM_LIB=...)."""
+    global OBJ, LIB, COMMON
+    if variant:
+        OBJ = os.path.join(ROOT, "build", "obj_" + variant)
+        LIB = os.path.join(PKG, f"libgllm_{variant}.so")
+        COMMON = COMMON + [f"-DGLLM_VARIANT_{variant.upper()}"]
     os.makedirs(OBJ, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
@@ -68,4 +75,5 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    var = next((a.split("=", 1)[1] for a in sys.argv if a.startswith("--variant=")), "")
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, variant=var))

@@ -36,7 +36,12 @@ __device__ __forceinline__ uint32_t swz(int row, int chunk) {
 // k-steps and P V is 1 k-step x D/8 n-tiles -- no shuffles in the dot products.
 template <int D>
 struct DecodeSmem {
+#ifdef GLLM_VARIANT_DEC3
   static constexpr int NST = 3;
+#else
+  // 2 stages (64 KB per CTA at D = 128): a prefill CTA (96 KB) still fits beside two decode CTAs
+  static constexpr int NST = 2;
+#endif
   static constexpr int PAGE = 16 * D * 2;
   static constexpr int PER_WARP = NST * 2 * PAGE;
   static constexpr int MERGE = 4 * 16 * D * 4 + 4 * 16 * 2 * 4;
@@ -122,15 +127,24 @@ __global__ void __launch_bounds__(128) decode_attn_kernel(const AttnArgs a, cons
     for (int n = 0; n < 2; ++n)
 #pragma unroll
       for (int e = 0; e < 4; ++e) s[n][e] = (kbase + n * 8 + 2 * tq + (e & 1) < k1) ? s[n][e] * sl2 : -INFINITY;
+    // online softmax with a lazy reference max: O and l are rescaled only when the running max
+    // grows by more than 2^8 (exact: p, l and O share the reference), which removes the
+    // per-page O rescale from the HBM-bound inner loop
     float corr[2];
+    bool rescale = false;
 #pragma unroll
     for (int hr = 0; hr < 2; ++hr) {
       float mx = fmaxf(fmaxf(s[0][2 * hr], s[0][2 * hr + 1]), fmaxf(s[1][2 * hr], s[1][2 * hr + 1]));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 1));
       mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, 2));
-      const float mn = fmaxf(mrow[hr], mx);
-      corr[hr] = exp2f(mrow[hr] - mn);
-      mrow[hr] = mn;
+      corr[hr] = 1.f;
+      if (mx > mrow[hr] + 8.f) {
+        corr[hr] = exp2f(mrow[hr] - mx);
+        mrow[hr] = mx;
+        lrow[hr] *= corr[hr];
+        rescale = true;
+      }
+      const float mn = mrow[hr];
       float sum = 0.f;
 #pragma unroll
       for (int n = 0; n < 2; ++n) {
@@ -138,7 +152,16 @@ __global__ void __launch_bounds__(128) decode_attn_kernel(const AttnArgs a, cons
         s[n][2 * hr + 1] = exp2f(s[n][2 * hr + 1] - mn);
         sum += s[n][2 * hr] + s[n][2 * hr + 1];
       }
-      lrow[hr] = lrow[hr] * corr[hr] + sum;
+      lrow[hr] += sum;
+    }
+    if (rescale) {
+#pragma unroll
+      for (int n = 0; n < D / 8; ++n) {
+        o[n][0] *= corr[0];
+        o[n][1] *= corr[0];
+        o[n][2] *= corr[1];
+        o[n][3] *= corr[1];
+      }
     }
     uint32_t pa[4];
     pa[0] = ptx::pack_bf16(s[0][0], s[0][1]);
@@ -147,14 +170,6 @@ __global__ void __launch_bounds__(128) decode_attn_kernel(const AttnArgs a, cons
     pa[3] = ptx::pack_bf16(s[1][2], s[1][3]);
 #pragma unroll
     for (int dp = 0; dp < D / 16; ++dp) {
-      o[2 * dp][0] *= corr[0];
-      o[2 * dp][1] *= corr[0];
-      o[2 * dp][2] *= corr[1];
-      o[2 * dp][3] *= corr[1];
-      o[2 * dp + 1][0] *= corr[0];
-      o[2 * dp + 1][1] *= corr[0];
-      o[2 * dp + 1][2] *= corr[1];
-      o[2 * dp + 1][3] *= corr[1];
       uint32_t b0, b1, b2, b3;
       ptx::ldsm_x4_t(vst + swz<D>((lane & 7) + (((lane >> 3) & 1) << 3), dp * 2 + (lane >> 4)), b0, b1, b2, b3);
       ptx::mma_bf16_16816(o[2 * dp], pa, b0, b1);

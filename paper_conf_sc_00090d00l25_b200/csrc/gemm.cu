@@ -39,7 +39,11 @@ struct Cfg {
   static constexpr int A_BYTES = GEMM_BM * GEMM_BK * 2;
   static constexpr int B_BYTES = B_ROWS * GEMM_BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+#ifdef GLLM_VARIANT_LOWSMEM  // measurement build: leave room for a co-resident attention CTA
+  static constexpr int STAGES = CG == 2 ? 4 : 3;
+#else
   static constexpr int STAGES = CG == 2 ? 6 : GEMM_STAGES;
+#endif
   static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
   static constexpr int TILE_M = GEMM_BM * CG;  // rows of one (cluster) tile
 };

@@ -1,6 +1,7 @@
 // Bandwidth-bound kernels of the stage forward: O4 weight init,
-// slot mapping (O2, a2), embedding gather (a3), RMSNorm (a4), fused RoPE +
-// paged KV append (a6) and the greedy argmax reduction (a11).
+// slot mapping + RoPE table (O2, a2), embedding gather (a3), RMSNorm statistics and
+// the final norm (a4) and the greedy argmax reduction (a11).  RoPE + KV append (a6)
+// live in the QKV GEMM epilogue.
 #include <cuda_bf16.h>
 
 #include "kernels.cuh"
@@ -158,43 +159,6 @@ __global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict_
   if (threadIdx.x == 0) ss[r] = acc;
 }
 
-// One CTA per token.  Work unit = one (head, i) rotation pair, i < D/2 (rotate-half convention):
-//   x'[i] = x[i] cos - x[i+D/2] sin ;  x'[i+D/2] = x[i+D/2] cos + x[i] sin
-__global__ void rope_kv_kernel(__nv_bfloat16* qkv, int Hq, int Hkv, int D, const float2* __restrict__ cs,
-                               const int32_t* __restrict__ slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int bs) {
-  const int t = blockIdx.x;
-  const int half = D / 2;
-  const int ld = (Hq + 2 * Hkv) * D;
-  __nv_bfloat16* row = qkv + (int64_t)t * ld;
-  const float2* c = cs + (int64_t)t * half;
-  const int slot = slots[t];
-  const int64_t blk = slot / bs, off = slot % bs;
-  const int nq = Hq * half, nk = Hkv * half;
-  for (int u = threadIdx.x; u < nq + nk; u += blockDim.x) {
-    const bool is_k = u >= nq;
-    const int uu = is_k ? u - nq : u;
-    const int h = uu / half, i = uu % half;
-    __nv_bfloat16* base = row + (is_k ? Hq * D : 0) + h * D;
-    const float x1 = __bfloat162float(base[i]), x2 = __bfloat162float(base[i + half]);
-    const float2 r = c[i];
-    const float y1 = x1 * r.x - x2 * r.y, y2 = x2 * r.x + x1 * r.y;
-    if (!is_k) {
-      base[i] = __float2bfloat16_rn(y1);
-      base[i + half] = __float2bfloat16_rn(y2);
-    } else {
-      __nv_bfloat16* dst = kc + ((blk * Hkv + h) * bs + off) * D;
-      dst[i] = __float2bfloat16_rn(y1);
-      dst[i + half] = __float2bfloat16_rn(y2);
-    }
-  }
-  const __nv_bfloat16* vrow = row + (Hq + Hkv) * D;
-  for (int u = threadIdx.x; u < Hkv * D / 8; u += blockDim.x) {
-    const int h = (u * 8) / D, d = (u * 8) % D;
-    *reinterpret_cast<uint4*>(vc + ((blk * Hkv + h) * bs + off) * D + d) =
-        *reinterpret_cast<const uint4*>(vrow + h * D + d);
-  }
-}
-
 __global__ void argmax_reduce_kernel(const float* __restrict__ pv, const int32_t* __restrict__ pi, int rows,
                                      int ntiles, int32_t* out) {
   const int r = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
@@ -261,12 +225,6 @@ void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int3
 void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s) {
   if (n <= 0) return;
   rms_stats_kernel<<<n, 256, 0, s>>>(x, xb, ss, H);
-}
-void launch_rope_kv_append(__nv_bfloat16* qkv, int T, int Hq, int Hkv, int D, const float2* rope_cs,
-                           const int32_t* slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int block_size,
-                           cudaStream_t s) {
-  if (T <= 0) return;
-  rope_kv_kernel<<<T, 256, 0, s>>>(qkv, Hq, Hkv, D, rope_cs, slots, kc, vc, block_size);
 }
 void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,
                           cudaStream_t s) {

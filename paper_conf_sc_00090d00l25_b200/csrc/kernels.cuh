@@ -31,11 +31,7 @@ void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int3
 // consumer GEMM scales its output rows by rsqrt(ss/H + eps).
 void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s);
 
-// RoPE on q (in place) and k of the fused qkv buffer, K/V appended to the paged cache at slots.
-// Cache layout per layer: [kv_blocks][Hkv][block_size][D] bf16 (K and V separately).
-void launch_rope_kv_append(__nv_bfloat16* qkv, int T, int Hq, int Hkv, int D, const float2* rope_cs,
-                           const int32_t* slots, __nv_bfloat16* kc, __nv_bfloat16* vc, int block_size,
-                           cudaStream_t s);
+// (RoPE + paged K/V append run in the QKV GEMM epilogue, gemm.cu EPI_QKV_ROPE.)
 
 // sampled[r] = argmax over n-tile partials (lowest id on ties, R18)
 void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,

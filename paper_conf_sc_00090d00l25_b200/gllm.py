@@ -14,7 +14,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgllm.so")
+LIB_PATH = os.environ.get("GLLM_LIB") or os.path.join(_HERE, "libgllm.so")  # GLLM_LIB: measurement builds
 
 GLLM_OK, GLLM_EMPTY = 0, 1
 ERRORS = {-1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ESTATE"}

@@ -133,9 +133,20 @@ def _bench_flow_worker(rank, world, port, q):
         pipe.run_batch(a, h)
     pipe.pending_samples.clear()
     pipe._expect.clear()
-    for _ in range(6):
-        pipe.tick()
+    # e2e leg: a fresh scheduler fast-forwarded to the value window replays the same ticks
+    if rank == 0:
+        sched = gllm.Sched(sp)
+        sched.add_stream(make_stream("C1", m.vocab, n=40))
+        for _ in range(int(batches[0]["tick"])):
+            sched.build_batch()
+        pipe.sched = sched
+    replay = [pipe.tick() for _ in range(5)]
     pipe.drain()
+    for a, b in zip(replay, batches):
+        assert int(a["tick"]) == int(b["tick"]) and int(a["num_tokens"]) == int(b["num_tokens"])
+        for key in ("token_ids", "positions", "cu_q", "kv_len", "slot_mapping", "block_table", "sample_idx"):
+            if key in a:
+                np.testing.assert_array_equal(np.asarray(a[key]), np.asarray(b[key]))
     dist.barrier()
     q.put(rank)
     dist.destroy_process_group()

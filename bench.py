@@ -133,6 +133,8 @@ def batch_work(m, a, n_layers, is_last):
         s = int(kvl[i]) - c
         pairs += c * s + c * (c + 1) // 2
     dec_keys = int(kvl[NP:].sum()) if kvl.shape[0] > NP else 0
+    pre_keys = int(kvl[:NP].sum())                    # each prefill chunk reads its context once
+    tp = int(cu[NP]) if NP else 0                     # prefill tokens
     nd = kvl.shape[0] - NP
     L = n_layers
 
@@ -143,10 +145,13 @@ def batch_work(m, a, n_layers, is_last):
         "o_gemm": gemm(T, H, qd, 8),            # fp32 residual read + write
         "gate_up_gemm": gemm(T, 2 * I, H, 1),   # bf16 SiLU*up output is half the columns
         "down_gemm": gemm(T, H, I, 8),
-        "prefill_attn": (4.0 * m.n_heads * m.head_dim * pairs * L, float(T * qd * 4 * L)),
+        "prefill_attn": (4.0 * m.n_heads * m.head_dim * pairs * L, float((pre_keys * kvb + tp * qd * 2 * 2) * L)),
         "decode_attn": (4.0 * m.n_heads * m.head_dim * dec_keys * L, float((dec_keys * kvb + nd * qd * 2 * 2) * L)),
         "rope_kv_append": (0.0, float(T * ((qd + 2 * kd) * 2 + qd * 2 + kvb) * L)),
-        "rmsnorm": (0.0, float(2 * T * H * (4 + 2) * L)),
+        # fused RMSNorm: one statistics pass at stage entry (x fp32 in, bf16 x + fp32 sum of squares
+        # out); the per-layer norms are GEMM epilogues.  Unfused (A/B): 2 passes per layer.
+        "rmsnorm": ((0.0, float(T * H * (4 + 2) + T * 4)) if os.environ.get("GLLM_UNFUSED_NORM", "0") != "1"
+                    else (0.0, float(2 * T * H * (4 + 2) * L))),
     }
     if is_last:
         w["lm_head"] = (2.0 * ns * H * V, float(V * H * 2 + ns * H * 2))

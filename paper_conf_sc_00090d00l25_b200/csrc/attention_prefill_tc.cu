@@ -1,4 +1,5 @@
 // Prefill (chunked, causal, paged) attention on 5th-gen tensor cores -- part of a7.
+// (The header below describes v1; v2 -- the default -- pipelines it, see prefill_attn_tc_kernel.)
 //
 // CTA = 128 flattened (token, group-head) query rows of one chunk x one kv head (the G query
 // heads sharing a kv head reuse every K/V tile); 4 warps, thread t owns row t = TMEM lane t.
@@ -13,6 +14,8 @@
 // one thread issues the MMAs and commits them to mbarriers; the next tile's K/V loads overlap
 // the current tile.  Final: O / l -> bf16 rows of the attention output.
 #include <cuda_bf16.h>
+
+#include <cstdlib>
 
 #include "attention.cuh"
 #include "common.h"
@@ -91,9 +94,10 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
+// v1 (kept for A/B, GLLM_PREFILL_V1=1): S_j, softmax_j and PV_j strictly in series per CTA.
 template <int D>
 __global__ void __launch_bounds__(128, 2)
-    prefill_attn_tc_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
+    prefill_attn_tc_v1_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
   using L = TcSmem<D>;
   constexpr int NCH = D / 8;  // 16-byte chunks per K/V/Q row
   extern __shared__ uint8_t smem_raw[];
@@ -270,14 +274,228 @@ __global__ void __launch_bounds__(128, 2)
   }
 }
 
+// v2: software-pipelined.  TMEM: two S buffers [0, 64) and [64, 128) (P_j overwrites S_j in place
+// once the row is in registers), O at [128, 128 + D).  Per key tile j the issuing thread queues
+// S_{j+1} = Q K_{j+1}^T BEFORE the softmax of S_j starts, so the tensor core computes the next
+// scores while the 128 threads run the softmax; tcgen05.mma executes in issue order, which makes
+// the overwrite of P_{j-1} by S_{j+1} safe behind PV_{j-1}.  K_{j+2} is fetched as soon as S_j
+// is done and V_{j+1} once PV_{j-1} is done, each as its own cp.async group (two K and two V
+// buffers; SMEM as v1).
+template <int D>
+__global__ void __launch_bounds__(128, 2)
+    prefill_attn_tc_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
+  using L = TcSmem<D>;
+  constexpr int NCH = D / 8;  // 16-byte chunks per K/V/Q row
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const uint32_t sbase = ptx::smem_u32(smem);
+  uint64_t* bar_s = reinterpret_cast<uint64_t*>(smem + L::BAR);  // [2]: S buffer b complete
+  uint64_t* bar_pv = bar_s + 2;
+  uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(bar_s + 3);
+
+  const PrefillItem it = items[blockIdx.x];
+  const int kvh = blockIdx.y;
+  const int G = a.Hq / a.Hkv;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int t0 = a.cu_q[it.seq];
+  const int c = a.cu_q[it.seq + 1] - t0;
+  const int s0 = a.kv_len[it.seq] - c;
+  const int nrows = c * G;
+  const int max_pos = s0 + min(it.row0 + TC_ROWS - 1, nrows - 1) / G;
+  const int n_kt = (max_pos + TC_KT) / TC_KT;
+  const int nblk_seq = (a.kv_len[it.seq] + 15) / 16;
+  const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
+  const float sl2 = LOG2E_T * rsqrtf((float)D);
+
+  if (tid == 0) {
+    ptx::mbar_init(&bar_s[0], 1);
+    ptx::mbar_init(&bar_s[1], 1);
+    ptx::mbar_init(bar_pv, 1);
+    ptx::fence_barrier_init();
+  }
+  if (warp == 0) ptx::tmem_alloc(tmem_ptr, 256);
+  if (warp == 0) ptx::tmem_relinquish();
+
+  for (int idx = tid; idx < TC_ROWS * NCH; idx += 128) {
+    const int r = idx / NCH, ch = idx % NCH;
+    const int rr = min(it.row0 + r, nrows - 1);
+    const int tok = rr / G, h = kvh * G + rr % G;
+    ptx::cp_async16(sbase + L::Q + sw128(TC_ROWS, r, ch),
+                    a.q + (size_t)(t0 + tok) * a.q_stride + (size_t)h * D + ch * 8, true);
+  }
+  // one 64-key tile of K (or V) of the paged cache into buffer `buf`
+  auto load_tile = [&](const __nv_bfloat16* cache, int kt, uint32_t dst) {
+    for (int idx = tid; idx < TC_KT * NCH; idx += 128) {
+      const int r = idx / NCH, ch = idx % NCH;
+      const int key = kt * TC_KT + r;
+      const int blk = key >> 4;
+      const bool ok = blk < nblk_seq;
+      const size_t page = ok ? (size_t)bt[blk] : 0;
+      ptx::cp_async16(dst + sw128(TC_KT, r, ch), cache + ((page * a.Hkv + kvh) * 16 + (key & 15)) * D + ch * 8, ok);
+    }
+  };
+  auto kbuf = [&](int b) { return sbase + (b ? L::K1 : L::K0); };
+  auto vbuf = [&](int b) { return sbase + (b ? L::V1 : L::V0); };
+  // cp.async groups, in commit order: {Q, K_0, K_1}, {V_0}, then per tile j: {K_{j+2}}, {V_{j+1}}
+  load_tile(a.kc, 0, kbuf(0));
+  if (n_kt > 1) load_tile(a.kc, 1, kbuf(1));
+  ptx::cp_async_commit();
+  load_tile(a.vc, 0, vbuf(0));
+  ptx::cp_async_commit();
+
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_ptr;
+  const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+  const uint32_t t_o = tmem + lane_off + 128;
+  constexpr uint32_t idesc_s = idesc_bf16(TC_ROWS, TC_KT, false);
+  constexpr uint32_t idesc_o = idesc_bf16(TC_ROWS, D, true);
+  auto issue_s = [&](int j) {  // thread 0: S_j -> S buffer j & 1
+    ptx::tc_fence_after();
+    const uint32_t kb = kbuf(j & 1);
+#pragma unroll
+    for (int ks = 0; ks < D / 16; ++ks)
+      ptx::umma_bf16(tmem + (j & 1) * TC_KT, desc_k(sbase + L::Q + (ks / 4) * L::Q_ATOM + (ks % 4) * 32),
+                     desc_k(kb + (ks / 4) * L::KV_ATOM + (ks % 4) * 32), idesc_s, ks > 0);
+    ptx::umma_commit(&bar_s[j & 1]);
+  };
+  ptx::cp_async_wait<1>();  // Q, K_0, K_1
+  fence_proxy_async_smem();
+  __syncthreads();
+  if (tid == 0) issue_s(0);
+
+  const int rr = it.row0 + tid;
+  const int rrc = min(rr, nrows - 1);
+  const int pos = s0 + rrc / G;  // this row's causal limit (keys 0..pos)
+  float m_ref = -INFINITY, l = 0.f;
+
+  for (int j = 0; j < n_kt; ++j) {
+    const int b = j & 1;
+    // A: queue S_{j+1} behind PV_{j-1} (K_{j+1} is the older of the two newest groups)
+    if (j + 1 < n_kt) {
+      ptx::cp_async_wait<1>();
+      fence_proxy_async_smem();
+      __syncthreads();
+      if (tid == 0) issue_s(j + 1);
+    }
+    // B: S_j -> registers; its K buffer is free for K_{j+2}
+    ptx::mbar_wait(&bar_s[b], (j >> 1) & 1);
+    ptx::tc_fence_after();
+    uint32_t sr[2][32];
+    const uint32_t t_s = tmem + lane_off + b * TC_KT;
+    ptx::tmem_ld_32x32b_x32(t_s, sr[0]);
+    ptx::tmem_ld_32x32b_x32(t_s + 32, sr[1]);
+    ptx::tmem_ld_wait();
+    if (j + 2 < n_kt) load_tile(a.kc, j + 2, kbuf(b));
+    ptx::cp_async_commit();
+    // C: online softmax (lazy rescale, see v1), P_j over S_j
+    float s[64];
+    float mx = -INFINITY;
+#pragma unroll
+    for (int i = 0; i < 64; ++i) {
+      const int key = j * TC_KT + i;
+      s[i] = key <= pos ? __uint_as_float(sr[i >> 5][i & 31]) * sl2 : -INFINITY;
+      mx = fmaxf(mx, s[i]);
+    }
+    const bool mine = mx > m_ref + RESCALE_LOG2;
+    const float corr = mine ? exp2f(m_ref - mx) : 1.f;
+    if (mine) {
+      l *= corr;
+      m_ref = mx;
+    }
+    if (j > 0 && __any_sync(0xffffffffu, mine)) {
+      ptx::mbar_wait(bar_pv, (j - 1) & 1);  // O final for tiles < j
+      ptx::tc_fence_after();
+#pragma unroll
+      for (int cb = 0; cb < D / 32; ++cb) {
+        uint32_t orr[32];
+        ptx::tmem_ld_32x32b_x32(t_o + cb * 32, orr);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int i = 0; i < 32; ++i) orr[i] = __float_as_uint(__uint_as_float(orr[i]) * corr);
+        tmem_st_32x32b_x32(t_o + cb * 32, orr);
+      }
+    }
+    {
+      uint32_t pw[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const float p0 = exp2f(s[2 * i] - m_ref), p1 = exp2f(s[2 * i + 1] - m_ref);
+        l += p0 + p1;
+        pw[i] = ptx::pack_bf16(p0, p1);
+      }
+      tmem_st_32x32b_x32(t_s, pw);
+      tmem_st_wait();
+    }
+    // D: PV_{j-1} done -> its V buffer takes V_{j+1}
+    if (j > 0) ptx::mbar_wait(bar_pv, (j - 1) & 1);
+    if (j + 1 < n_kt) load_tile(a.vc, j + 1, vbuf(b ^ 1));
+    ptx::cp_async_commit();
+    // E: O += P_j V_j (V_j is the oldest of the three newest groups)
+    ptx::cp_async_wait<2>();
+    fence_proxy_async_smem();
+    ptx::tc_fence_before();
+    __syncthreads();
+    if (tid == 0) {
+      ptx::tc_fence_after();
+      const uint32_t vb = vbuf(b);
+#pragma unroll
+      for (int kk = 0; kk < TC_KT / 16; ++kk)
+        umma_bf16_ta(tmem + 128, tmem + b * TC_KT + kk * 8, desc_mn(vb + kk * 2048, L::KV_ATOM), idesc_o,
+                     (j > 0 || kk > 0) ? 1u : 0u);
+      ptx::umma_commit(bar_pv);
+    }
+  }
+  ptx::mbar_wait(bar_pv, (n_kt - 1) & 1);
+  ptx::tc_fence_after();
+  const bool valid = rr < nrows;
+  const float inv = 1.f / l;
+  __nv_bfloat16* dst = a.out + (size_t)(t0 + rrc / G) * a.Hq * D + (size_t)(kvh * G + rrc % G) * D;
+#pragma unroll
+  for (int cb = 0; cb < D / 32; ++cb) {
+    uint32_t orr[32];
+    ptx::tmem_ld_32x32b_x32(t_o + cb * 32, orr);
+    ptx::tmem_ld_wait();
+    if (valid) {
+      uint4* d4 = reinterpret_cast<uint4*>(dst + cb * 32);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 w;
+        w.x = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 0]) * inv, __uint_as_float(orr[q * 8 + 1]) * inv);
+        w.y = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 2]) * inv, __uint_as_float(orr[q * 8 + 3]) * inv);
+        w.z = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 4]) * inv, __uint_as_float(orr[q * 8 + 5]) * inv);
+        w.w = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 6]) * inv, __uint_as_float(orr[q * 8 + 7]) * inv);
+        d4[q] = w;
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, 256);
+  }
+}
+
+const bool g_prefill_v1 = [] {
+  const char* e = std::getenv("GLLM_PREFILL_V1");
+  return e && e[0] == '1';
+}();
+
 template <int D>
 int launch_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
   static bool set = false;
   if (!set) {
     cudaFuncSetAttribute(prefill_attn_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, TcSmem<D>::BYTES);
+    cudaFuncSetAttribute(prefill_attn_tc_v1_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         TcSmem<D>::BYTES);
     set = true;
   }
-  prefill_attn_tc_kernel<D><<<dim3(n_items, a.Hkv), 128, TcSmem<D>::BYTES, s>>>(a, items);
+  if (g_prefill_v1)
+    prefill_attn_tc_v1_kernel<D><<<dim3(n_items, a.Hkv), 128, TcSmem<D>::BYTES, s>>>(a, items);
+  else
+    prefill_attn_tc_kernel<D><<<dim3(n_items, a.Hkv), 128, TcSmem<D>::BYTES, s>>>(a, items);
   return GLLM_OK;
 }
 

@@ -125,6 +125,7 @@ struct gllm_stage {
   float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
   bool fused_norm = true;
   bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
+  bool attn_overlap = true;                // GLLM_ATTN_SERIAL=1: prefill and decode attention in series (A/B)
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
@@ -393,6 +394,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
   if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
   if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
+  if (const char* e = std::getenv("GLLM_ATTN_SERIAL")) st->attn_overlap = e[0] != '1';
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
@@ -676,7 +678,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     aa.vc = w.vc;
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
-    const bool overlap = P.n_pi > 0 && P.n_di > 0;
+    const bool overlap = st->attn_overlap && P.n_pi > 0 && P.n_di > 0;
     if (P.n_pi > 0) {
       cudaStream_t ps = overlap ? st->side : s;
       if (overlap) {

@@ -58,7 +58,7 @@ def main():
     x = torch.randn((sp.maxp + sp.max_seqs + 64, m.hidden), device="cuda")
     out = {}
     kvb = 2 * m.n_kv_heads * m.head_dim * 2
-    for name, seqs in (("decode", list(range(NP, S))), ("prefill", list(range(NP)))):
+    for name, seqs in (("decode", list(range(NP, S))), ("prefill", list(range(NP))), ("mixed", list(range(S)))):
         if not seqs:
             continue
         d, keep = gllm.desc_from_arrays(subset(full, seqs))
@@ -71,6 +71,12 @@ def main():
             st.forward(d, x.data_ptr(), x.data_ptr(), 0, 0)
         tm = st.last_timing()
         st.set_profiling(False)
+        if name == "mixed":
+            # the whole batch's attention phase (prefill || decode): stage span minus the other kernels
+            span = tm["total"] - sum(v for k, v in tm.items() if k != "total" and not k.endswith("_attn"))
+            out[name] = {"us": round(span / a.reps * 1e3, 1),
+                         "serial_us": round((out.get("decode", {}).get("us", 0) + out.get("prefill", {}).get("us", 0)), 1)}
+            continue
         ms = tm[name + "_attn"] / a.reps
         kvl, cu = keep["kv_len"], keep["cu_q"]
         if name == "decode":

@@ -1,5 +1,5 @@
 // Prefill (chunked, causal, paged) attention on 5th-gen tensor cores -- part of a7.
-// (The header below describes v1; v2 -- the default -- pipelines it, see prefill_attn_tc_kernel.)
+// (The header below describes v1, the default; v2 (GLLM_PREFILL_V2=1) pipelines it, see prefill_attn_tc_kernel.)
 //
 // CTA = 128 flattened (token, group-head) query rows of one chunk x one kv head (the G query
 // heads sharing a kv head reuse every K/V tile); 4 warps, thread t owns row t = TMEM lane t.
@@ -94,7 +94,7 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
-// v1 (kept for A/B, GLLM_PREFILL_V1=1): S_j, softmax_j and PV_j strictly in series per CTA.
+// v1 (default): S_j, softmax_j and PV_j in series per CTA; two CTAs per SM overlap each other.
 template <int D>
 __global__ void __launch_bounds__(128, 2)
     prefill_attn_tc_v1_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
@@ -478,9 +478,11 @@ __global__ void __launch_bounds__(128, 2)
   }
 }
 
+// v1 is the default: measured on B200 (tools/ab.sh, profiles/r01/ab_prefill.txt) the pipelined v2
+// is 10-20% slower -- two co-resident CTAs per SM already interleave softmax and MMA phases.
 const bool g_prefill_v1 = [] {
-  const char* e = std::getenv("GLLM_PREFILL_V1");
-  return e && e[0] == '1';
+  const char* e = std::getenv("GLLM_PREFILL_V2");
+  return !(e && e[0] == '1');
 }();
 
 template <int D>

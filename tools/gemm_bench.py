@@ -17,7 +17,30 @@ SHAPES = {
     "C1": [(2094, 6144, 4096, 0), (2094, 4096, 4096, 1), (2094, 28672, 4096, 2), (2094, 4096, 14336, 1)],
     "C4": [(128, 10240, 8192, 0), (128, 8192, 8192, 1), (128, 57344, 8192, 2), (128, 8192, 28672, 1)],
     "sq": [(8192, 8192, 8192, 0)],
+    # the C1 O / down shapes with the plain bf16-store epilogue (isolates the residual epilogue)
+    "C1s": [(2094, 4096, 4096, 0), (2094, 4096, 14336, 0)],
 }
+
+
+def bench_cublas(M, N, K, reps=20):
+    """cuBLAS (torch.mm, bf16 out) on the same shape: the library reference for the plain GEMM."""
+    A = torch.randn((M, K), device="cuda").to(torch.bfloat16)
+    W = (torch.randn((N, K), device="cuda") * K ** -0.5).to(torch.bfloat16)
+    flush = torch.empty(256 << 20, dtype=torch.int8, device="cuda")
+    for _ in range(3):
+        torch.mm(A, W.t())
+    ts = []
+    for _ in range(reps):
+        flush.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        torch.mm(A, W.t())
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    ts.sort()
+    ms = ts[len(ts) // 2]
+    return dict(M=M, N=N, K=K, epi="cublas", us=round(ms * 1e3, 1), tflops=round(2.0 * M * N * K / (ms * 1e-3) / 1e12, 1))
 
 
 def bench(M, N, K, epi, reps=20):
@@ -53,7 +76,12 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--shapes", default="C1,C4,sq")
     ap.add_argument("--variants", default="0", help="comma list: 0 auto, 1 one-CTA, 2 CTA pair")
+    ap.add_argument("--cublas", action="store_true", help="also time torch.mm (cuBLAS) per shape")
     a = ap.parse_args()
+    if a.cublas:
+        for key in a.shapes.split(","):
+            for shp in SHAPES[key]:
+                print(json.dumps({"variant": "cublas", "set": key, **bench_cublas(*shp[:3])}), flush=True)
     for v in [int(x) for x in a.variants.split(",")]:
         gllm.op_set_gemm_variant(v)
         for key in a.shapes.split(","):

@@ -37,6 +37,9 @@ from workloads.streams import make_stream  # noqa: E402
 METRIC = "mixed-batch tokens/s at PP=1/2/4/8 B200; bubble fraction; stage roofline %"
 UNIT = "tokens/s"
 FALLBACK_PEAKS = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+# The driver's MEASURED_PEAKS.json of this round's pool, as copied into BASELINE.md §2 (the file
+# itself is git-ignored and driver-written; a re-created container may not have it).
+RECORDED_PEAKS = {"hbm_gbs": 6546.6, "bf16_tflops": 1626.2, "bf16_tflops_sustained": 1344.0}
 
 
 def peaks():
@@ -44,6 +47,8 @@ def peaks():
     if os.path.exists(p):
         d = json.load(open(p))
         return d, "measured"
+    if os.path.exists(os.path.join(ROOT, "BASELINE.md")):
+        return RECORDED_PEAKS, "measured (MEASURED_PEAKS.json as recorded in BASELINE.md §2)"
     return FALLBACK_PEAKS, "fallback"
 
 
@@ -165,7 +170,7 @@ def roofline_report(timing_ms, work, launches, pk):
     pi = float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"])) * 1e12
     beta = float(pk["hbm_gbs"]) * 1e9
     for name, ms in timing_ms.items():
-        if name in ("total", "other") or name not in work or ms <= 0:
+        if name in ("total", "other", "attention_span") or name not in work or ms <= 0:
             continue
         flops, nbytes = work[name]
         sec = ms * 1e-3
@@ -178,6 +183,31 @@ def roofline_report(timing_ms, work, launches, pk):
                       "share": round(ms / max(timing_ms.get("total", ms), 1e-9), 4)}
     dom = max(kern, key=lambda k: kern[k]["ms"]) if kern else None
     return dom, kern
+
+
+def stage_roofline(timing_ms, work, pk):
+    """Per-stage roofline %: sum over the step's kernels of max(FLOPs/Pi, bytes/beta)
+    divided by the measured stage time.  Prefill and decode attention run concurrently (tensor
+    pipe vs HBM): their joint bound is max(prefill FLOPs/Pi, (prefill + decode bytes)/beta)."""
+    pi = float(pk.get("bf16_tflops_sustained", pk["bf16_tflops"])) * 1e12
+    beta = float(pk["hbm_gbs"]) * 1e9
+    t = 0.0
+    w = dict(work)
+    if "rope_kv_append" in w:  # fused into the QKV GEMM epilogue: one kernel, bytes add up
+        rf, rb = w.pop("rope_kv_append")
+        qf, qb = w.get("qkv_gemm", (0.0, 0.0))
+        w["qkv_gemm"] = (qf + rf, qb + rb)
+    for name, (fl, by) in w.items():
+        if name in ("prefill_attn", "decode_attn"):
+            continue
+        t += max(fl / pi, by / beta)
+    pf, pb = work.get("prefill_attn", (0.0, 0.0))
+    df, db = work.get("decode_attn", (0.0, 0.0))
+    t += max((pf + df) / pi, (pb + db) / beta)
+    total = timing_ms.get("total", 0.0) * 1e-3
+    return {"roofline_ms": round(t * 1e3, 3), "measured_ms": round(total * 1e3, 3),
+            "frac": round(t / total, 4) if total > 0 else None,
+            "attention_span_ms": round(timing_ms.get("attention_span", 0.0), 3)}
 
 
 # ---------------------------------------------------------------------------- our arm
@@ -302,6 +332,7 @@ def run_ours(args):
             work[kname] = (f0 + fl, b0 + by)
     pk, pk_src = peaks()
     dom, kern = roofline_report(timing, work, launches, pk)
+    stage_rl = stage_roofline(timing, work, pk)
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if dom and os.path.exists(tp):
@@ -368,6 +399,7 @@ def run_ours(args):
                           "traffic": traffic, "peak_source": pk_src + (" sustained" if kern[dom]["bound"] == "tensor" else "")}
                          if dom else None),
             "kernels": kern,
+            "stage_roofline": stage_rl,
             "bubble_fraction": {"per_stage": [round(b, 4) for b in bubbles], "max": round(max(bubbles), 4),
                                 "mean": round(float(np.mean(bubbles)), 4)},
             "cpu_baseline": cpu,

@@ -46,7 +46,7 @@ enum Kind { K_WQ = 0, K_WK, K_WV, K_WO, K_WG, K_WU, K_WD, K_BQ, K_BK, K_BV };
 inline uint64_t layer_tid(int l, int kind) { return 1 + 16 * (uint64_t)l + kind; }
 
 // profiling categories (gllm_stage_last_timing)
-enum Cat { C_TOTAL = 0, C_QKV, C_O, C_GU, C_DOWN, C_PREFILL, C_DECODE, C_ROPE, C_NORM, C_LMHEAD, C_OTHER, C_N };
+enum Cat { C_TOTAL = 0, C_QKV, C_O, C_GU, C_DOWN, C_PREFILL, C_DECODE, C_ROPE, C_NORM, C_LMHEAD, C_OTHER, C_ATTN, C_N };
 
 struct LayerW {
   bf16 *wqkv = nullptr, *wo = nullptr, *wgu = nullptr, *wd = nullptr;
@@ -184,7 +184,10 @@ struct Prof {
       cudaEventRecord(a, s);
     }
   }
-  ~Prof() {
+  bool closed = false;
+  void close() {
+    if (closed) return;
+    closed = true;
     if (st->profiling) {
       cudaEvent_t b = st->next_ev();
       cudaEventRecord(b, s);
@@ -195,6 +198,7 @@ struct Prof {
       std::fprintf(stderr, "[gllm] cat %d done: %s\n", cat, cudaGetErrorString(e));
     }
   }
+  ~Prof() { close(); }
   static bool g_sync_debug;
 };
 bool Prof::g_sync_debug = std::getenv("GLLM_SYNC_DEBUG") != nullptr;
@@ -679,6 +683,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
     const bool overlap = st->attn_overlap && P.n_pi > 0 && P.n_di > 0;
+    Prof p_attn(st, s, C_ATTN);  // span of the attention step (prefill || decode), on the main stream
     if (P.n_pi > 0) {
       cudaStream_t ps = overlap ? st->side : s;
       if (overlap) {
@@ -694,15 +699,18 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       st->last_launches += 1;
     }
     if (overlap) {
-      Prof p(st, s, C_DECODE);
-      RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
-      st->last_launches += P.n_mi ? 2 : 1;
+      {
+        Prof p(st, s, C_DECODE);  // the decode kernels alone (the join wait is outside)
+        RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
+        st->last_launches += P.n_mi ? 2 : 1;
+      }
       CK(cudaStreamWaitEvent(s, st->ev_join, 0));
     } else if (P.n_di > 0) {
       Prof p(st, s, C_DECODE);
       RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
       st->last_launches += P.n_mi ? 2 : 1;
     }
+    p_attn.close();
     {
       Prof p(st, s, C_O);
       RC(residual_gemm(st->tm_attn, w.tm_o, qd, st->ss_b));

@@ -20,7 +20,7 @@ GLLM_OK, GLLM_EMPTY = 0, 1
 ERRORS = {-1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ESTATE"}
 
 TIMING_NAMES = ["total", "qkv_gemm", "o_gemm", "gate_up_gemm", "down_gemm", "prefill_attn", "decode_attn",
-                "rope_kv_append", "rmsnorm", "lm_head", "other"]
+                "rope_kv_append", "rmsnorm", "lm_head", "other", "attention_span"]
 
 
 class GllmError(RuntimeError):

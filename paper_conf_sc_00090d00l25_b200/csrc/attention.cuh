@@ -1,5 +1,6 @@
 // Varlen paged causal attention over one mixed batch (a7 of DESIGN.md §2) -- internal interface.
 #pragma once
+#include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -42,5 +43,13 @@ int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_
 int launch_prefill_attention_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
 int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
                             int n_merges, cudaStream_t s);
+// persistent warp-worker decode kernel fed by TMA (attention_decode.cu), the default; `tmk` /
+// `tmv` map the layer's K / V cache as [kv_blocks*Hkv*16, D] bf16 with 16 x 64 SW128 boxes;
+// `ctr` = 2 device ints, zero before the first launch (the kernel leaves them zero)
+bool decode_tma_supported(int D, int G);
+void set_decode_warps(int warps);
+int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
+                                const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
+                                int num_sms, cudaStream_t s);
 
 }  // namespace gllm

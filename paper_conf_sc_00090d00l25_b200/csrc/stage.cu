@@ -53,6 +53,7 @@ struct LayerW {
   float* bqkv = nullptr;
   bf16 *kc = nullptr, *vc = nullptr;
   CUtensorMap tm_qkv, tm_o, tm_gu, tm_d;
+  CUtensorMap tm_kc, tm_vc;  // paged K / V cache as [kv_blocks*Hkv*16, D] (16 x 64 SW128 boxes)
 };
 
 constexpr int RING = 4;
@@ -126,6 +127,8 @@ struct gllm_stage {
   bool fused_norm = true;
   bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
   bool attn_overlap = true;                // GLLM_ATTN_SERIAL=1: prefill and decode attention in series (A/B)
+  bool decode_v1 = false;                  // GLLM_DECODE_V1=1: the per-CTA cp.async decode kernel (A/B)
+  int* dec_ctr = nullptr;                  // persistent decode kernel: work counter + done counter
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
@@ -364,7 +367,9 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_B_BOX)) ||
         (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_B_BOX)) ||
         (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)))
+        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_kc, w.kc, (uint64_t)kv_blocks * Hkv * block_size, D, 16)) ||
+        (rc = gllm::make_tmap_bf16(&w.tm_vc, w.vc, (uint64_t)kv_blocks * Hkv * block_size, D, 16)))
       return fail(rc);
     st->layers.push_back(w);
   }
@@ -392,13 +397,17 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = st->dalloc(&st->slots, R)) ||
       // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
       (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)) || (rc = st->dalloc(&st->ss_a, R)) ||
-      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)))
+      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)) || (rc = st->dalloc(&st->dec_ctr, 2)))
     return fail(rc);
+  CK(cudaMemsetAsync(st->dec_ctr, 0, 2 * sizeof(int), s0));
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
   gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
   if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
   if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
   if (const char* e = std::getenv("GLLM_ATTN_SERIAL")) st->attn_overlap = e[0] != '1';
+  if (const char* e = std::getenv("GLLM_DECODE_V1")) st->decode_v1 = e[0] == '1';
+  if (const char* e = std::getenv("GLLM_DECODE_WARPS")) gllm::set_decode_warps(std::atoi(e));
+  if (!gllm::decode_tma_supported(D, cfg->n_heads / Hkv) || block_size != 16) st->decode_v1 = true;
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
@@ -407,7 +416,10 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     return fail(rc);
   for (int i = 0; i < RING; ++i)
     if ((rc = new_slot(st)) < 0) return fail(rc);
-  if (cudaStreamCreateWithFlags(&st->side, cudaStreamNonBlocking) != cudaSuccess ||
+  int prio_lo = 0, prio_hi = 0;
+  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  const char* sp = std::getenv("GLLM_SIDE_PRIO");  // A/B: prefill attention stream at the highest priority
+  if (cudaStreamCreateWithPriority(&st->side, cudaStreamNonBlocking, (sp && sp[0] == '1') ? prio_hi : 0) != cudaSuccess ||
       cudaEventCreateWithFlags(&st->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&st->ev_join, cudaEventDisableTiming) != cudaSuccess)
     return fail(gllm::set_error(GLLM_ECUDA, "side stream / events"));
@@ -492,9 +504,11 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   if (ND > 0) {
     // split long contexts so that the decode grid has >= ~8 CTAs per SM of work; a split is
     // at least 32 pages (512 keys) so the merge pass stays negligible
-    const int64_t target = 8LL * st->num_sms;  // CTAs
+    // (persistent kernel: ~32 work units per SM for the dynamic longest-first schedule, a split
+    // is at least 16 pages)
+    const int64_t target = (st->decode_v1 ? 8LL : 32LL) * st->num_sms;  // work units
     int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
-    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(32, per));
+    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(st->decode_v1 ? 32 : 16, per));
   }
   std::vector<gllm::DecodeItem> ditems;
   std::vector<gllm::MergeItem> merges;
@@ -680,6 +694,12 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     }
     aa.kc = w.kc;
     aa.vc = w.vc;
+    auto decode = [&](cudaStream_t ds) -> int {
+      st->last_launches += P.n_mi ? 2 : 1;
+      if (st->decode_v1) return gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, ds);
+      return gllm::launch_decode_attention_tma(aa, w.tm_kc, w.tm_vc, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
+                                               st->num_sms, ds);
+    };
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
     const bool overlap = st->attn_overlap && P.n_pi > 0 && P.n_di > 0;
@@ -701,14 +721,12 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     if (overlap) {
       {
         Prof p(st, s, C_DECODE);  // the decode kernels alone (the join wait is outside)
-        RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
-        st->last_launches += P.n_mi ? 2 : 1;
+        RC(decode(s));
       }
       CK(cudaStreamWaitEvent(s, st->ev_join, 0));
     } else if (P.n_di > 0) {
       Prof p(st, s, C_DECODE);
-      RC(gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, s));
-      st->last_launches += P.n_mi ? 2 : 1;
+      RC(decode(s));
     }
     p_attn.close();
     {

@@ -72,8 +72,8 @@ def main():
         tm = st.last_timing()
         st.set_profiling(False)
         if name == "mixed":
-            # the whole batch's attention phase (prefill || decode): stage span minus the other kernels
-            span = tm["total"] - sum(v for k, v in tm.items() if k != "total" and not k.endswith("_attn"))
+            # the whole batch's attention phase (prefill || decode), timed on the main stream
+            span = tm["attention_span"]
             out[name] = {"us": round(span / a.reps * 1e3, 1),
                          "serial_us": round((out.get("decode", {}).get("us", 0) + out.get("prefill", {}).get("us", 0)), 1)}
             continue

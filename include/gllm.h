@@ -58,6 +58,9 @@ typedef struct {
 /* Scheduler: Token Throttling (L145-L183 §3.1-3.2) + paged-KV block manager */
 /* (L136 Fig.6).  Host-only, deterministic, single-threaded per object. */
 /* ------------------------------------------------------------------------ */
+/* build_batch policies (gllm_sched_cfg.policy) */
+enum { GLLM_POLICY_THROTTLE = 0, GLLM_POLICY_SARATHI = 1, GLLM_POLICY_NO_WT = 2, GLLM_POLICY_NO_UT = 3 };
+
 typedef struct {
   int32_t iterp;          /* #T  (Eq.1/Eq.3; default 8, L248) */
   int32_t maxp, minp;     /* #MaxP, #MinP (L151; 2048 / 32, L248) */
@@ -67,7 +70,11 @@ typedef struct {
   int32_t num_blocks;     /* N, KV blocks shared by all stages (L136) */
   int32_t block_size;     /* tokens per KV block (16) */
   int32_t max_seqs;       /* max running sequences (1024, L575) */
-  int32_t policy;         /* 0 = Token Throttling; 1 = Sarathi-Serve (decodes first, prefill to budget) */
+  int32_t policy;         /* GLLM_POLICY_*: 0 = Token Throttling (Eq.3 + threshold, Eq.4);
+                             1 = Sarathi-Serve (every ready decode, prefill to token_budget; "w/ CK", L310);
+                             2 = ablation "w/o WT" (Eq.3 without the #WP/#T term, L308);
+                             3 = ablation "w/o UT" (Eq.1 + the L165 threshold, L308).
+                             Policies 2-3 keep Eq.4 for decodes (§4.5, Fig. 15). */
   int32_t token_budget;   /* Sarathi only (2048, L248) */
 } gllm_sched_cfg;
 

@@ -36,11 +36,19 @@ import numpy as np
 
 
 def throttle_prefill(cfg, wp: int, free: int) -> int:
-    """#P by Eq.3 with the L165 threshold, exact integer reading R10."""
+    """#P by Eq.3 with the L165 threshold, exact integer reading R10.
+
+    Ablations of §4.5 (L305-L310, Fig. 15): policy 2 "w/o WT" drops the #WP/#T term of Eq.3
+    (R19); policy 3 "w/o UT" is Eq.1 (L153) with the L165 threshold kept (R20)."""
     n, num, den = cfg.num_blocks, cfg.kvthresh_num, cfg.kvthresh_den
     if wp == 0 or free * den < num * n:          # KV_free < KV_thresh: suspend prefill (L165)
         return 0
     cap = (cfg.maxp * (free * den - num * n)) // (n * (den - num))   # MaxP*(KVfree-th)/(1-th)
+    policy = getattr(cfg, "policy", 0)
+    if policy == 2:                              # w/o WT: max(MaxP*(KVfree-th)/(1-th), MinP)
+        return min(max(cap, cfg.minp), wp)
+    if policy == 3:                              # w/o UT: Eq.1 = min(max(WP/T, MinP), MaxP)
+        return min(max(wp // cfg.iterp, cfg.minp), cfg.maxp, wp)
     return min(max(min(wp // cfg.iterp, cap), cfg.minp), wp)         # Eq.3, capped by WP (R11)
 
 

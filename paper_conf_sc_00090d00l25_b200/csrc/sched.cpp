@@ -139,7 +139,13 @@ int32_t throttle_prefill(const gllm_sched_cfg& c, int64_t wp, int64_t free_block
   const int64_t n = c.num_blocks, num = c.kvthresh_num, den = c.kvthresh_den;
   if (wp == 0 || free_blocks * den < num * n) return 0;  // KV_free < KV_thresh: suspend (L165)
   int64_t cap = ((int64_t)c.maxp * (free_blocks * den - num * n)) / (n * (den - num));
-  int64_t p = std::min(wp / c.iterp, cap);               // Eq.3 inner min (WT vs UT)
+  int64_t p;
+  if (c.policy == GLLM_POLICY_NO_WT)
+    p = cap;                                             // R19: Eq.3 without the #WP/#T term
+  else if (c.policy == GLLM_POLICY_NO_UT)
+    p = std::min<int64_t>(wp / c.iterp, c.maxp);         // R20: Eq.1 (threshold kept)
+  else
+    p = std::min(wp / c.iterp, cap);                     // Eq.3 inner min (WT vs UT)
   p = std::max(p, (int64_t)c.minp);                      // Eq.3 outer max (#MinP)
   return (int32_t)std::min(p, wp);                       // R11: cannot exceed #WP
 }
@@ -155,7 +161,8 @@ int check_cfg(const gllm_sched_cfg* c) {
     return gllm::set_error(GLLM_EINVAL, "scheduler cfg: non-positive size");
   if (c->kvthresh_den < 1 || c->kvthresh_num < 0 || c->kvthresh_num >= c->kvthresh_den)
     return gllm::set_error(GLLM_EINVAL, "scheduler cfg: KV_thresh must be in [0,1)");
-  if (c->policy != 0 && c->policy != 1) return gllm::set_error(GLLM_EINVAL, "unknown policy");
+  if (c->policy < GLLM_POLICY_THROTTLE || c->policy > GLLM_POLICY_NO_UT)
+    return gllm::set_error(GLLM_EINVAL, "unknown policy %d", c->policy);
   return GLLM_OK;
 }
 
@@ -349,7 +356,7 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   auto& allocs = b.allocs;
   auto& preempted = b.preempted;
   // 4. decode selection (Eq.4; R6-R9; R14): the first min(#D, |ready|) of the ready FIFO
-  const int32_t d_cnt = cfg.policy == 1 ? (int32_t)rd : throttle_decode(cfg, rd);
+  const int32_t d_cnt = cfg.policy == GLLM_POLICY_SARATHI ? (int32_t)rd : throttle_decode(cfg, rd);
   const size_t n_try = std::min<size_t>((size_t)d_cnt, s->readyq.size());
   std::vector<Req*> cand(s->readyq.begin(), s->readyq.begin() + n_try);
   s->readyq.erase(s->readyq.begin(), s->readyq.begin() + n_try);
@@ -381,7 +388,7 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   for (auto i = skipped.rbegin(); i != skipped.rend(); ++i) s->readyq.push_front(*i);
   // 5. prefill count (Eq.3 + L165; R10-R12)
   int32_t p_cnt;
-  if (cfg.policy == 1)
+  if (cfg.policy == GLLM_POLICY_SARATHI)
     p_cnt = (int32_t)std::min<int64_t>(std::max<int64_t>(cfg.token_budget - (int64_t)b.decodes.size(), 0), wp);
   else
     p_cnt = throttle_prefill(cfg, wp, free0);

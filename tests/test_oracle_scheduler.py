@@ -65,6 +65,46 @@ def test_eq1_eq2_special_cases():
         assert throttle_prefill(cfg, 10 ** 9, free) == (eq2 if free > 0 else 32)
 
 
+NO_WT, NO_UT = DEF.with_(policy=2), DEF.with_(policy=3)
+
+
+@pytest.mark.parametrize("cfg,wp,free,expect", [
+    # "w/o WT" (R19): max(MaxP*(KV_free-th)/(1-th), MinP), capped by WP
+    (NO_WT, 10000, 1000, 2048),   # KV fully free -> MaxP (WP/T = 1250 no longer caps it)
+    (NO_WT, 10000, 500, 970),     # floor(2048*9000/19000)
+    (NO_WT, 100, 1000, 100),      # capped by WP (R11)
+    (NO_WT, 10000, 49, 0),        # threshold kept (L165)
+    (NO_WT, 10000, 50, 32),       # cap 0 -> MinP
+    # "w/o UT" (R20): Eq.1 = min(max(WP/T, MinP), MaxP) with the L165 threshold
+    (NO_UT, 10000, 500, 1250),    # KV pressure ignored: WP/T
+    (NO_UT, 20000, 60, 2048),     # MaxP even with 6% free
+    (NO_UT, 100, 1000, 32),       # MinP
+    (NO_UT, 20, 1000, 20),        # capped by WP
+    (NO_UT, 10000, 49, 0),        # threshold kept
+])
+def test_ablation_examples(cfg, wp, free, expect):
+    assert throttle_prefill(cfg, wp, free) == expect
+
+
+def test_ablations_match_eq1_eq2_exact_rationals():
+    # policy 2 is floor(Eq.2 rescaled over the threshold), policy 3 is floor(Eq.1) (L153, L161),
+    # both behind the L165 threshold and capped by #WP (R11), in exact rationals
+    from fractions import Fraction as F
+    rng = np.random.default_rng(1)
+    for _ in range(2000):
+        n = int(rng.integers(1, 5000))
+        base = SchedParams(iterp=int(rng.integers(1, 17)), maxp=int(rng.integers(1, 4096)),
+                           minp=int(rng.integers(0, 64)), kvthresh_num=int(rng.integers(0, 5)),
+                           kvthresh_den=int(rng.integers(5, 40)), num_blocks=n)
+        wp, free = int(rng.integers(0, 50000)), int(rng.integers(0, n + 1))
+        kvf, th = F(free, n), F(base.kvthresh_num, base.kvthresh_den)
+        off = wp == 0 or kvf < th
+        eq2 = max(base.maxp * (kvf - th) / (1 - th), base.minp)
+        eq1 = min(max(F(wp, base.iterp), base.minp), base.maxp)
+        assert throttle_prefill(base.with_(policy=2), wp, free) == (0 if off else min(int(eq2), wp))
+        assert throttle_prefill(base.with_(policy=3), wp, free) == (0 if off else min(int(eq1), wp))
+
+
 def test_eq4_examples():
     c4 = SchedParams(pp_depth=4)
     assert throttle_decode(c4, 1000) == 250

@@ -81,6 +81,29 @@ def test_sarathi_policy_identical():
     _diff_run(SchedParams(pp_depth=4, num_blocks=3000, policy=1, token_budget=2048), st)
 
 
+@pytest.mark.parametrize("policy", [2, 3])
+def test_ablation_policies_identical(policy):
+    # PAPER.md §4.5 ablations ("w/o WT", "w/o UT"): C++ build_batch == oracle, byte for byte,
+    # including a KV-pressured run (w/o UT ignores KV pressure and so preempts)
+    st = make_stream("C1", 1000, n=400)
+    _diff_run(SchedParams(pp_depth=4, num_blocks=3000, policy=policy), st)
+    _diff_run(SchedParams(pp_depth=2, num_blocks=400, policy=policy), make_stream("C1", 1000, n=120))
+
+
+def test_policy_counts_abi():
+    from paper_conf_sc_00090d00l25_b200 import gllm
+    from oracle.scheduler import throttle_prefill
+    rng = np.random.default_rng(5)
+    for policy in (0, 2, 3):
+        cfg = SchedParams(num_blocks=1000, policy=policy)
+        for _ in range(300):
+            wp, free = int(rng.integers(0, 40000)), int(rng.integers(0, 1001))
+            P, _ = gllm.throttle_counts(cfg, wp, 0, free)
+            assert P == throttle_prefill(cfg, wp, free)
+    with pytest.raises(gllm.GllmError):
+        gllm.throttle_counts(SchedParams(num_blocks=1000, policy=7), 1, 0, 1)
+
+
 def test_warm_start_identical():
     st = make_stream("C4", 1000, n=40)
     st.warm = st.warm[:64]

@@ -50,7 +50,7 @@ class SchedParams:
     num_blocks: int = 64
     block_size: int = 16
     max_seqs: int = 1024      # L575
-    policy: int = 0           # 0 = Token Throttling; 1 = Sarathi-Serve (NEXT)
+    policy: int = 0           # 0 = Token Throttling; 1 = Sarathi-Serve; 2 = w/o WT; 3 = w/o UT (§4.5)
     token_budget: int = 2048  # Sarathi only (L248)
 
     def with_(self, **kw) -> "SchedParams":

@@ -26,10 +26,10 @@ from workloads.configs import MODELS, SCHED, STREAMS  # noqa: E402
 from workloads.streams import make_stream  # noqa: E402
 
 
-def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_us=0.0):
+def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_us=0.0, **sched_kw):
     m = MODELS[config]
     sp = SCHED[config].with_(pp_depth=pp, policy=policy, token_budget=2048,
-                             num_blocks=kv_blocks or SCHED[config].num_blocks)
+                             num_blocks=kv_blocks or SCHED[config].num_blocks, **sched_kw)
     lb, le = split_layers(m.n_layers, pp)[stage_idx]
     max_tokens = max(sp.maxp, sp.token_budget) + sp.max_seqs + 64
     st = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs)
@@ -96,11 +96,21 @@ if __name__ == "__main__":
     ap.add_argument("--stage", type=int, default=1)
     ap.add_argument("--ticks", type=int, default=160)
     ap.add_argument("--preroll", type=int, default=None)
+    ap.add_argument("--policies", default="0,1",
+                    help="0 token throttling, 1 Sarathi-Serve (w/ CK), 2 w/o WT, 3 w/o UT (PAPER.md §4.5)")
+    ap.add_argument("--sweep", default="",
+                    help="hyperparameter sensitivity (PAPER.md §4.6, Fig. 16) under token throttling, e.g. "
+                         "'iterp=1,2,4,8,16' or 'maxp=512,1024,2048' or 'kvthresh_num=0,1,2' (den 20)")
     a = ap.parse_args()
     preroll = a.preroll if a.preroll is not None else int(STREAMS[a.config].get("window", (400, None))[0])
     out = {"config": a.config, "pp": a.pp, "stage": a.stage, "ticks": a.ticks, "preroll": preroll}
-    for name, pol in (("token_throttling", 0), ("sarathi_serve", 1)):
-        t, toks, pre, dec = measure(a.config, a.pp, a.stage, pol, preroll, a.ticks)
+    names = {0: "token_throttling", 1: "sarathi_serve", 2: "no_wt", 3: "no_ut"}
+    runs = [(names[int(p)], int(p), {}) for p in a.policies.split(",") if p != ""]
+    if a.sweep:
+        key, vals = a.sweep.split("=")
+        runs = [(f"{key}={v}", 0, {key: int(v)}) for v in vals.split(",")]
+    for name, pol, kw in runs:
+        t, toks, pre, dec = measure(a.config, a.pp, a.stage, pol, preroll, a.ticks, **kw)
         mk, bub = simulate(t, a.pp)
         out[name] = {"tokens_per_s": round(float(toks.sum()) / (mk * 1e-3), 1), "bubble_fraction": round(bub, 4),
                      "stage_ms_mean": round(float(t.mean()), 3), "stage_ms_cv": round(float(t.std() / t.mean()), 3),

@@ -34,6 +34,7 @@ struct AttnArgs {
   float* part_o;       // [nparts, Hkv, G, D]
   float* part_ml;      // [nparts, Hkv, G, 2]
   int split_len;       // decode keys per split (multiple of 16)
+  int* part_ctr;       // [nparts * Hkv] split arrival counters (persistent decode kernel; kept zero)
 };
 
 // flattened (token, group-head) rows per prefill work item

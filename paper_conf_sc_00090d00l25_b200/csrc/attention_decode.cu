@@ -8,13 +8,14 @@
 // independent persistent worker: it claims work with one atomicAdd, and streams the item's
 // 16-key pages (K 4 KB + V 4 KB at D = 128, one contiguous [16][D] tile each in the paged
 // cache) through a private NST-slot ring in SMEM.  Lane 0 issues the loads as TMA tensor copies
-// (SW128 boxes of 16 x 64) plus a 1-D bulk copy of the item's G query rows, completing on the
-// slot's mbarrier; the page stream runs ahead ACROSS item boundaries, so the ring never drains
+// (SW128 boxes of 16 x 64) completing on the slot's mbarrier (the item's G query rows are read
+// from global, L2-hot, when its first page is consumed); the page stream runs ahead ACROSS item
+// boundaries, so the ring never drains
 // between items (the v1 kernel, attention.cu, paid a fill + merge per CTA).  The G heads are
 // the rows of an m16n8k16 tile: S = Q K^T (2 n-tiles x D/16 k-steps), online softmax with a
 // lazy reference max (rescale only when the max grows by > 2^8), O += P V (D/8 n-tiles).
-// A finished item writes bf16 rows, or (split rows) an fp32 partial merged by
-// decode_merge_kernel.  The last CTA to finish resets the work counter for the next launch.
+// A finished item writes bf16 rows, or (split rows) an fp32 partial; the last split of a row to
+// finish merges the partials in place.  The last CTA to finish resets the work counter.
 #include <cuda.h>
 #include <cuda_bf16.h>
 
@@ -28,12 +29,6 @@ namespace {
 
 constexpr float LOG2E_D = 1.4426950408889634f;
 
-__device__ __forceinline__ void bulk_load_1d(uint32_t smem_dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_dst),
-               "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(ptx::smem_u32(bar))
-               : "memory");
-}
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 // (row, 16-byte chunk) of a 16-row page stored as D/64 SW128 atoms of 16 x 128 B (TMA box layout)
@@ -45,10 +40,8 @@ template <int D, int G, int NST, int WARPS>
 struct DecLayout {
   static constexpr int PAGE = 16 * D * 2;          // one K (or V) page
   static constexpr int SLOT = 2 * PAGE;            // K page + V page
-  static constexpr int QB = G * D * 2;             // the G query rows of one (row, kv head)
   static constexpr int RING = NST * SLOT;          // per warp
-  static constexpr int QOFF = WARPS * RING;        // Q slots: [WARPS][NST][QB]
-  static constexpr int META = QOFF + WARPS * NST * QB;  // int4 [WARPS][NST]
+  static constexpr int META = WARPS * RING;        // int4 [WARPS][NST]
   static constexpr int BAR = META + WARPS * NST * 16;   // uint64 [WARPS][NST]
   static constexpr int BYTES = BAR + WARPS * NST * 8 + 1024;  // + 1024-B alignment slack
 };
@@ -66,8 +59,6 @@ __global__ void __launch_bounds__(WARPS * 32)
   const int g = lane >> 2, tq = lane & 3;
   uint8_t* ring = smem + warp * Lay::RING;
   const uint32_t ring_u32 = ptx::smem_u32(ring);
-  const uint32_t q_u32 = ptx::smem_u32(smem + Lay::QOFF + warp * NST * Lay::QB);
-  const uint8_t* qbase = smem + Lay::QOFF + warp * NST * Lay::QB;
   int4* meta = reinterpret_cast<int4*>(smem + Lay::META) + warp * NST;
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem + Lay::BAR) + warp * NST;
   const int Hkv = a.Hkv;
@@ -84,22 +75,45 @@ __global__ void __launch_bounds__(WARPS * 32)
   }
   __syncwarp();
 
-  // ---- issue side of the page stream (warp-uniform state; lane 0 issues)
-  int iw = 0, ip = 0, inp = 0, iq = 0;  // work index, page within the item, pages of the item, Q slot
+  // ---- issue side of the page stream (warp-uniform state; lane 0 issues).  Global reads on
+  // this path are issued a step before their value is needed: the next work item is claimed
+  // (atomicAdd) two pages before the current one ends -- not earlier, so a warp never sits on a
+  // claimed item while others idle (longest-first balance) -- and its header is read one page
+  // later; the block table is read 32 entries at a time (lane l holds page base + l).
+  int iw = 0, ip = 0, inp = 0;  // work index, page within the item, pages of the item
   int i_seq = 0, i_kvh = 0, i_nb0 = 0;
+  int nst = 0;                  // next item: 0 none claimed, 1 claimed (nv in flight), 2 header read
+  int nv = 0, n_iw = 0, n_L = 0;
+  DecodeItem n_it{0, 0, -1, 1};
+  int btw = 0;
+  const int32_t* bt_row = a.block_table;
+  auto claim = [&]() {
+    if (lane == 0) nv = atomicAdd(ctr, 1);
+    nst = 1;
+  };
+  auto resolve = [&]() {
+    n_iw = __shfl_sync(0xffffffffu, nv, 0);
+    if (n_iw < n_work) {
+      n_it = items[n_iw / Hkv];
+      n_L = a.kv_len[n_it.seq];
+    }
+    nst = 2;
+  };
   auto fetch = [&]() {
-    int v = 0;
-    if (lane == 0) v = atomicAdd(ctr, 1);
-    iw = __shfl_sync(0xffffffffu, v, 0);
+    if (nst == 0) claim();
+    if (nst == 1) resolve();
+    nst = 0;
+    iw = n_iw;
     ip = 0;
     if (iw < n_work) {
-      const DecodeItem it = items[iw / Hkv];
       i_kvh = iw % Hkv;
-      i_seq = it.seq;
-      const int L = a.kv_len[it.seq];
-      const int k0 = it.split * a.split_len, k1 = min(L, k0 + a.split_len);
+      i_seq = n_it.seq;
+      const int k0 = n_it.split * a.split_len, k1 = min(n_L, k0 + a.split_len);
       i_nb0 = k0 / 16;
       inp = (k1 + 15) / 16 - i_nb0;
+      bt_row = a.block_table + (size_t)i_seq * a.maxblk + i_nb0;
+      btw = lane < inp ? __ldg(bt_row + lane) : 0;
+      if (inp <= 2) claim();
     }
   };
   auto issue = [&](int s) {
@@ -107,27 +121,28 @@ __global__ void __launch_bounds__(WARPS * 32)
       if (lane == 0) meta[s] = make_int4(-1, 0, 0, 0);
       return;
     }
-    const int blk = a.block_table[(size_t)i_seq * a.maxblk + i_nb0 + ip];
+    const int blk = __shfl_sync(0xffffffffu, btw, ip & 31);
     if (lane == 0) {
       const int row = (blk * Hkv + i_kvh) * 16;
       const bool first = ip == 0;
       fence_proxy_async();  // this slot's earlier generic reads (ldmatrix) before the async writes
-      ptx::mbar_arrive_expect_tx(&bar[s], Lay::SLOT + (first ? Lay::QB : 0));
+      ptx::mbar_arrive_expect_tx(&bar[s], Lay::SLOT);
       uint8_t* dst = ring + s * Lay::SLOT;
 #pragma unroll
       for (int at = 0; at < ATOMS; ++at) {
         ptx::tma_load_2d_hint(dst + at * 2048, &tmk, &bar[s], at * 64, row, pol);
         ptx::tma_load_2d_hint(dst + Lay::PAGE + at * 2048, &tmv, &bar[s], at * 64, row, pol);
       }
-      if (first) {
-        const int t = a.cu_q[i_seq];
-        bulk_load_1d(q_u32 + iq * Lay::QB, a.q + (size_t)t * a.q_stride + (size_t)i_kvh * G * D, Lay::QB, &bar[s]);
-      }
-      meta[s] = make_int4(iw, ip, (ip == inp - 1 ? 1 : 0) | (first ? 2 : 0), iq);
+      meta[s] = make_int4(iw, ip, (ip == inp - 1 ? 1 : 0) | (first ? 2 : 0), 0);
     }
     if (++ip == inp) {
-      iq = (iq + 1) % NST;
       fetch();
+    } else {
+      if ((ip & 31) == 0) btw = ip + lane < inp ? __ldg(bt_row + ip + lane) : 0;
+      if (nst == 1)
+        resolve();
+      else if (nst == 0 && ip == inp - 2)
+        claim();
     }
   };
 
@@ -139,7 +154,7 @@ __global__ void __launch_bounds__(WARPS * 32)
   uint32_t qa[D / 16][4];
   float o[D / 8][4];
   float mrow[2] = {-INFINITY, -INFINITY}, lrow[2] = {0.f, 0.f};
-  int c_seq = 0, c_kvh = 0, c_k1 = 0, c_nb0 = 0, c_part = -1;
+  int c_seq = 0, c_kvh = 0, c_k1 = 0, c_nb0 = 0, c_part = -1, c_split = 0, c_nsplit = 1;
 #pragma unroll 1
   for (int i = 0;; ++i) {
     const int s = i % NST;
@@ -147,8 +162,7 @@ __global__ void __launch_bounds__(WARPS * 32)
     __syncwarp();
     const int4 mt = meta[s];
     if (mt.x < 0) break;
-    ptx::mbar_wait(&bar[s], (uint32_t)((i / NST) & 1));
-    if (mt.z & 2) {  // first page of a work item: its Q rows arrived with this page
+    if (mt.z & 2) {  // first page of a work item: its G query rows straight from global (L2)
       const DecodeItem it = items[mt.x / Hkv];
       c_kvh = mt.x % Hkv;
       c_seq = it.seq;
@@ -157,13 +171,15 @@ __global__ void __launch_bounds__(WARPS * 32)
       c_k1 = min(L, k0 + a.split_len);
       c_nb0 = k0 / 16;
       c_part = it.part;
-      const uint8_t* qs = qbase + mt.w * Lay::QB;
+      c_split = it.split;
+      c_nsplit = it.nsplit;
+      const __nv_bfloat16* qrow = a.q + (size_t)a.cu_q[c_seq] * a.q_stride + (size_t)(c_kvh * G + (g < G ? g : 0)) * D;
 #pragma unroll
       for (int ks = 0; ks < D / 16; ++ks) {
         const int c0 = ks * 16 + 2 * tq;
-        qa[ks][0] = g < G ? *reinterpret_cast<const uint32_t*>(qs + (g * D + c0) * 2) : 0u;
+        qa[ks][0] = g < G ? __ldg(reinterpret_cast<const unsigned int*>(qrow + c0)) : 0u;
         qa[ks][1] = 0u;  // rows 8..15 (G <= 8)
-        qa[ks][2] = g < G ? *reinterpret_cast<const uint32_t*>(qs + (g * D + c0 + 8) * 2) : 0u;
+        qa[ks][2] = g < G ? __ldg(reinterpret_cast<const unsigned int*>(qrow + c0 + 8)) : 0u;
         qa[ks][3] = 0u;
       }
 #pragma unroll
@@ -171,6 +187,7 @@ __global__ void __launch_bounds__(WARPS * 32)
       mrow[0] = mrow[1] = -INFINITY;
       lrow[0] = lrow[1] = 0.f;
     }
+    ptx::mbar_wait(&bar[s], (uint32_t)((i / NST) & 1));
     const uint32_t kst = ring_u32 + s * Lay::SLOT;
     const uint32_t vst = kst + Lay::PAGE;
     float sc[2][4] = {{0.f, 0.f, 0.f, 0.f}, {0.f, 0.f, 0.f, 0.f}};
@@ -248,6 +265,57 @@ __global__ void __launch_bounds__(WARPS * 32)
           }
         }
       }
+      if (c_part >= 0) {
+        // split row: the last split to arrive merges all partials of (row, kv head) in place
+        // (threadfence + arrival counter, as split-K fix-up) -- no separate merge launch
+        const int first = c_part - c_split;
+        __threadfence();
+        __syncwarp();
+        int prev = 0;
+        if (lane == 0) prev = atomicAdd(a.part_ctr + (size_t)first * Hkv + c_kvh, 1);
+        prev = __shfl_sync(0xffffffffu, prev, 0);
+        if (prev == c_nsplit - 1) {
+          __threadfence();
+          if (lane == 0) a.part_ctr[(size_t)first * Hkv + c_kvh] = 0;  // ready for the next launch
+          // lane owns elements lane + 32k of the G x D output; all loads of one split are
+          // independent (issued together), so the merge costs ~nsplit L2 round trips
+          constexpr int PER = G * D / 32;
+          const int t = a.cu_q[c_seq];
+          float M[G], Ls[G], acc[PER];
+#pragma unroll
+          for (int h = 0; h < G; ++h) {
+            M[h] = -INFINITY;
+            Ls[h] = 0.f;
+          }
+#pragma unroll
+          for (int k = 0; k < PER; ++k) acc[k] = 0.f;
+          for (int sp = 0; sp < c_nsplit; ++sp) {
+            const size_t b0 = ((size_t)(first + sp) * Hkv + c_kvh) * G;
+#pragma unroll
+            for (int h = 0; h < G; ++h) M[h] = fmaxf(M[h], __ldcg(a.part_ml + (b0 + h) * 2));
+          }
+          for (int sp = 0; sp < c_nsplit; ++sp) {
+            const size_t b0 = ((size_t)(first + sp) * Hkv + c_kvh) * G;
+            float f[G];
+#pragma unroll
+            for (int h = 0; h < G; ++h) {
+              const float2 ml = __ldcg(reinterpret_cast<const float2*>(a.part_ml + (b0 + h) * 2));
+              f[h] = exp2f(ml.x - M[h]);
+              Ls[h] += ml.y * f[h];
+            }
+#pragma unroll
+            for (int k = 0; k < PER; ++k) {
+              const int idx = lane + 32 * k;
+              acc[k] += __ldcg(a.part_o + b0 * D + idx) * f[idx / D];
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < PER; ++k) {
+            const int idx = lane + 32 * k;
+            a.out[(size_t)t * a.Hq * D + (size_t)c_kvh * G * D + idx] = __float2bfloat16_rn(acc[k] / Ls[idx / D]);
+          }
+        }
+      }
     }
     __syncwarp();  // all lanes done reading slot s before it is refilled
   }
@@ -261,27 +329,6 @@ __global__ void __launch_bounds__(WARPS * 32)
       ctr[1] = 0;
       __threadfence();
     }
-  }
-}
-
-template <int D, int G>
-__global__ void __launch_bounds__(128) decode_merge2_kernel(const AttnArgs a, const MergeItem* __restrict__ merges) {
-  const MergeItem mi = merges[blockIdx.x];
-  const int kvh = blockIdx.y;
-  const int t = a.cu_q[mi.seq];
-  for (int idx = threadIdx.x; idx < G * D; idx += blockDim.x) {
-    const int h = idx / D, d = idx % D;
-    float M = -INFINITY;
-    for (int s = 0; s < mi.nsplit; ++s)
-      M = fmaxf(M, a.part_ml[(((size_t)(mi.first + s) * a.Hkv + kvh) * G + h) * 2]);
-    float Ls = 0.f, A = 0.f;
-    for (int s = 0; s < mi.nsplit; ++s) {
-      const size_t base = ((size_t)(mi.first + s) * a.Hkv + kvh) * G + h;
-      const float f = exp2f(a.part_ml[base * 2] - M);
-      Ls += a.part_ml[base * 2 + 1] * f;
-      A += a.part_o[base * D + d] * f;
-    }
-    a.out[(size_t)t * a.Hq * D + (size_t)(kvh * G + h) * D + d] = __float2bfloat16_rn(A / Ls);
   }
 }
 
@@ -306,7 +353,8 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
     if (grid > need) grid = need;
     decode_attn_tma_kernel<D, G, NST, WARPS><<<grid, WARPS * 32, Lay::BYTES, s>>>(a, items, n_work, ctr, tmk, tmv);
   }
-  if (n_merges > 0) decode_merge2_kernel<D, G><<<dim3(n_merges, a.Hkv), 128, 0, s>>>(a, merges);
+  (void)merges;
+  (void)n_merges;  // split rows are merged inside the kernel by their last split
   return GLLM_OK;
 }
 
@@ -315,6 +363,7 @@ int launch_g(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
              const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   if (g_dec_warps == 8) return launch_t<D, G, 3, 8>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
   if (g_dec_warps == 2) return launch_t<D, G, 4, 2>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
+  if (g_dec_warps == 3) return launch_t<D, G, 4, 3>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
   return launch_t<D, G, 3, 4>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
 }
 

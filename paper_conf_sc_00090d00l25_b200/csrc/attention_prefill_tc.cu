@@ -79,6 +79,11 @@ __device__ __forceinline__ void tmem_st_32x32b_x32(uint32_t taddr, const uint32_
       "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
       : "memory");
 }
+__device__ __forceinline__ float fast_exp2(float x) {  // ex2.approx: 2^-inf = +0
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 __device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 // D[tmem] (+)= A[tmem] . B[smem]: the A operand (here P, bf16 pairs per 32-bit column, row = lane)
 // is read from TMEM
@@ -190,14 +195,20 @@ __global__ void __launch_bounds__(128, 2)
     ptx::tmem_ld_32x32b_x32(t_s, sr[0]);
     ptx::tmem_ld_32x32b_x32(t_s + 32, sr[1]);
     ptx::tmem_ld_wait();
+    // raw scores; the causal mask is applied only on tiles that cross this row's diagonal, and
+    // the 1/sqrt(D)*log2(e) scale is folded into the max and into the exp2 argument (one FFMA)
     float s[64];
-    float mx = -INFINITY;
 #pragma unroll
-    for (int i = 0; i < 64; ++i) {
-      const int key = j * TC_KT + i;
-      s[i] = key <= pos ? __uint_as_float(sr[i >> 5][i & 31]) * sl2 : -INFINITY;
-      mx = fmaxf(mx, s[i]);
+    for (int i = 0; i < 64; ++i) s[i] = __uint_as_float(sr[i >> 5][i & 31]);
+    if (j * TC_KT + TC_KT - 1 > pos) {
+#pragma unroll
+      for (int i = 0; i < 64; ++i)
+        if (j * TC_KT + i > pos) s[i] = -INFINITY;
     }
+    float mx4[4] = {s[0], s[1], s[2], s[3]};
+#pragma unroll
+    for (int i = 4; i < 64; ++i) mx4[i & 3] = fmaxf(mx4[i & 3], s[i]);
+    const float mx = fmaxf(fmaxf(mx4[0], mx4[1]), fmaxf(mx4[2], mx4[3])) * sl2;
     // lazy rescale: exact because l and O share the reference max.  tcgen05.ld/st are warp-
     // collective (.sync.aligned), so the O pass runs for the whole warp when any lane needs it
     // (lanes that do not rescale multiply by 1).
@@ -222,12 +233,15 @@ __global__ void __launch_bounds__(128, 2)
     // P row (bf16 pairs) -> TMEM cols [64, 96): the A operand of the PV MMA
     {
       uint32_t pw[32];
+      float la = 0.f, lb = 0.f;
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
-        const float p0 = exp2f(s[2 * i] - m_ref), p1 = exp2f(s[2 * i + 1] - m_ref);
-        l += p0 + p1;
+        const float p0 = fast_exp2(fmaf(s[2 * i], sl2, -m_ref)), p1 = fast_exp2(fmaf(s[2 * i + 1], sl2, -m_ref));
+        la += p0;
+        lb += p1;
         pw[i] = ptx::pack_bf16(p0, p1);
       }
+      l += la + lb;
       tmem_st_32x32b_x32(t_p, pw);
       tmem_st_wait();
     }

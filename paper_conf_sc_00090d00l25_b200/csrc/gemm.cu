@@ -258,6 +258,10 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     // added, and chunk 0 is in flight while the MMAs finish
     float4 xa[8], xb[8];
     if (ok && !partial) {
+      // the whole 1 KB residual row segment is pulled into L2 while this tile's MMAs still run
+      // (the register double buffer below only looks one 128-B chunk ahead)
+#pragma unroll
+      for (int c = 0; c < GEMM_BN / 32; ++c) asm volatile("prefetch.global.L2 [%0];" ::"l"(rowp + c * 32));
 #pragma unroll
       for (int q = 0; q < 8; ++q) xa[q] = reinterpret_cast<const float4*>(rowp)[q];
     }

@@ -132,6 +132,7 @@ struct gllm_stage {
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
   float *part_o = nullptr, *part_ml = nullptr;
+  int* part_ctr = nullptr;
   int parts_cap = 0;
   std::vector<Prepared> prep;  // [0, RING): internal ring of stage_forward; others: gllm_stage_prepare handles
   int ring_i = 0;
@@ -243,6 +244,8 @@ void destroy(gllm_stage* st) {
   cudaSetDevice(st->device);
   cudaDeviceSynchronize();
   for (void* p : st->allocs) cudaFree(p);
+  for (void* p : {(void*)st->part_o, (void*)st->part_ml, (void*)st->part_ctr})
+    if (p) cudaFree(p);
   for (auto& p : st->prep) {
     if (p.host) cudaFreeHost(p.host);
     if (p.dev) cudaFree(p.dev);
@@ -287,12 +290,17 @@ int ensure_parts(gllm_stage* st, int parts) {
   const int cap = std::max(parts * 2, 1024);
   const size_t G = st->cfg.n_heads / st->cfg.n_kv_heads;
   float *po = nullptr, *pm = nullptr;
+  int* pc = nullptr;
   CK(cudaMalloc(&po, (size_t)cap * st->cfg.n_kv_heads * G * st->cfg.head_dim * sizeof(float)));
   CK(cudaMalloc(&pm, (size_t)cap * st->cfg.n_kv_heads * G * 2 * sizeof(float)));
+  CK(cudaMalloc(&pc, (size_t)cap * st->cfg.n_kv_heads * sizeof(int)));
+  CK(cudaMemset(pc, 0, (size_t)cap * st->cfg.n_kv_heads * sizeof(int)));
   if (st->part_o) cudaFree(st->part_o);
   if (st->part_ml) cudaFree(st->part_ml);
+  if (st->part_ctr) cudaFree(st->part_ctr);
   st->part_o = po;
   st->part_ml = pm;
+  st->part_ctr = pc;
   st->parts_cap = cap;
   return GLLM_OK;
 }
@@ -504,9 +512,9 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   if (ND > 0) {
     // split long contexts so that the decode grid has >= ~8 CTAs per SM of work; a split is
     // at least 32 pages (512 keys) so the merge pass stays negligible
-    // (persistent kernel: ~32 work units per SM for the dynamic longest-first schedule, a split
-    // is at least 16 pages)
-    const int64_t target = (st->decode_v1 ? 8LL : 32LL) * st->num_sms;  // work units
+    // (persistent kernel: one warp worker's fair share -- 8 resident warps per SM -- so only rows
+    // longer than the average per-warp work are split; a split is at least 16 pages)
+    const int64_t target = 8LL * st->num_sms;  // CTAs (v1) / warp workers (persistent kernel)
     int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
     split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(st->decode_v1 ? 32 : 16, per));
   }
@@ -624,6 +632,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
   aa.out = st->attn;
   aa.part_o = st->part_o;
   aa.part_ml = st->part_ml;
+  aa.part_ctr = st->part_ctr;
   aa.split_len = P.split_len;
   // Fused RMSNorm (a4): y holds bf16(x) and ss_a / ss_b the per-row sum of squares of x; the
   // consumer GEMMs (QKV, gate_up) scale their rows by rsqrt(ss/H + eps) in the epilogue and the
@@ -695,7 +704,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     aa.kc = w.kc;
     aa.vc = w.vc;
     auto decode = [&](cudaStream_t ds) -> int {
-      st->last_launches += P.n_mi ? 2 : 1;
+      st->last_launches += (P.n_mi && st->decode_v1) ? 2 : 1;  // the persistent kernel merges in place
       if (st->decode_v1) return gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, ds);
       return gllm::launch_decode_attention_tma(aa, w.tm_kc, w.tm_vc, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
                                                st->num_sms, ds);

@@ -499,19 +499,30 @@ const bool g_prefill_v1 = [] {
   return !(e && e[0] == '1');
 }();
 
+// Dynamic SMEM actually reserved per prefill CTA.  Padding it past half an SM (GLLM_PREFILL_PAD_KB)
+// caps prefill at one CTA per SM, leaving the other slot to a persistent decode CTA that runs
+// concurrently (A/B knob; see stage.cu attention step).
+int prefill_smem_bytes(int need) {
+  static const int pad = [] {
+    const char* e = std::getenv("GLLM_PREFILL_PAD_KB");
+    return e ? std::atoi(e) * 1024 : 0;
+  }();
+  return need > pad ? need : pad;
+}
+
 template <int D>
 int launch_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
+  const int bytes = prefill_smem_bytes(TcSmem<D>::BYTES);
   static bool set = false;
   if (!set) {
-    cudaFuncSetAttribute(prefill_attn_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, TcSmem<D>::BYTES);
-    cudaFuncSetAttribute(prefill_attn_tc_v1_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         TcSmem<D>::BYTES);
+    cudaFuncSetAttribute(prefill_attn_tc_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(prefill_attn_tc_v1_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
   if (g_prefill_v1)
-    prefill_attn_tc_v1_kernel<D><<<dim3(n_items, a.Hkv), 128, TcSmem<D>::BYTES, s>>>(a, items);
+    prefill_attn_tc_v1_kernel<D><<<dim3(n_items, a.Hkv), 128, bytes, s>>>(a, items);
   else
-    prefill_attn_tc_kernel<D><<<dim3(n_items, a.Hkv), 128, TcSmem<D>::BYTES, s>>>(a, items);
+    prefill_attn_tc_kernel<D><<<dim3(n_items, a.Hkv), 128, bytes, s>>>(a, items);
   return GLLM_OK;
 }
 

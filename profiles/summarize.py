@@ -108,7 +108,7 @@ def main(src, dst):
                 traffic[cat] = d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
         md.append("")
     open(os.path.join(dst, "ncu_summary.md"), "w").write("\n".join(md) + "\n")
-    tp = os.path.join(os.path.dirname(dst.rstrip("/")), "traffic.json")
+    tp = os.path.join(os.path.dirname(os.path.abspath(__file__)), "traffic.json")
     allt = json.load(open(tp)) if os.path.exists(tp) else {}
     allt["C1-pp1"] = {**allt.get("C1-pp1", {}), **traffic}
     json.dump(allt, open(tp, "w"), indent=1)

@@ -44,7 +44,8 @@ struct Cfg {
 #else
   static constexpr int STAGES = CG == 2 ? 6 : GEMM_STAGES;
 #endif
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int STG_FLOATS = 32 * 36;  // per epilogue warp: 32 x 32 transpose tile (row stride 36)
+  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + 4 * STG_FLOATS * 4;
   static constexpr int TILE_M = GEMM_BM * CG;  // rows of one (cluster) tile
 };
 
@@ -217,7 +218,7 @@ __device__ __forceinline__ float row_scale(const GemmArgs& p, int row) {
 // apply the fused epilogue.  `partial`: stream-K segment, combine atomically.
 template <int EPI>
 __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
-                                              uint64_t* tfull_bar, uint32_t parity) {
+                                              uint64_t* tfull_bar, uint32_t parity, float* stg) {
   const bool row_ok = row < p.M;
   const float rs = (EPI == EPI_ADD_F32 || EPI == EPI_ARGMAX) ? 1.0f : row_scale(p, row);
   if (p.zero_rows != nullptr && n_blk == 0 && row_ok && !partial && p.ws == nullptr) p.zero_rows[row] = 0.f;
@@ -252,58 +253,82 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       }
     }
   } else if constexpr (EPI == EPI_ADD_F32) {
-    float* rowp = reinterpret_cast<float*>(p.out) + (size_t)row * p.ldo + n_blk * GEMM_BN;
-    const bool ok = row_ok && n_blk * GEMM_BN < p.N;
-    // residual chunks are double-buffered in registers: chunk c+1 is loaded while chunk c is
-    // added, and chunk 0 is in flight while the MMAs finish
-    float4 xa[8], xb[8];
-    if (ok && !partial) {
-      // the whole 1 KB residual row segment is pulled into L2 while this tile's MMAs still run
-      // (the register double buffer below only looks one 128-B chunk ahead)
-#pragma unroll
-      for (int c = 0; c < GEMM_BN / 32; ++c) asm volatile("prefetch.global.L2 [%0];" ::"l"(rowp + c * 32));
-#pragma unroll
-      for (int q = 0; q < 8; ++q) xa[q] = reinterpret_cast<const float4*>(rowp)[q];
-    }
-    wait_acc();
-    float ssl = 0.f;  // fused RMSNorm statistics of the new residual row (this tile's columns)
-#pragma unroll
-    for (int c = 0; c < GEMM_BN / 32; ++c) {
-      if (ok && !partial && c + 1 < GEMM_BN / 32) {
-#pragma unroll
-        for (int q = 0; q < 8; ++q) xb[q] = reinterpret_cast<const float4*>(rowp + (c + 1) * 32)[q];
+    if (partial) {  // stream-K segment: fp32 vector reductions, one row per thread
+      float* rowp = reinterpret_cast<float*>(p.out) + (size_t)row * p.ldo + n_blk * GEMM_BN;
+      wait_acc();
+#pragma unroll 1
+      for (int c = 0; c < GEMM_BN / 32; ++c) {
+        ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+        ptx::tmem_ld_wait();
+        if (row_ok && n_blk * GEMM_BN + c * 32 < p.N) atomic_add_f32x32(rowp + c * 32, r);
       }
-      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-      ptx::tmem_ld_wait();
-      if (ok) {
-        if (partial) {
-          atomic_add_f32x32(rowp + c * 32, r);
-        } else {
-          float4* dst = reinterpret_cast<float4*>(rowp + c * 32);
-          float nx[32];
+    } else {
+      // Whole tile: each 32 x 32 chunk of the accumulator (thread = row after tcgen05.ld) is
+      // re-laid through SMEM so that 8 lanes cover one row's 32 columns (float4 each): every
+      // warp access of the residual read-modify-write and of the bf16 copy for the next norm
+      // is 4 whole 128-B (64-B) row segments instead of 32 scattered rows, which keeps the
+      // L1/SMEM pipe free for the concurrent mainloop's operand reads.
+      const int lane = threadIdx.x & 31, row0 = row - lane;
+      const int rsub = lane >> 3, c4 = (lane & 7) * 4;  // this lane: rows rsub + 4k, columns c4..c4+3
+      float ss[8];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            float4 x = xa[q];
-            x.x += __uint_as_float(r[q * 4 + 0]);
-            x.y += __uint_as_float(r[q * 4 + 1]);
-            x.z += __uint_as_float(r[q * 4 + 2]);
-            x.w += __uint_as_float(r[q * 4 + 3]);
-            dst[q] = x;
-            xa[q] = xb[q];
-            nx[q * 4 + 0] = x.x;
-            nx[q * 4 + 1] = x.y;
-            nx[q * 4 + 2] = x.z;
-            nx[q * 4 + 3] = x.w;
-          }
-          if (p.xb_out) {
+      for (int k = 0; k < 8; ++k) ss[k] = 0.f;
+      wait_acc();
+#pragma unroll 1
+      for (int c = 0; c < GEMM_BN / 32; ++c) {
+        ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+        ptx::tmem_ld_wait();
 #pragma unroll
-            for (int j = 0; j < 32; ++j) ssl = fmaf(nx[j], nx[j], ssl);
-            store_bf16x32(p.xb_out + (size_t)row * p.ldo + n_blk * GEMM_BN + c * 32, nx);
+        for (int q = 0; q < 8; ++q)  // row `lane` of the chunk (stride 36 floats: conflict-free v4)
+          *reinterpret_cast<float4*>(stg + lane * 36 + 4 * q) =
+              make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]), __uint_as_float(r[4 * q + 2]),
+                          __uint_as_float(r[4 * q + 3]));
+        __syncwarp();
+        const int col = n_blk * GEMM_BN + c * 32 + c4;
+        const bool col_ok = col < p.N;
+        float4 xv[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int rr = rsub + 4 * k;
+          xv[k] = (col_ok && row0 + rr < p.M)
+                      ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.out) +
+                                                         (size_t)(row0 + rr) * p.ldo + col)
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int rr = rsub + 4 * k;
+          if (col_ok && row0 + rr < p.M) {
+            const float4 a4 = *reinterpret_cast<const float4*>(stg + rr * 36 + c4);
+            float4 x = xv[k];
+            x.x += a4.x;
+            x.y += a4.y;
+            x.z += a4.z;
+            x.w += a4.w;
+            *reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + (size_t)(row0 + rr) * p.ldo + col) = x;
+            if (p.xb_out) {
+              uint2 b;
+              b.x = ptx::pack_bf16(x.x, x.y);
+              b.y = ptx::pack_bf16(x.z, x.w);
+              *reinterpret_cast<uint2*>(p.xb_out + (size_t)(row0 + rr) * p.ldo + col) = b;
+              ss[k] = fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, fmaf(x.w, x.w, ss[k]))));
+            }
           }
+        }
+        __syncwarp();
+      }
+      if (p.ss_out) {  // row rsub + 4k: its 32 columns of this tile are spread over 8 lanes
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          float v = ss[k];
+          v += __shfl_xor_sync(0xffffffffu, v, 1);
+          v += __shfl_xor_sync(0xffffffffu, v, 2);
+          v += __shfl_xor_sync(0xffffffffu, v, 4);
+          const int rw = row0 + rsub + 4 * k;
+          if ((lane & 7) == 0 && rw < p.M && n_blk * GEMM_BN < p.N) atomicAdd(p.ss_out + rw, v);
         }
       }
     }
-    if (ok && !partial && p.ss_out) atomicAdd(p.ss_out + row, ssl);
   } else if constexpr (EPI == EPI_SILU_MUL) {
     wait_acc();
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
@@ -385,6 +410,7 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(tempty + 2);
+  float* stg = reinterpret_cast<float*>(sB + C::STAGES * C::B_BYTES + 256);  // epilogue transpose tiles
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -501,7 +527,7 @@ __global__ void __launch_bounds__(256, 1)
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
-      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase);
+      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) {

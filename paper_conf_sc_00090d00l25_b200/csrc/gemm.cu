@@ -19,6 +19,8 @@
 #include <cudaTypedefs.h>
 
 #include <cstdio>
+#include <cstdlib>
+#include <cstring>
 #include <mutex>
 
 #include "common.h"
@@ -606,16 +608,22 @@ int choose_streamk(int M, int N, int ntiles, int nk, int epi, int num_sms) {
   return (eff < 0.5 && (size_t)M * N <= GEMM_WS_ELEMS) ? 1 : 0;
 }
 
-// CTA-pair tiles need at least one wave of 256 x 256 tiles.  Measured on B200 (tools/gemm_bench.py,
-// profiles/r01): the pair kernel is +17% on the C1 QKV shape (2094x6144x4096) and +11% on
-// 8192^3, but 3-7% slower on the O / gate_up / down shapes at T ~ 2094, so those keep the
-// 1-CTA kernel unless M is large.
+// CTA-pair tiles need at least one wave of 256 x 256 tiles.  Measured on B200 (tools/ab_bench.sh,
+// profiles/r01/ab_gemm_cg.txt): with the coalesced residual epilogue the pair kernel wins for
+// every epilogue at the C1 shapes (T ~ 2090: O 0.62 -> 0.67, down 0.83 -> 0.93, gate_up 0.96 ->
+// 1.0 of sustained cuBLAS bf16; QKV was already on it).  GLLM_GEMM_CG1=1 restores the 1-CTA
+// kernel for the residual-add / SiLU epilogues (A/B).
+const bool g_cg1_rest = [] {
+  const char* e = std::getenv("GLLM_GEMM_CG1");
+  return e && e[0] == '1';
+}();
+
 int choose_cg(int M, int N, int epi, int num_sms) {
   if (g_force_cg) return g_force_cg;
   const int tiles2 = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
   if (M < 256 || tiles2 * 2 < num_sms || epi == EPI_ARGMAX) return 1;
   if (epi == EPI_STORE_BF16 || epi == EPI_QKV_ROPE) return 2;
-  return M >= 4096 ? 2 : 1;
+  return g_cg1_rest && M < 4096 ? 1 : 2;
 }
 
 }  // namespace

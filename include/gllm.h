@@ -59,7 +59,8 @@ typedef struct {
 /* (L136 Fig.6).  Host-only, deterministic, single-threaded per object. */
 /* ------------------------------------------------------------------------ */
 /* build_batch policies (gllm_sched_cfg.policy) */
-enum { GLLM_POLICY_THROTTLE = 0, GLLM_POLICY_SARATHI = 1, GLLM_POLICY_NO_WT = 2, GLLM_POLICY_NO_UT = 3 };
+enum { GLLM_POLICY_THROTTLE = 0, GLLM_POLICY_SARATHI = 1, GLLM_POLICY_NO_WT = 2, GLLM_POLICY_NO_UT = 3,
+       GLLM_POLICY_CTX = 4 };
 
 typedef struct {
   int32_t iterp;          /* #T  (Eq.1/Eq.3; default 8, L248) */
@@ -74,8 +75,14 @@ typedef struct {
                              1 = Sarathi-Serve (every ready decode, prefill to token_budget; "w/ CK", L310);
                              2 = ablation "w/o WT" (Eq.3 without the #WP/#T term, L308);
                              3 = ablation "w/o UT" (Eq.1 + the L165 threshold, L308).
-                             Policies 2-3 keep Eq.4 for decodes (§4.5, Fig. 15). */
+                             Policies 2-3 keep Eq.4 for decodes (§4.5, Fig. 15).
+                             4 = context-aware Token Throttling (the paper's future work, L354;
+                             reading R21 in DESIGN.md): #P of Eq.3 is a budget in token
+                             equivalents and a chunk of c tokens at offset s costs
+                             c + floor((c*s + c*(c+1)/2) / attn_pairs_per_token). */
   int32_t token_budget;   /* Sarathi only (2048, L248) */
+  int32_t attn_pairs_per_token; /* policy 4 only: causal (query, key) pairs whose attention costs
+                             as much as one token's linear layers (>= 1) */
 } gllm_sched_cfg;
 
 typedef struct gllm_sched gllm_sched;

@@ -52,6 +52,15 @@ def throttle_prefill(cfg, wp: int, free: int) -> int:
     return min(max(min(wp // cfg.iterp, cap), cfg.minp), wp)         # Eq.3, capped by WP (R11)
 
 
+def chunk_cost(s: int, c: int, a: int) -> int:
+    """Reading R21 (policy 4, context-aware Token Throttling; PAPER.md L354 future work): the
+    token-equivalent cost of a prefill chunk of c tokens at offset s = its c tokens of linear
+    work plus its causal (query, key) pairs c*s + c(c+1)/2 (query s+j sees keys 0..s+j), in units
+    of `a` pairs per token, rounded down."""
+    pairs = sum(s + j + 1 for j in range(c))
+    return c + pairs // a
+
+
 def throttle_decode(cfg, rd: int) -> int:
     """#D = ceil(#RD / #PP_depth) (Eq.4; ceil per reading R6)."""
     return -(-rd // cfg.pp_depth)
@@ -252,9 +261,22 @@ class Scheduler:
             if fresh and running >= cfg.max_seqs:
                 continue
             remaining = r.prefill_len - r.sched_prompt
-            want = min(remaining, p_left)
             capacity = (len(r.blocks) + len(self.free)) * bs - r.sched_prompt
-            c = min(want, capacity)
+            if cfg.policy == 4:
+                # R21: the longest chunk whose cost fits the budget left (linear scan from 0)
+                a, s0 = cfg.attn_pairs_per_token, r.sched_prompt
+                c, pairs = 0, 0
+                while c < min(remaining, capacity):
+                    nxt = pairs + (s0 + c + 1)  # query s0+c attends keys 0..s0+c
+                    if (c + 1) + nxt // a > p_left:
+                        break
+                    c, pairs = c + 1, nxt
+                if c == 0 and not chunks and capacity > 0:
+                    c, pairs = 1, s0 + 1        # progress: at least one token per tick
+                cost = c + pairs // a
+            else:
+                c = min(remaining, p_left, capacity)
+                cost = c
             if c <= 0:
                 break
             need = -(-(r.sched_prompt + c) // bs) - len(r.blocks)
@@ -264,8 +286,8 @@ class Scheduler:
                 running += 1
             chunks.append((r, r.sched_prompt, c))
             r.sched_prompt += c
-            p_left -= c
-            if c < want:
+            p_left = max(p_left - cost, 0)
+            if c < remaining:                   # budget spent or KV capacity reached (R13)
                 break
         # layout (R15): prefill chunks first, then decodes
         tok, pos_l, slot, cu, kvl, samp, seq_ids, rows = [], [], [], [0], [], [], [], []

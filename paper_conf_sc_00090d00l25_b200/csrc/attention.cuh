@@ -42,6 +42,11 @@ int prefill_rows_per_item();
 int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
 // same work items on tcgen05 (S and O in TMEM); the default prefill path
 int launch_prefill_attention_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
+// warp-specialised tcgen05 prefill (attention_prefill_ws.cu), the default: items of
+// prefill_ws_rows_per_item() rows (two 128-row Q tiles); K/V pages by TMA through the decode page maps
+int prefill_ws_rows_per_item();
+int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
+                                const PrefillItem* items, int n_items, cudaStream_t s);
 int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
                             int n_merges, cudaStream_t s);
 // persistent warp-worker decode kernel fed by TMA (attention_decode.cu), the default; `tmk` /

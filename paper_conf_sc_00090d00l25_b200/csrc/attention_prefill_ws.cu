@@ -1,0 +1,439 @@
+// Prefill (chunked, causal, paged) attention, warp-specialised on tcgen05 -- part of a7.
+//
+// PAPER.md L77 (prefill is compute-bound), L212 (attention over the paged KV cache), L354 (cost
+// quadratic in context).  Computes, for every row of a prefill chunk at offset s0,
+//   o = softmax(q K[0..s0+j]^T / sqrt(D)) V[0..s0+j]      (GQA: query head h reads kv head h / G)
+//
+// CTA = two Q tiles (A, B) of 128 flattened (token, group-head) rows of one chunk x one kv head;
+// both tiles share every K/V tile, and their softmax phases alternate with the other tile's MMAs
+// (ping-pong), so the tensor core and the SFU/FMA pipes run concurrently.  12 warps:
+//   warp 0      TMA producer: 128-key K and V tiles = 8 pages (16 x 64 SW128 boxes of the
+//               [kv_blocks*Hkv*16, D] page map) per tile, NS-stage ring, block table read a tile
+//               ahead; also owns the TMEM allocation (512 columns)
+//   warp 1      MMA issuer (one thread):  S_X = Q_X K_j^T  (M=128 N=128 K=D, both K-major)
+//                                          O_X += P_X V_j    (M=128 N=D K=128, P from TMEM, V MN-major)
+//               issue order per key tile j: PV_A(j), S_A(j+1), PV_B(j), [release stage], S_B(j+1),
+//               so S_A(j+1) computes while tile B's softmax runs and vice versa
+//   warps 4-7   softmax of tile A, warps 8-11 tile B: thread = row = TMEM lane; max pass over
+//               the 128 scores (tcgen05.ld), lazy O rescale (only when the max grows by > 2^8,
+//               exact because l and O share the reference max), exp2 pass writing bf16 P over
+//               S in TMEM (tcgen05.st) -- P is the A operand of the PV MMA
+// TMEM: S_A [0,128) S_B [128,256) O_A [256,256+D) O_B [384,384+D); P_X = first 64 cols of S_X.
+// SMEM: Q 2 x 128 x D, NS x (K + V) 128 x D tiles (D=128: 64 KB + 2 x 64 KB).
+#include <cuda_bf16.h>
+
+#include "attention.cuh"
+#include "common.h"
+#include "ptx.cuh"
+
+namespace gllm {
+
+namespace {
+
+constexpr float LOG2E_W = 1.4426950408889634f;
+constexpr int WS_ROWS = 128;  // rows per Q tile (= TMEM lanes)
+constexpr int WS_KT = 128;    // keys per tile
+constexpr int WS_NS = 2;      // K/V ring stages
+constexpr int WS_THREADS = 384;
+constexpr float WS_RESCALE_LOG2 = 8.0f;
+
+template <int D>
+struct WsSmem {
+  static constexpr int ATOMS = D / 64;            // 64-element (128-byte) swizzle atoms along D
+  static constexpr int Q_ATOM = WS_ROWS * 128;    // one atom column of a Q tile
+  static constexpr int KV_ATOM = WS_KT * 128;     // one atom column of a K (or V) tile
+  static constexpr int Q_TILE = ATOMS * Q_ATOM;
+  static constexpr int KV_TILE = ATOMS * KV_ATOM;
+  static constexpr int Q = 0;
+  static constexpr int K = Q + 2 * Q_TILE;
+  static constexpr int V = K + WS_NS * KV_TILE;
+  static constexpr int BAR = V + WS_NS * KV_TILE;
+  // barriers: q_full, kfull[NS], vfull[NS], kvempty[NS], sfull[2], pfull[2], ofull[2]; tmem slot
+  static constexpr int NBAR = 1 + 3 * WS_NS + 6;
+  static constexpr int BYTES = BAR + NBAR * 8 + 16 + 1024;  // + 1024-B alignment slack
+};
+
+__device__ __forceinline__ uint32_t sw128(int rows, int row, int chunk) {
+  return (chunk >> 3) * (rows * 128) + row * 128 + (((chunk & 7) ^ (row & 7)) << 4);
+}
+__device__ __forceinline__ uint64_t desc_mn(uint32_t addr, uint32_t lbo_bytes) {
+  uint64_t d = 0;
+  d |= (uint64_t)((addr & 0x3FFFFu) >> 4);
+  d |= (uint64_t)((lbo_bytes >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)(1024 >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N, bool b_mn_major) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((b_mn_major ? 1u : 0u) << 16) | ((uint32_t)(N >> 3) << 17) |
+         ((uint32_t)(M >> 4) << 24);
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_st_x16(uint32_t taddr, const uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+      "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st_x32(uint32_t taddr, const uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+      "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]), "r"(r[18]),
+      "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]),
+      "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ float ex2(float x) {  // ex2.approx: 2^-inf = +0
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// D[tmem] (+)= A[tmem] . B[smem]
+__device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc, uint32_t idesc,
+                                             uint32_t accumulate) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
+template <int D>
+__global__ void __launch_bounds__(WS_THREADS, 1)
+    prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items,
+                           const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
+  using L = WsSmem<D>;
+  constexpr int ATOMS = L::ATOMS;
+  constexpr int NCH = D / 8;  // 16-byte chunks per Q row
+  constexpr int PAGES = WS_KT / 16;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const uint32_t sbase = ptx::smem_u32(smem);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L::BAR);
+  uint64_t* q_full = bars;
+  uint64_t* kfull = bars + 1;
+  uint64_t* vfull = kfull + WS_NS;
+  uint64_t* kvempty = vfull + WS_NS;
+  uint64_t* sfull = kvempty + WS_NS;
+  uint64_t* pfull = sfull + 2;
+  uint64_t* ofull = pfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + L::NBAR);
+
+  const PrefillItem it = items[blockIdx.x];
+  const int kvh = blockIdx.y;
+  const int G = a.Hq / a.Hkv;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int t0 = a.cu_q[it.seq];
+  const int c = a.cu_q[it.seq + 1] - t0;
+  const int s0 = a.kv_len[it.seq] - c;
+  const int nrows = c * G;
+  const bool hasB = it.row0 + WS_ROWS < nrows;
+  // key tiles each Q tile needs (causal): tile X covers keys 0 .. s0 + (its last row) / G
+  const int nA = (s0 + min(it.row0 + WS_ROWS - 1, nrows - 1) / G) / WS_KT + 1;
+  const int nB = hasB ? (s0 + min(it.row0 + 2 * WS_ROWS - 1, nrows - 1) / G) / WS_KT + 1 : 0;
+  const int n_kt = hasB ? nB : nA;
+  const int nblk_seq = (a.kv_len[it.seq] + 15) / 16;
+  const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
+
+  if (tid == 0) {
+    ptx::mbar_init(q_full, 2 * WS_ROWS);
+    for (int s = 0; s < WS_NS; ++s) {
+      ptx::mbar_init(&kfull[s], 1);
+      ptx::mbar_init(&vfull[s], 1);
+      ptx::mbar_init(&kvempty[s], 1);
+    }
+    for (int x = 0; x < 2; ++x) {
+      ptx::mbar_init(&sfull[x], 1);
+      ptx::mbar_init(&pfull[x], WS_ROWS);
+      ptx::mbar_init(&ofull[x], 1);
+    }
+    ptx::fence_barrier_init();
+    ptx::tma_prefetch(&tmk);
+    ptx::tma_prefetch(&tmv);
+  }
+  if (warp == 0) {
+    ptx::tmem_alloc(tmem_slot, 512);
+    ptx::tmem_relinquish();
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ---------------- TMA producer
+    int bnext = 0;
+    auto read_bt = [&](int j) {  // lanes 0..7: block ids of tile j's pages (past the sequence: its page 0)
+      const int kb = j * PAGES + lane;
+      return (lane < PAGES && j < n_kt) ? __ldg(bt + (kb < nblk_seq ? kb : 0)) : 0;
+    };
+    bnext = read_bt(0);
+#pragma unroll 1
+    for (int j = 0; j < n_kt; ++j) {
+      const int s = j % WS_NS;
+      int bp[PAGES];
+#pragma unroll
+      for (int p = 0; p < PAGES; ++p) bp[p] = __shfl_sync(0xffffffffu, bnext, p);
+      bnext = read_bt(j + 1);
+      if (lane == 0) {
+        if (j >= WS_NS) ptx::mbar_wait(&kvempty[s], (uint32_t)(((j / WS_NS) - 1) & 1));
+        const uint32_t kdst = L::K + s * L::KV_TILE, vdst = L::V + s * L::KV_TILE;
+        ptx::mbar_arrive_expect_tx(&kfull[s], L::KV_TILE);
+#pragma unroll
+        for (int p = 0; p < PAGES; ++p)
+#pragma unroll
+          for (int at = 0; at < ATOMS; ++at)
+            ptx::tma_load_2d(smem + kdst + at * L::KV_ATOM + p * 2048, &tmk, &kfull[s], at * 64,
+                             (bp[p] * a.Hkv + kvh) * 16);
+        ptx::mbar_arrive_expect_tx(&vfull[s], L::KV_TILE);
+#pragma unroll
+        for (int p = 0; p < PAGES; ++p)
+#pragma unroll
+          for (int at = 0; at < ATOMS; ++at)
+            ptx::tma_load_2d(smem + vdst + at * L::KV_ATOM + p * 2048, &tmv, &vfull[s], at * 64,
+                             (bp[p] * a.Hkv + kvh) * 16);
+      }
+      __syncwarp();
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer
+    if (lane == 0) {
+      constexpr uint32_t idesc_s = idesc_bf16(WS_ROWS, WS_KT, false);
+      constexpr uint32_t idesc_o = idesc_bf16(WS_ROWS, D, true);
+      auto issue_s = [&](int x, int j) {
+        const uint32_t qb = sbase + L::Q + x * L::Q_TILE;
+        const uint32_t kb = sbase + L::K + (j % WS_NS) * L::KV_TILE;
+#pragma unroll
+        for (int ks = 0; ks < D / 16; ++ks)
+          ptx::umma_bf16(tmem + x * 128, ptx::umma_desc_sw128(qb + (ks / 4) * L::Q_ATOM + (ks % 4) * 32),
+                         ptx::umma_desc_sw128(kb + (ks / 4) * L::KV_ATOM + (ks % 4) * 32), idesc_s, ks > 0);
+        ptx::umma_commit(&sfull[x]);
+      };
+      auto issue_pv = [&](int x, int j) {
+        const uint32_t vb = sbase + L::V + (j % WS_NS) * L::KV_TILE;
+#pragma unroll
+        for (int kk = 0; kk < WS_KT / 16; ++kk)  // 16 keys = 8 TMEM columns of packed P per step
+          umma_bf16_ta(tmem + 256 + x * 128, tmem + x * 128 + kk * 8, desc_mn(vb + kk * 2048, L::KV_ATOM), idesc_o,
+                       (j > 0 || kk > 0) ? 1u : 0u);
+      };
+      auto wait_k = [&](int j) {
+        ptx::mbar_wait(&kfull[j % WS_NS], (uint32_t)((j / WS_NS) & 1));
+        ptx::tc_fence_after();
+      };
+      ptx::mbar_wait(q_full, 0);
+      ptx::tc_fence_after();
+      wait_k(0);
+      issue_s(0, 0);
+      if (hasB) issue_s(1, 0);
+#pragma unroll 1
+      for (int j = 0; j < n_kt; ++j) {
+        const int s = j % WS_NS;
+        ptx::mbar_wait(&vfull[s], (uint32_t)((j / WS_NS) & 1));
+        bool k_next = false;
+        if (j < nA) {
+          ptx::mbar_wait(&pfull[0], (uint32_t)(j & 1));
+          ptx::tc_fence_after();
+          issue_pv(0, j);
+          if (j + 1 < nA) {
+            wait_k(j + 1);
+            k_next = true;
+            issue_s(0, j + 1);
+          } else {
+            ptx::umma_commit(&ofull[0]);
+          }
+        }
+        if (hasB) {
+          ptx::mbar_wait(&pfull[1], (uint32_t)(j & 1));
+          ptx::tc_fence_after();
+          issue_pv(1, j);
+        }
+        ptx::umma_commit(&kvempty[s]);  // stage s free once every MMA issued so far completes
+        if (hasB) {
+          if (j + 1 < nB) {
+            if (!k_next) wait_k(j + 1);
+            issue_s(1, j + 1);
+          } else {
+            ptx::umma_commit(&ofull[1]);
+          }
+        }
+      }
+    }
+  } else if (warp >= 4) {
+    // ---------------- softmax warpgroups (tile X = 0: warps 4-7, X = 1: warps 8-11)
+    const int x = (warp - 4) >> 2;
+    const int r = (warp & 3) * 32 + lane;  // row of the Q tile = TMEM lane
+    const int rr = it.row0 + x * WS_ROWS + r;
+    const int rrc = min(rr, nrows - 1);
+    // Q row -> SMEM (rows past the chunk repeat the last row; their output is never stored)
+    {
+      const int tok = rrc / G, h = kvh * G + rrc % G;
+      const __nv_bfloat16* src = a.q + (size_t)(t0 + tok) * a.q_stride + (size_t)h * D;
+      const uint32_t qb = sbase + L::Q + x * L::Q_TILE;
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch) ptx::cp_async16(qb + sw128(WS_ROWS, r, ch), src + ch * 8, true);
+      ptx::cp_async_commit();
+      ptx::cp_async_wait<0>();
+      fence_proxy_async_smem();
+      ptx::mbar_arrive(q_full);
+    }
+    const int nx = x == 0 ? nA : nB;
+    const int pos = s0 + rrc / G;  // this row's causal limit (keys 0..pos)
+    const float sl2 = LOG2E_W * rsqrtf((float)D);
+    const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
+    const uint32_t t_s = tmem + lane_off + x * 128;
+    const uint32_t t_o = tmem + lane_off + 256 + x * 128;
+    float m_ref = -INFINITY, l = 0.f;
+#pragma unroll 1
+    for (int j = 0; j < nx; ++j) {
+      ptx::mbar_wait(&sfull[x], (uint32_t)(j & 1));
+      ptx::tc_fence_after();
+      const int kbase = j * WS_KT;
+      const bool diag = kbase + WS_KT - 1 > pos;  // keys past this row's position in this tile
+      // pass 1: row max of the raw scores
+      float mx;
+      {
+        float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int h2 = 0; h2 < 2; ++h2) {
+          uint32_t r0[32], r1[32];
+          ptx::tmem_ld_32x32b_x32(t_s + h2 * 64, r0);
+          ptx::tmem_ld_32x32b_x32(t_s + h2 * 64 + 32, r1);
+          ptx::tmem_ld_wait();
+          if (diag) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+              if (kbase + h2 * 64 + i > pos) r0[i] = __float_as_uint(-INFINITY);
+              if (kbase + h2 * 64 + 32 + i > pos) r1[i] = __float_as_uint(-INFINITY);
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(r0[i]));
+            m4[(i + 2) & 3] = fmaxf(m4[(i + 2) & 3], __uint_as_float(r1[i]));
+          }
+        }
+        mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * sl2;
+      }
+      const bool mine = mx > m_ref + WS_RESCALE_LOG2;
+      const float corr = mine ? ex2(m_ref - mx) : 1.f;
+      if (mine) {
+        l *= corr;
+        m_ref = mx;
+      }
+      // O_X holds PV_X(0..j-1), complete: S_X(j) was committed after PV_X(j-1)
+      if (j > 0 && __any_sync(0xffffffffu, mine)) {
+#pragma unroll 1
+        for (int cb = 0; cb < D / 32; ++cb) {
+          uint32_t orr[32];
+          ptx::tmem_ld_32x32b_x32(t_o + cb * 32, orr);
+          ptx::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) orr[i] = __float_as_uint(__uint_as_float(orr[i]) * corr);
+          tmem_st_x32(t_o + cb * 32, orr);
+        }
+      }
+      // pass 2: P = exp2(s * scale - m) as bf16 pairs over the consumed S columns
+      float la = 0.f, lb = 0.f;
+#pragma unroll
+      for (int cq = 0; cq < WS_KT / 32; ++cq) {
+        uint32_t sr[32];
+        ptx::tmem_ld_32x32b_x32(t_s + cq * 32, sr);
+        ptx::tmem_ld_wait();
+        uint32_t pw[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          float p0 = ex2(fmaf(__uint_as_float(sr[2 * i]), sl2, -m_ref));
+          float p1 = ex2(fmaf(__uint_as_float(sr[2 * i + 1]), sl2, -m_ref));
+          if (diag) {
+            if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
+            if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
+          }
+          la += p0;
+          lb += p1;
+          pw[i] = ptx::pack_bf16(p0, p1);
+        }
+        tmem_st_x16(t_s + cq * 16, pw);
+      }
+      l += la + lb;
+      tmem_st_wait();
+      ptx::tc_fence_before();
+      ptx::mbar_arrive(&pfull[x]);
+    }
+    if (nx > 0) {
+      ptx::mbar_wait(&ofull[x], 0);
+      ptx::tc_fence_after();
+      const bool valid = rr < nrows;
+      const float inv = 1.f / l;
+      __nv_bfloat16* dst = a.out + (size_t)(t0 + rrc / G) * a.Hq * D + (size_t)(kvh * G + rrc % G) * D;
+#pragma unroll
+      for (int cb = 0; cb < D / 32; ++cb) {
+        uint32_t orr[32];
+        ptx::tmem_ld_32x32b_x32(t_o + cb * 32, orr);
+        ptx::tmem_ld_wait();
+        if (valid) {
+          uint4* d4 = reinterpret_cast<uint4*>(dst + cb * 32);
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            uint4 w;
+            w.x = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 0]) * inv, __uint_as_float(orr[q * 8 + 1]) * inv);
+            w.y = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 2]) * inv, __uint_as_float(orr[q * 8 + 3]) * inv);
+            w.z = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 4]) * inv, __uint_as_float(orr[q * 8 + 5]) * inv);
+            w.w = ptx::pack_bf16(__uint_as_float(orr[q * 8 + 6]) * inv, __uint_as_float(orr[q * 8 + 7]) * inv);
+            d4[q] = w;
+          }
+        }
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, 512);
+  }
+}
+
+template <int D>
+int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
+              int n_items, cudaStream_t s) {
+  constexpr int bytes = WsSmem<D>::BYTES;
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(prefill_attn_ws_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    set = true;
+  }
+  prefill_attn_ws_kernel<D><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
+  return GLLM_OK;
+}
+
+}  // namespace
+
+int prefill_ws_rows_per_item() { return 2 * WS_ROWS; }
+
+int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
+                                const PrefillItem* items, int n_items, cudaStream_t s) {
+  if (n_items <= 0) return GLLM_OK;
+  if (a.bs != 16) return set_error(GLLM_EINVAL, "prefill attention (ws): block size %d unsupported", a.bs);
+  if (a.D == 128)
+    launch_ws<128>(a, tmk, tmv, items, n_items, s);
+  else if (a.D == 64)
+    launch_ws<64>(a, tmk, tmv, items, n_items, s);
+  else
+    return set_error(GLLM_EINVAL, "prefill attention (ws): head_dim %d unsupported", a.D);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GLLM_OK
+                          : set_error(GLLM_ECUDA, "prefill attention (ws) launch: %s", cudaGetErrorString(e));
+}
+
+}  // namespace gllm

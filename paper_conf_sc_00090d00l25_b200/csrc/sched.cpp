@@ -150,6 +150,23 @@ int32_t throttle_prefill(const gllm_sched_cfg& c, int64_t wp, int64_t free_block
   return (int32_t)std::min(p, wp);                       // R11: cannot exceed #WP
 }
 
+// R21 (policy 4, L354): token-equivalent cost of a chunk of c tokens at offset s -- its linear
+// work (c) plus its causal attention pairs c*s + c(c+1)/2 in units of attn_pairs_per_token.
+int64_t chunk_cost(int64_t s, int64_t c, int64_t a) { return c + (c * s + c * (c + 1) / 2) / a; }
+
+// largest c in [0, cmax] with chunk_cost(s, c) <= budget (chunk_cost is increasing in c)
+int64_t max_chunk_within(int64_t s, int64_t cmax, int64_t budget, int64_t a) {
+  int64_t lo = 0, hi = std::min(cmax, budget);  // cost >= c
+  while (lo < hi) {
+    const int64_t mid = lo + (hi - lo + 1) / 2;
+    if (chunk_cost(s, mid, a) <= budget)
+      lo = mid;
+    else
+      hi = mid - 1;
+  }
+  return lo;
+}
+
 int32_t throttle_decode(const gllm_sched_cfg& c, int64_t rd) {
   return (int32_t)ceil_div(rd, c.pp_depth);  // Eq.4 with ceil (R6)
 }
@@ -161,8 +178,10 @@ int check_cfg(const gllm_sched_cfg* c) {
     return gllm::set_error(GLLM_EINVAL, "scheduler cfg: non-positive size");
   if (c->kvthresh_den < 1 || c->kvthresh_num < 0 || c->kvthresh_num >= c->kvthresh_den)
     return gllm::set_error(GLLM_EINVAL, "scheduler cfg: KV_thresh must be in [0,1)");
-  if (c->policy < GLLM_POLICY_THROTTLE || c->policy > GLLM_POLICY_NO_UT)
+  if (c->policy < GLLM_POLICY_THROTTLE || c->policy > GLLM_POLICY_CTX)
     return gllm::set_error(GLLM_EINVAL, "unknown policy %d", c->policy);
+  if (c->policy == GLLM_POLICY_CTX && c->attn_pairs_per_token < 1)
+    return gllm::set_error(GLLM_EINVAL, "context-aware policy: attn_pairs_per_token must be >= 1");
   return GLLM_OK;
 }
 
@@ -393,31 +412,41 @@ int gllm_build_batch(gllm_sched* s, gllm_batch_desc* out) {
   else
     p_cnt = throttle_prefill(cfg, wp, free0);
   // 6. prefill selection, FCFS with CPP (R13)
-  int64_t p_left = p_cnt;
+  int64_t p_left = p_cnt, p_tokens = 0;
+  const bool ctx = cfg.policy == GLLM_POLICY_CTX;
   for (size_t wi = 0; wi < s->waitq.size() && p_left > 0; ++wi) {
     Req* r = s->waitq[wi];
     if (!r->waiting()) continue;  // stale entry
     const bool fresh = r->blocks.empty() && r->sched_prompt == 0;
     if (fresh && s->running >= cfg.max_seqs) continue;
     const int64_t remaining = r->prefill_len - r->sched_prompt;
-    const int64_t want = std::min(remaining, p_left);
     const int64_t capacity = ((int64_t)r->blocks.size() + (int64_t)s->free_pool.size()) * bs - r->sched_prompt;
-    const int64_t c = std::min(want, capacity);
-    if (c <= 0) break;
+    int64_t c, cost;
+    if (ctx) {  // R21: the chunk's token-equivalent cost (linear + causal attention) fits the budget
+      c = max_chunk_within(r->sched_prompt, std::min(remaining, capacity), p_left, cfg.attn_pairs_per_token);
+      if (c == 0 && b.chunks.empty() && capacity > 0) c = 1;  // progress: one token at least
+      if (c <= 0) break;
+      cost = chunk_cost(r->sched_prompt, c, cfg.attn_pairs_per_token);
+    } else {
+      c = std::min(std::min(remaining, p_left), capacity);
+      if (c <= 0) break;
+      cost = c;
+    }
     const int64_t need = ceil_div(r->sched_prompt + c, bs) - (int64_t)r->blocks.size();
     for (int64_t j = 0; j < need; ++j) s->alloc(r, &allocs);
     b.chunks.push_back({r, r->sched_prompt, (int32_t)c, r->sched_prompt + c == r->prefill_len});
     r->sched_prompt += (int32_t)c;
     s->wp -= c;
     if (!r->waiting()) s->waitq_stale += 1;
-    p_left -= c;
-    if (c < want) break;
+    p_left = std::max<int64_t>(p_left - cost, 0);
+    p_tokens += c;
+    if (c < remaining) break;  // cut by the budget (then p_left is spent) or by KV capacity (R13)
   }
   // 7. layout (R15): prefill chunks, then decodes
   b.P = p_cnt;
   b.D = d_cnt;
   const size_t S = b.chunks.size() + b.decodes.size();
-  const size_t T = (size_t)(p_cnt - p_left) + b.decodes.size();
+  const size_t T = (size_t)p_tokens + b.decodes.size();
   b.token_ids.reserve(T);
   b.positions.reserve(T);
   b.slots.reserve(T);

@@ -126,6 +126,7 @@ struct gllm_stage {
   float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
   bool fused_norm = true;
   bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
+  bool prefill_ws = false;                 // GLLM_PREFILL_WS=1: warp-specialised tcgen05 prefill (A/B)
   bool attn_overlap = true;                // GLLM_ATTN_SERIAL=1: prefill and decode attention in series (A/B)
   bool decode_v1 = false;                  // GLLM_DECODE_V1=1: the per-CTA cp.async decode kernel (A/B)
   int* dec_ctr = nullptr;                  // persistent decode kernel: work counter + done counter
@@ -149,6 +150,7 @@ struct gllm_stage {
   bool timing_pending = false;
 
   bool is_first() const { return lb == 0; }
+  bool use_prefill_ws() const { return prefill_ws && !prefill_mma_sync; }
   bool is_last() const { return le == cfg.n_layers; }
   int qd() const { return cfg.n_heads * cfg.head_dim; }
   int kd() const { return cfg.n_kv_heads * cfg.head_dim; }
@@ -412,6 +414,8 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
   if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
   if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
+  if (const char* e = std::getenv("GLLM_PREFILL_WS")) st->prefill_ws = e[0] == '1';
+  if (block_size != 16) st->prefill_ws = false;
   if (const char* e = std::getenv("GLLM_ATTN_SERIAL")) st->attn_overlap = e[0] != '1';
   if (const char* e = std::getenv("GLLM_DECODE_V1")) st->decode_v1 = e[0] == '1';
   if (const char* e = std::getenv("GLLM_DECODE_WARPS")) gllm::set_decode_warps(std::atoi(e));
@@ -494,7 +498,7 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   for (int i = 0; i < NP; ++i) {
     const int n = d->cu_q[i + 1] - d->cu_q[i];
     const int rows = n * G, s0 = d->kv_len[i] - n;
-    const int rpi = gllm::prefill_rows_per_item();
+    const int rpi = st->use_prefill_ws() ? gllm::prefill_ws_rows_per_item() : gllm::prefill_rows_per_item();
     for (int r0 = 0; r0 < rows; r0 += rpi) {
       const int last = std::min(r0 + rpi - 1, rows - 1) / G;
       pcost.push_back({(s0 + last + 64) / 64, (int)pitems.size()});
@@ -721,8 +725,11 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       }
       {
         Prof p(st, ps, C_PREFILL);
-        RC(st->prefill_mma_sync ? gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps)
-                                : gllm::launch_prefill_attention_tc(aa, d_pi, P.n_pi, ps));
+        if (st->use_prefill_ws())
+          RC(gllm::launch_prefill_attention_ws(aa, w.tm_kc, w.tm_vc, d_pi, P.n_pi, ps));
+        else
+          RC(st->prefill_mma_sync ? gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps)
+                                  : gllm::launch_prefill_attention_tc(aa, d_pi, P.n_pi, ps));
       }
       if (overlap) CK(cudaEventRecord(st->ev_join, ps));
       st->last_launches += 1;

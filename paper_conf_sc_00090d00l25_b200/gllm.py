@@ -38,7 +38,8 @@ class ModelCfg(C.Structure):
 
 class SchedCfg(C.Structure):
     _fields_ = [(n, C.c_int32) for n in ("iterp", "maxp", "minp", "kvthresh_num", "kvthresh_den", "pp_depth",
-                                           "num_blocks", "block_size", "max_seqs", "policy", "token_budget")]
+                                           "num_blocks", "block_size", "max_seqs", "policy", "token_budget",
+                                           "attn_pairs_per_token")]
 
 
 _P32 = C.POINTER(C.c_int32)

@@ -147,6 +147,20 @@ def test_full_width_other_shapes_stage_local(cfg_name, n_req, ticks, kvb):
     assert errs.max() <= TOL_HIDDEN, errs.max()
 
 
+def test_c3_long_prompt_chunks_stage_local():
+    # Qwen2.5-32B shapes (GQA group 5, bias): the C3 long-prompt stream at PP=1 prefills ~4k-token
+    # prompts in Token-Throttled chunks, so later chunks sit at offsets of thousands of keys (many
+    # 128-key tiles, both Q tiles of the warp-specialised prefill kernel, causal tails that end in
+    # different key tiles for the two tiles)
+    m = MODELS["C3"].with_layers(4)
+    st = make_stream("C3", m.vocab, n=4)
+    cfg = SCHED["C3"].with_(num_blocks=3000, pp_depth=1)
+    # ticks 3-5: chunks of 1563, 1977 and 1751 tokens at offsets 0, 1563 and 3540
+    n, errs, _ = _run_pair(m, cfg, st, lb=1, le=2, max_ticks=6, kv_blocks=3000, check_kv=False)
+    assert n == 5291
+    assert errs.max() <= TOL_HIDDEN, errs.max()
+
+
 def test_c1_last_stage_full_vocab_lm_head():
     # last stage of a 2-layer Llama-3-8B-shaped model: layer 1 + final norm + 128256-wide LM head with the
     # fused argmax epilogue (501 N tiles) -> greedy ids tolerance-aware vs the oracle's fp32 logits

@@ -263,3 +263,58 @@ def test_decode_fairness_once_per_pp_ticks():
             if rid in last:
                 assert b.tick - last[rid] >= cfg.pp_depth
             last[rid] = b.tick
+
+
+# ---- R21: context-aware Token Throttling (policy 4; PAPER.md L354 future work) ----------------
+
+def test_chunk_cost_closed_form_and_examples():
+    from oracle.scheduler import chunk_cost
+    # pairs of a chunk of c tokens at offset s = c*s + c(c+1)/2 (query s+j sees keys 0..s+j)
+    for s0 in (0, 1, 17, 1000):
+        for c in (0, 1, 2, 15, 64):
+            for a in (1, 7, 100, 10 ** 9):
+                assert chunk_cost(s0, c, a) == c + (c * s0 + c * (c + 1) // 2) // a
+    # hand-worked (R21): a = 100
+    assert chunk_cost(0, 164, 100) == 164 + 13530 // 100 == 299
+    assert chunk_cost(0, 165, 100) == 301
+    assert chunk_cost(164, 47, 100) == 47 + (7708 + 1128) // 100 == 135
+    assert chunk_cost(164, 48, 100) == 138
+
+
+def test_ctx_policy_hand_worked_trace():
+    # one 300-token prompt, #T = 1, PP = 1, a = 100 pairs/token; Eq.3 gives the budget P = WP each tick
+    cfg = SchedParams(iterp=1, maxp=2048, minp=1, pp_depth=1, num_blocks=64, policy=4, attn_pairs_per_token=100)
+    st = Stream("ctx", [Request(0, 0, 300, 2, np.zeros(301, np.int32))])
+    s, bs = run(cfg, st)
+    # tick 0: budget 300 -> c = 164 (cost 299; 165 would cost 301)
+    # tick 1: budget 136 at offset 164 -> c = 47 (cost 135; 48 would cost 138)
+    assert [(b.P, [(c[1], c[2]) for c in b.chunks]) for b in bs[:2]] == [(300, [(0, 164)]), (136, [(164, 47)])]
+    # every tick takes the longest chunk whose cost fits its budget; when not even one token fits,
+    # one token is taken anyway (progress rule of R21)
+    from oracle.scheduler import chunk_cost
+    for b in bs:
+        for (_rid, s0, c, _d) in b.chunks:
+            assert chunk_cost(s0, c, 100) <= b.P or c == 1
+            assert c == 300 - s0 or chunk_cost(s0, c + 1, 100) > b.P
+    assert sum(c[2] for b in bs for c in b.chunks) == 300
+
+
+def test_ctx_policy_reduces_to_token_throttling_for_large_a():
+    # a -> infinity: every chunk costs its token count, so the trace equals policy 0 byte for byte
+    from oracle.scheduler import trace_bytes
+    st = make_stream("C1", 1024, n=150)
+    base = SchedParams(pp_depth=2, num_blocks=3000)
+    s0 = Scheduler(base, st.requests)
+    s4 = Scheduler(base.with_(policy=4, attn_pairs_per_token=2 ** 31 - 1), st.requests)
+    while not s0.done():
+        assert trace_bytes(s0.build_batch()) == trace_bytes(s4.build_batch())
+    assert s4.done()
+
+
+def test_ctx_policy_invariants_and_long_prompts():
+    # C3-like long prompts: chunks deep into a prompt get fewer tokens than Eq.3's count
+    st = make_stream("C3", 1024, n=12)
+    cfg = SCHED["C3"].with_(num_blocks=6000, pp_depth=4, policy=4, attn_pairs_per_token=4096)
+    s, total_p = _check_invariants(cfg, st, max_ticks=None)
+    assert s.done() and total_p == sum(r.prompt_len for r in st.requests)
+    assert sorted(s.free) == list(range(cfg.num_blocks))

@@ -124,3 +124,16 @@ def test_library_scheduler_overhead_vs_paper():
     us = (time.perf_counter() - t0) / k * 1e6
     print(f"build_batch: {us:.1f} us/tick (paper: 45 us)")
     assert us < 2000
+
+
+def test_ctx_policy_identical():
+    # R21 (policy 4): the library's binary search over chunk lengths == the oracle's linear scan,
+    # byte for byte, on long-prompt (C3) and ShareGPT-like (C1) streams, incl. a KV-pressured run
+    _diff_run(SCHED["C3"].with_(num_blocks=6000, pp_depth=4, policy=4, attn_pairs_per_token=4096),
+              make_stream("C3", 1000, n=30), max_ticks=400)
+    _diff_run(SchedParams(pp_depth=2, num_blocks=3000, policy=4, attn_pairs_per_token=300),
+              make_stream("C1", 1000, n=300))
+    _diff_run(SchedParams(pp_depth=2, num_blocks=400, policy=4, attn_pairs_per_token=50),
+              make_stream("C1", 1000, n=100))
+    with pytest.raises(gllm.GllmError):
+        gllm.Sched(SchedParams(num_blocks=100, policy=4, attn_pairs_per_token=0))

@@ -6,7 +6,7 @@ mkdir -p $OUT
 for rep in ${REPS:-1}; do
 for v in ${AB:-base}; do
   envs=""; [ "$v" != "base" ] && envs="${v//,/ }"
-  env $envs timeout 900 python bench.py --config ${CONFIG:-C1} --steps ${STEPS:-10} --warmup 5 --no-cpu-baseline > $OUT/$v.json 2> $OUT/$v.err
+  env $envs timeout 900 python bench.py --config ${CONFIG:-C1} ${EXTRA} --steps ${STEPS:-10} --warmup 5 --no-cpu-baseline > $OUT/$v.json 2> $OUT/$v.err
   python - "$v" "$OUT/$v.json" <<'PY'
 import json, sys
 try:

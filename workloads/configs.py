@@ -50,8 +50,9 @@ class SchedParams:
     num_blocks: int = 64
     block_size: int = 16
     max_seqs: int = 1024      # L575
-    policy: int = 0           # 0 = Token Throttling; 1 = Sarathi-Serve; 2 = w/o WT; 3 = w/o UT (§4.5)
+    policy: int = 0           # 0 = Token Throttling; 1 = Sarathi-Serve; 2 = w/o WT; 3 = w/o UT (§4.5); 4 = R21
     token_budget: int = 2048  # Sarathi only (L248)
+    attn_pairs_per_token: int = 0  # policy 4 (context-aware throttling, R21, L354) only
 
     def with_(self, **kw) -> "SchedParams":
         return replace(self, **kw)

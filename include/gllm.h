@@ -227,7 +227,9 @@ GLLM_API int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n);
 GLLM_API int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed);
 
 /* Timing of the forwards since the previous call, from CUDA events recorded on each forward's own
- * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).
+ * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).  on = 2 also runs the
+ * prefill and decode attention kernels in series instead of on two concurrent streams, so that each
+ * one's events bracket that kernel alone (an attribution pass; the forward's results are the same).
  * out[n] receives milliseconds per category (synchronises on the events):
  *   [0] whole forward  [1] QKV GEMM  [2] O GEMM  [3] gate_up GEMM  [4] down GEMM
  *   [5] prefill attention  [6] decode attention  [7] RoPE+KV append  [8] RMSNorm

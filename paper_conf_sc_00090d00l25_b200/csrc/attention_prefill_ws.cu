@@ -22,6 +22,8 @@
 // SMEM: Q 2 x 128 x D, NS x (K + V) 128 x D tiles (D=128: 64 KB + 2 x 64 KB).
 #include <cuda_bf16.h>
 
+#include <cstdlib>
+
 #include "attention.cuh"
 #include "common.h"
 #include "ptx.cuh"
@@ -96,6 +98,19 @@ __device__ __forceinline__ float ex2(float x) {  // ex2.approx: 2^-inf = +0
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
+// 2^x on the FMA pipe (x <= ~8): round-to-nearest split x = j + f, f in [-1/2, 1/2], cubic for
+// 2^f (relative error < 1e-3, below bf16's 2^-8 rounding of P), j added to the exponent bits.
+// Takes a share of the exponentials off the 16/clk/SM MUFU unit (FA4's trick).
+__device__ __forceinline__ float exp2_fma(float x) {
+  x = fmaxf(x, -126.f);
+  const float t = x + 12582912.f;  // 1.5 * 2^23: the integer part lands in the low mantissa bits
+  const float f = x - (t - 12582912.f);
+  float p = fmaf(f, 0.0555041087f, 0.240226507f);
+  p = fmaf(p, f, 0.693147181f);
+  p = fmaf(p, f, 1.0f);
+  return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
+}
+
 // D[tmem] (+)= A[tmem] . B[smem]
 __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc, uint32_t idesc,
                                              uint32_t accumulate) {
@@ -109,7 +124,7 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
-template <int D>
+template <int D, bool EMU>
 __global__ void __launch_bounds__(WS_THREADS, 1)
     prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items,
                            const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
@@ -353,8 +368,11 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
         uint32_t pw[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
-          float p0 = ex2(fmaf(__uint_as_float(sr[2 * i]), sl2, -m_ref));
-          float p1 = ex2(fmaf(__uint_as_float(sr[2 * i + 1]), sl2, -m_ref));
+          const float x0 = fmaf(__uint_as_float(sr[2 * i]), sl2, -m_ref);
+          const float x1 = fmaf(__uint_as_float(sr[2 * i + 1]), sl2, -m_ref);
+          // EMU: one pair in four on the FMA pipe (MUFU and FMA pipes then finish together)
+          float p0 = (EMU && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
+          float p1 = (EMU && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
           if (diag) {
             if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
             if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
@@ -404,16 +422,21 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   }
 }
 
-template <int D>
+const bool g_prefill_emu = [] {
+  const char* e = std::getenv("GLLM_PREFILL_EMU");
+  return e && e[0] == '1';
+}();
+
+template <int D, bool EMU>
 int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
               int n_items, cudaStream_t s) {
   constexpr int bytes = WsSmem<D>::BYTES;
   static bool set = false;
   if (!set) {
-    cudaFuncSetAttribute(prefill_attn_ws_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(prefill_attn_ws_kernel<D, EMU>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  prefill_attn_ws_kernel<D><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
+  prefill_attn_ws_kernel<D, EMU><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
   return GLLM_OK;
 }
 
@@ -426,9 +449,11 @@ int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const
   if (n_items <= 0) return GLLM_OK;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "prefill attention (ws): block size %d unsupported", a.bs);
   if (a.D == 128)
-    launch_ws<128>(a, tmk, tmv, items, n_items, s);
+    g_prefill_emu ? launch_ws<128, true>(a, tmk, tmv, items, n_items, s)
+                  : launch_ws<128, false>(a, tmk, tmv, items, n_items, s);
   else if (a.D == 64)
-    launch_ws<64>(a, tmk, tmv, items, n_items, s);
+    g_prefill_emu ? launch_ws<64, true>(a, tmk, tmv, items, n_items, s)
+                  : launch_ws<64, false>(a, tmk, tmv, items, n_items, s);
   else
     return set_error(GLLM_EINVAL, "prefill attention (ws): head_dim %d unsupported", a.D);
   cudaError_t e = cudaGetLastError();

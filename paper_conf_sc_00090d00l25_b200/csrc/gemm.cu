@@ -123,15 +123,19 @@ __device__ __forceinline__ void tmem_dealloc_cg(uint32_t taddr, uint32_t ncols) 
 
 // Job iterator shared by the three warp roles (each role walks the same sequence).  `unit` is
 // the CTA (CG=1) or the cluster (CG=2) index, `nunits` their count.
+// mode 0: whole tiles round robin.  mode 1: stream-K over all (tile, k-block) units.  mode 2
+// (hybrid): whole tiles for the first dp_tiles = full waves, then stream-K over the tail tiles'
+// k-blocks, so a last wave that would be mostly empty is spread over every unit.
 struct Jobs {
-  int mode, ntiles, nk, per, total, unit, nunits;
+  int mode, ntiles, nk, per, total, unit, nunits, dp_tiles;
   int it, u, u1;
   __device__ void init(const GemmArgs& p, int unit_, int nunits_, int num_m) {
     mode = p.streamk;
     ntiles = num_m * p.num_n_tiles;
     nk = p.K / GEMM_BK;
     per = p.units_per_cta;
-    total = ntiles * nk;
+    dp_tiles = mode == 2 ? p.dp_tiles : 0;
+    total = (ntiles - dp_tiles) * nk;
     unit = unit_;
     nunits = nunits_;
     it = 0;
@@ -139,18 +143,19 @@ struct Jobs {
     u1 = min(total, u + per);
   }
   __device__ bool next(int& tile, int& kb0, int& kb1) {
-    if (mode == 0) {
+    if (mode == 0 || (mode == 2 && unit + it * nunits < dp_tiles)) {
       tile = unit + it * nunits;
       ++it;
       kb0 = 0;
       kb1 = nk;
-      return tile < ntiles;
+      return tile < (mode == 0 ? ntiles : dp_tiles);
     }
     if (u >= u1) return false;
     tile = u / nk;
     kb0 = u - tile * nk;
     kb1 = min(nk, kb0 + (u1 - u));
     u += kb1 - kb0;
+    tile += dp_tiles;
     return true;
   }
 };
@@ -217,20 +222,25 @@ __device__ __forceinline__ float row_scale(const GemmArgs& p, int row) {
 }
 
 // One warp's 32 rows of one 256-column accumulator tile: wait for the MMAs (tfull), drain TMEM,
-// apply the fused epilogue.  `partial`: stream-K segment, combine atomically.
+// apply the fused epilogue.  `partial`: stream-K segment, combine atomically.  Non-additive
+// epilogues combine partial segments in the fp32 workspace ws: with tile counters (p.tile_ctr)
+// the last of the tile's `contrib` segments to arrive reads the sum back (and re-zeroes ws and
+// the counter) and runs the epilogue itself -- no memset and no finish pass.
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
 template <int EPI>
 __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
-                                              uint64_t* tfull_bar, uint32_t parity, float* stg) {
+                                              uint64_t* tfull_bar, uint32_t parity, float* stg, int tile,
+                                              int contrib, int* fix_flag) {
   const bool row_ok = row < p.M;
   const float rs = (EPI == EPI_ADD_F32 || EPI == EPI_ARGMAX) ? 1.0f : row_scale(p, row);
-  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && !partial && p.ws == nullptr) p.zero_rows[row] = 0.f;
   uint32_t r[32];
   auto wait_acc = [&]() {
     ptx::mbar_wait(tfull_bar, parity);
     ptx::tc_fence_after();
   };
-  if (p.ws != nullptr) {
-    // workspace mode (stream-K for non-additive epilogues): every segment adds into ws
+  bool from_ws = false;  // this CTA finishes a stream-K tile from the workspace sums
+  if (p.ws != nullptr && (partial || p.tile_ctr == nullptr)) {  // (legacy mode: every segment via ws)
     wait_acc();
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
@@ -239,13 +249,56 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       const int col0 = n_blk * GEMM_BN + c * 32;
       if (row_ok && col0 < p.N) atomic_add_f32x32(p.ws + (size_t)row * p.N + col0, r);
     }
-  } else if constexpr (EPI == EPI_STORE_BF16) {
-    wait_acc();
+    if (p.tile_ctr == nullptr) return;  // gemm_finish_kernel applies the epilogue
+    __threadfence();                     // this thread's reductions before the tile count
+    epi_bar();
+    if (threadIdx.x == 128) *fix_flag = atomicAdd(p.tile_ctr + tile, 1) == contrib - 1;
+    epi_bar();
+    const bool last = *fix_flag != 0;
+    epi_bar();                           // every warp has read the flag before it is reused
+    if (!last) return;
+    __threadfence();
+    if (threadIdx.x == 128) p.tile_ctr[tile] = 0;
+    from_ws = true;
+  }
+  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && (!partial || from_ws)) p.zero_rows[row] = 0.f;
+  float* wrow = p.ws + (size_t)(row_ok ? row : 0) * p.N + n_blk * GEMM_BN;
+  // accumulator columns [col, col + 32) of this tile's row: from TMEM or (finisher) from ws,
+  // re-zeroing ws behind the read
+  auto ld = [&](int col, uint32_t(&v)[32]) {
+    if (!from_ws) {
+      ptx::tmem_ld_32x32b_x32(tbase + col, v);
+      return;
+    }
+    if (row_ok && n_blk * GEMM_BN + col < p.N) {
+      float4* src = reinterpret_cast<float4*>(wrow + col);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const float4 x = __ldcg(src + q);
+        v[4 * q] = __float_as_uint(x.x);
+        v[4 * q + 1] = __float_as_uint(x.y);
+        v[4 * q + 2] = __float_as_uint(x.z);
+        v[4 * q + 3] = __float_as_uint(x.w);
+        __stcg(src + q, make_float4(0.f, 0.f, 0.f, 0.f));
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < 32; ++q) v[q] = 0u;
+    }
+  };
+  auto ld_wait = [&]() {
+    if (!from_ws) ptx::tmem_ld_wait();
+  };
+  auto wait_src = [&]() {
+    if (!from_ws) wait_acc();
+  };
+  if constexpr (EPI == EPI_STORE_BF16) {
+    wait_src();
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
-      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-      ptx::tmem_ld_wait();
+      ld(c * 32, r);
+      ld_wait();
       const int col0 = n_blk * GEMM_BN + c * 32;
       if (row_ok && col0 < p.N) {
         float v[32];
@@ -332,14 +385,14 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       }
     }
   } else if constexpr (EPI == EPI_SILU_MUL) {
-    wait_acc();
+    wait_src();
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
     uint32_t u[32];
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 64; ++c) {
-      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);                // gate columns
-      ptx::tmem_ld_32x32b_x32(tbase + GEMM_BN / 2 + c * 32, u);  // up columns
-      ptx::tmem_ld_wait();
+      ld(c * 32, r);                // gate columns
+      ld(GEMM_BN / 2 + c * 32, u);  // up columns
+      ld_wait();
       const int col0 = n_blk * (GEMM_BN / 2) + c * 32;
       if (row_ok && col0 < p.N / 2) {
         float h[32];
@@ -355,14 +408,14 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     const int slot = row_ok ? __ldg(p.slots + row) : 0;
     const int64_t blk = slot / p.block_size, off = slot % p.block_size;
     uint32_t u[32];
-    wait_acc();
+    wait_src();
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
       const int hpos = c % per_head;
       if (hpos >= per_head / 2) continue;
-      ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-      ptx::tmem_ld_32x32b_x32(tbase + (c + per_head / 2) * 32, u);
-      ptx::tmem_ld_wait();
+      ld(c * 32, r);
+      ld((c + per_head / 2) * 32, u);
+      ld_wait();
       const int col1 = n_blk * GEMM_BN + c * 32;
       if (!row_ok || col1 >= p.N) continue;
       float x1[32], x2[32];
@@ -412,6 +465,7 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(tempty + 2);
+  int* fix_flag = reinterpret_cast<int*>(tmem_ptr + 1);
   float* stg = reinterpret_cast<float*>(sB + C::STAGES * C::B_BYTES + 256);  // epilogue transpose tiles
 
   const int warp = threadIdx.x >> 5;
@@ -529,7 +583,13 @@ __global__ void __launch_bounds__(256, 1)
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
-      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
+      int contrib = 1;
+      if (jobs.mode != 0 && tile >= jobs.dp_tiles) {  // stream-K segments covering this tile
+        const int u0 = (tile - jobs.dp_tiles) * nk;
+        contrib = (u0 + nk - 1) / jobs.per - u0 / jobs.per + 1;
+      }
+      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS,
+                         tile * CG + (int)rank, contrib, fix_flag);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) {
@@ -596,8 +656,13 @@ PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_encode_once;
 
 // Scheduling decision (host).  Returns 1 for stream-K (CG=1 only).
+const bool g_no_sk = [] {  // GLLM_GEMM_NO_SK=1: never stream-K (A/B)
+  const char* e = std::getenv("GLLM_GEMM_NO_SK");
+  return e && e[0] == '1';
+}();
+
 int choose_streamk(int M, int N, int ntiles, int nk, int epi, int num_sms) {
-  if (epi == EPI_ARGMAX || nk < 8) return 0;
+  if (g_no_sk || epi == EPI_ARGMAX || nk < 8) return 0;
   const int waves = (ntiles + num_sms - 1) / num_sms;
   const double eff = (double)ntiles / ((double)waves * num_sms);
   // Measured on B200: with >= one wave of tiles the reductions of partial tiles cost more than
@@ -626,10 +691,32 @@ int choose_cg(int M, int N, int epi, int num_sms) {
   return g_cg1_rest && M < 4096 ? 1 : 2;
 }
 
+// CTA-pair hybrid (Jobs mode 2) for the residual-add epilogue: when the last wave of 256 x 256
+// tiles would be less than ~60% full (e.g. C3's O / down GEMMs at T ~ 900: 80 tiles on 74
+// pairs), the tail tiles' k-blocks are spread over every pair and combined with fp32 vector
+// reductions.  Returns the whole-tile count (0 = no hybrid).  GLLM_GEMM_NO_HYBRID=1 disables it.
+const bool g_no_hybrid = [] {
+  const char* e = std::getenv("GLLM_GEMM_NO_HYBRID");
+  return e && e[0] == '1';
+}();
+// Non-additive epilogues (QKV / SiLU / store) take the hybrid too when their fp32 workspace fits
+// (`ws_ok`): partial tiles then combine in ws and the last segment finishes the tile in-kernel.
+int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms, bool ws_ok) {
+  if (g_no_hybrid || cg != 2 || epi == EPI_ARGMAX || K / GEMM_BK < 8) return 0;
+  const int units = num_sms / 2;
+  const int ntiles = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
+  if (epi != EPI_ADD_F32 && (!ws_ok || (size_t)M * N > GEMM_WS_ELEMS || ntiles * 2 > GEMM_MAX_SK_TILES)) return 0;
+  const int tail = ntiles % units;
+  if (ntiles < units || tail == 0 || tail * 10 >= units * 8) return 0;
+  return ntiles - tail;
+}
+
 }  // namespace
 
 bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms) {
-  if (M <= 0 || choose_cg(M, N, epi, num_sms) == 2) return false;
+  if (M <= 0) return false;
+  const int cg = choose_cg(M, N, epi, num_sms);
+  if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms, false) > 0;
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
   return choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms) != 0;
 }
@@ -685,15 +772,17 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
   const int num_m = (args.M + C::TILE_M - 1) / C::TILE_M;
   const int ntiles = num_m * args.num_n_tiles;
   int grid;
-  if (args.streamk) {
+  if (args.streamk == 1) {
     const int total = ntiles * (args.K / GEMM_BK);
     grid = (total + args.units_per_cta - 1) / args.units_per_cta;
+  } else if (args.streamk == 2) {
+    grid = (num_sms / CG) * CG;
   } else {
     const int units = num_sms / CG;
     grid = (ntiles < units ? ntiles : units) * CG;
   }
   if (grid <= 0) return GLLM_OK;
-  if (args.ws) {
+  if (args.ws && !args.tile_ctr) {
     cudaError_t e = cudaMemsetAsync(args.ws, 0, (size_t)args.M * args.N * sizeof(float), stream);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm workspace memset: %s", cudaGetErrorString(e));
   }
@@ -715,7 +804,7 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
     cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_tc_kernel<EPI, 2>, a, b, args);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (2-CTA) launch: %s", cudaGetErrorString(e));
   }
-  if (args.ws) {
+  if (args.ws && !args.tile_ctr) {
     const int chunks = args.M * ((EPI == EPI_SILU_MUL) ? args.N / 64 : args.N / 32);
     gemm_finish_kernel<EPI><<<(chunks + 255) / 256, 256, 0, stream>>>(args);
   }
@@ -742,10 +831,24 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   const int ntiles = args.num_m_tiles * args.num_n_tiles, nk = args.K / GEMM_BK;
   args.streamk = cg == 1 ? choose_streamk(args.M, args.N, ntiles, nk, epi, num_sms) : 0;
   args.units_per_cta = args.streamk ? (ntiles * nk + num_sms - 1) / num_sms : 0;
+  args.dp_tiles = 0;
+  bool hybrid = false;
+  if (cg == 2 && !args.xb_out && !args.ss_out) {  // partial tiles cannot produce the next norm's inputs
+    const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms, args0.ws && args0.tile_ctr);
+    if (dp > 0) {
+      const int ntiles2 = ((args.M + 255) / 256) * args.num_n_tiles, units = num_sms / 2;
+      args.streamk = 2;
+      args.dp_tiles = dp;
+      args.units_per_cta = ((ntiles2 - dp) * nk + units - 1) / units;
+      hybrid = true;
+    }
+  }
   if (args.streamk && epi != EPI_ADD_F32) {
     if (!args0.ws) return set_error(GLLM_EINVAL, "gemm: stream-K workspace required");
+    if (!hybrid && args.tile_ctr && ntiles > GEMM_MAX_SK_TILES) args.tile_ctr = nullptr;  // legacy memset + finish
   } else {
     args.ws = nullptr;
+    args.tile_ctr = nullptr;
   }
   switch (epi) {
     case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, args, stream, num_sms, cg);

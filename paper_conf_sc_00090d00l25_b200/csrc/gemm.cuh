@@ -33,8 +33,14 @@ struct GemmArgs {
   // 1 = stream-K: CTA i owns k-block units [i*units_per_cta, (i+1)*units_per_cta) of the
   // (tile, k-block) space; partial tiles combine with fp32 atomics into `out` (EPI_ADD_F32) or
   // into the fp32 workspace `ws` [M, N], finished by gemm_finish_kernel.
-  int streamk, units_per_cta;
+  // 2 = hybrid (CTA pairs, residual add only): whole tiles [0, dp_tiles) round robin, then
+  // stream-K over the remaining tiles' k-blocks (units_per_cta per pair), partial tiles reduced.
+  int streamk, units_per_cta, dp_tiles;
   float* ws;
+  // stream-K fixup counters (>= tiles ints).  Non-null: ws and tile_ctr are all zero on entry and
+  // the kernel leaves them zero (the last segment of each tile finishes it in-kernel); null: ws
+  // is zeroed before and gemm_finish_kernel applies the epilogue after.
+  int* tile_ctr;
   // fused RMSNorm (a4).  Consumers (EPI_STORE_BF16 / EPI_QKV_ROPE / EPI_SILU_MUL) read the bf16
   // copy of the residual as A and scale each output row by r = rsqrt(row_ss[row] * inv_h + eps)
   // (the norm gain is folded into W; it is exactly 1 for the O4 weights).  The producer
@@ -55,6 +61,7 @@ size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms);
 
 constexpr int GEMM_BM = 128, GEMM_BN = 256, GEMM_BK = 64, GEMM_STAGES = 4;
 constexpr size_t GEMM_WS_ELEMS = size_t(8) << 20;  // stream-K fp32 workspace capacity (32 MB)
+constexpr int GEMM_MAX_SK_TILES = 4096;             // stream-K fixup counters per workspace
 // TMA box rows of the B (weight) tensor maps: one 128-row half of a 256-wide N tile, so the same
 // map serves the 1-CTA kernel (two loads per stage) and the CTA-pair kernel (one per CTA).
 constexpr int GEMM_B_BOX = 128;

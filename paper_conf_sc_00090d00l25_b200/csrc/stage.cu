@@ -121,12 +121,13 @@ struct gllm_stage {
   float2* rope_cs = nullptr;
   int32_t* slots = nullptr;
   int32_t* sampled_tmp = nullptr;
-  float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T)
+  float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T), kept zero
+  int* sk_ctr = nullptr;     // stream-K fixup tile counters, kept zero
   float *ss_a = nullptr, *ss_b = nullptr;  // fused-RMSNorm row statistics (sum of squares of x)
   float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
   bool fused_norm = true;
   bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
-  bool prefill_ws = false;                 // GLLM_PREFILL_WS=1: warp-specialised tcgen05 prefill (A/B)
+  bool prefill_ws = true;                  // warp-specialised tcgen05 prefill (GLLM_PREFILL_WS=0: v1, A/B)
   bool attn_overlap = true;                // GLLM_ATTN_SERIAL=1: prefill and decode attention in series (A/B)
   bool decode_v1 = false;                  // GLLM_DECODE_V1=1: the per-CTA cp.async decode kernel (A/B)
   int* dec_ctr = nullptr;                  // persistent decode kernel: work counter + done counter
@@ -143,6 +144,7 @@ struct gllm_stage {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int last_T = 0, last_launches = 0;
   bool profiling = false;
+  bool prof_serial_attn = false;  // gllm_stage_set_profiling(st, 2): attribution pass, attention in series
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> prof_ev;
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
@@ -221,6 +223,7 @@ int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmE
   g.part_val = st->part_val;
   g.part_idx = st->part_idx;
   g.ws = st->gemm_ws;
+  g.tile_ctr = st->sk_ctr;
   st->last_launches += 1;
   return gllm::launch_gemm(a, b, epi, g, s, st->num_sms);
 }
@@ -407,14 +410,17 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = st->dalloc(&st->slots, R)) ||
       // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
       (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)) || (rc = st->dalloc(&st->ss_a, R)) ||
-      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)) || (rc = st->dalloc(&st->dec_ctr, 2)))
+      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)) || (rc = st->dalloc(&st->dec_ctr, 2)) ||
+      (rc = st->dalloc(&st->sk_ctr, gllm::GEMM_MAX_SK_TILES)))
     return fail(rc);
+  CK(cudaMemsetAsync(st->gemm_ws, 0, gllm::GEMM_WS_ELEMS * sizeof(float), s0));
+  CK(cudaMemsetAsync(st->sk_ctr, 0, gllm::GEMM_MAX_SK_TILES * sizeof(int), s0));
   CK(cudaMemsetAsync(st->dec_ctr, 0, 2 * sizeof(int), s0));
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
   gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
   if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
   if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
-  if (const char* e = std::getenv("GLLM_PREFILL_WS")) st->prefill_ws = e[0] == '1';
+  if (const char* e = std::getenv("GLLM_PREFILL_WS")) st->prefill_ws = e[0] != '0';
   if (block_size != 16) st->prefill_ws = false;
   if (const char* e = std::getenv("GLLM_ATTN_SERIAL")) st->attn_overlap = e[0] != '1';
   if (const char* e = std::getenv("GLLM_DECODE_V1")) st->decode_v1 = e[0] == '1';
@@ -698,6 +704,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.n_kv_heads = c.n_kv_heads;
       g.block_size = bs;
       g.ws = st->gemm_ws;
+      g.tile_ctr = st->sk_ctr;
+  g.tile_ctr = st->sk_ctr;
       g.row_ss = fused ? st->ss_a : nullptr;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
@@ -715,7 +723,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     };
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
-    const bool overlap = st->attn_overlap && P.n_pi > 0 && P.n_di > 0;
+    const bool overlap = st->attn_overlap && !st->prof_serial_attn && P.n_pi > 0 && P.n_di > 0;
     Prof p_attn(st, s, C_ATTN);  // span of the attention step (prefill || decode), on the main stream
     if (P.n_pi > 0) {
       cudaStream_t ps = overlap ? st->side : s;
@@ -759,6 +767,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.out = st->act;
       g.ldo = I;
       g.ws = st->gemm_ws;
+      g.tile_ctr = st->sk_ctr;
+  g.tile_ctr = st->sk_ctr;
       g.row_ss = fused ? st->ss_b : nullptr;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
@@ -844,6 +854,7 @@ int gllm_stage_sync(gllm_stage* st) {
 int gllm_stage_set_profiling(gllm_stage* st, int32_t on) {
   if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
   st->profiling = on != 0;
+  st->prof_serial_attn = on == 2;
   return GLLM_OK;
 }
 

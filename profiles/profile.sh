@@ -13,7 +13,7 @@ for t in 403 412; do timeout 300 python tools/attn_bench.py --tick $t >> $OUT/at
 timeout 300 python tools/attn_bench.py --config C3 --tick 500 >> $OUT/attn_bench.jsonl
 timeout 1200 ncu --nvtx --nvtx-include "timed/" --metrics gpu__time_duration.sum --clock-control none \
   --csv --log-file $OUT/launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $OUT/ncu_bench.json 2>&1
-for K in ${KERNELS:-gemm_tc_kernel decode_attn_kernel prefill_attn_tc_kernel}; do
+for K in ${KERNELS:-gemm_tc_kernel decode_attn_tma_kernel prefill_attn_ws_kernel}; do
   timeout 1200 ncu --nvtx --nvtx-include "timed/" --set full --clock-control none --import-source on \
     -k regex:$K -c ${NCU_COUNT:-5} -o $OUT/prof_$K -f python bench.py --steps 1 --warmup 3 --no-cpu-baseline \
     > $OUT/ncu_$K.log 2>&1

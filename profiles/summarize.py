@@ -15,7 +15,7 @@ import sys
 
 CAT = {"gemm_tc_kernel<0,": "qkv_gemm", "gemm_tc_kernel<4,": "qkv_gemm", "gemm_tc_kernel<2,": "gate_up_gemm",
        "gemm_tc_kernel<3,": "lm_head", "decode_attn_tma_kernel": "decode_attn", "decode_attn_kernel": "decode_attn",
-       "prefill_attn_tc": "prefill_attn", "prefill_attn_kernel": "prefill_attn", "rms_stats_kernel": "rmsnorm",
+       "prefill_attn_tc": "prefill_attn", "prefill_attn_ws": "prefill_attn", "prefill_attn_kernel": "prefill_attn", "rms_stats_kernel": "rmsnorm",
        "rmsnorm_kernel": "rmsnorm"}
 UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}
 

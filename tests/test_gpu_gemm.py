@@ -56,6 +56,21 @@ def test_residual_add_f32(M, N, K):
     assert err < 1e-3, err
 
 
+@pytest.mark.parametrize("M,N,K", [(900, 5120, 5120), (900, 5120, 27648), (1100, 4096, 4096), (2094, 5120, 5120)])
+def test_residual_add_f32_hybrid_tail(M, N, K):
+    # CTA-pair tiles whose last wave is mostly empty (C3's O / down GEMMs at T ~ 900: 80 tiles of
+    # 256 x 256 on 74 pairs): whole tiles first, the tail tiles' k-blocks spread over every pair
+    # and reduced into the residual (Jobs mode 2)
+    A, W = _bf16((M, K), 1.0, 14), _bf16((N, K), K ** -0.5, 15)
+    x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(16))
+    dA, dW, x = A.cuda(), W.cuda(), x0.clone().cuda()
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 1, x.data_ptr())
+    torch.cuda.synchronize()
+    ref = x0.double().numpy() + _ref(A, W)
+    err = np.abs(x.cpu().double().numpy() - ref).max()
+    assert err < 1e-3, err
+
+
 @pytest.mark.parametrize("M", [5, 128, 700])
 def test_silu_mul_interleaved(M):
     I, K = 1024, 512

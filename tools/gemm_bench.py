@@ -17,6 +17,9 @@ SHAPES = {
     "C1": [(2094, 6144, 4096, 0), (2094, 4096, 4096, 1), (2094, 28672, 4096, 2), (2094, 4096, 14336, 1)],
     "C4": [(128, 10240, 8192, 0), (128, 8192, 8192, 1), (128, 57344, 8192, 2), (128, 8192, 28672, 1)],
     "sq": [(8192, 8192, 8192, 0)],
+    # emulated PP stages at their window-mean T: C2 (PP=4, T ~ 625) and C3 (PP=8, T ~ 900)
+    "C2": [(625, 7168, 5120, 0), (625, 5120, 5120, 1), (625, 27648, 5120, 2), (625, 5120, 13824, 1)],
+    "C3": [(900, 7168, 5120, 0), (900, 5120, 5120, 1), (900, 55296, 5120, 2), (900, 5120, 27648, 1)],
     # the C1 O / down shapes with the plain bf16-store epilogue (isolates the residual epilogue)
     "C1s": [(2094, 4096, 4096, 0), (2094, 4096, 14336, 0)],
 }

@@ -97,15 +97,19 @@ if __name__ == "__main__":
     ap.add_argument("--ticks", type=int, default=160)
     ap.add_argument("--preroll", type=int, default=None)
     ap.add_argument("--policies", default="0,1",
-                    help="0 token throttling, 1 Sarathi-Serve (w/ CK), 2 w/o WT, 3 w/o UT (PAPER.md §4.5)")
+                    help="0 token throttling, 1 Sarathi-Serve (w/ CK), 2 w/o WT, 3 w/o UT (PAPER.md §4.5), "
+                         "4 context-aware throttling (R21, L354)")
+    ap.add_argument("--ctx-a", type=int, default=20000,
+                    help="policy 4 (context-aware throttling, R21): attention pairs per token-equivalent")
     ap.add_argument("--sweep", default="",
                     help="hyperparameter sensitivity (PAPER.md §4.6, Fig. 16) under token throttling, e.g. "
                          "'iterp=1,2,4,8,16' or 'maxp=512,1024,2048' or 'kvthresh_num=0,1,2' (den 20)")
     a = ap.parse_args()
     preroll = a.preroll if a.preroll is not None else int(STREAMS[a.config].get("window", (400, None))[0])
     out = {"config": a.config, "pp": a.pp, "stage": a.stage, "ticks": a.ticks, "preroll": preroll}
-    names = {0: "token_throttling", 1: "sarathi_serve", 2: "no_wt", 3: "no_ut"}
-    runs = [(names[int(p)], int(p), {}) for p in a.policies.split(",") if p != ""]
+    names = {0: "token_throttling", 1: "sarathi_serve", 2: "no_wt", 3: "no_ut", 4: "context_aware"}
+    runs = [(names[int(p)], int(p), {"attn_pairs_per_token": a.ctx_a} if int(p) == 4 else {})
+            for p in a.policies.split(",") if p != ""]
     if a.sweep:
         key, vals = a.sweep.split("=")
         runs = [(f"{key}={v}", 0, {key: int(v)}) for v in vals.split(",")]

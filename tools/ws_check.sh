@@ -10,3 +10,6 @@ done
 cat $OUT/attn.txt
 OUT=$OUT/ab AB="base GLLM_PREFILL_WS=1" bash tools/ab_bench.sh
 OUT=$OUT/ab3 CONFIG=C3 EXTRA="--pp 8 --stage 7" AB="base GLLM_PREFILL_WS=1" bash tools/ab_bench.sh
+timeout 600 python tools/gemm_bench.py --shapes C4 > $OUT/gemm_c4.txt 2>&1; cat $OUT/gemm_c4.txt
+timeout 1200 ncu --nvtx --nvtx-include "timed/" --metrics gpu__time_duration.sum --clock-control none \
+  --csv --log-file $OUT/launches_c4.csv python bench.py --config C4 --pp 8 --stage 7 --steps 2 --warmup 3 --no-cpu-baseline > $OUT/ncu_c4.json 2>&1

@@ -685,8 +685,18 @@ const bool g_cg1_rest = [] {
 
 int choose_cg(int M, int N, int epi, int num_sms) {
   if (g_force_cg) return g_force_cg;
-  const int tiles2 = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
+  const int nn = (N + GEMM_BN - 1) / GEMM_BN;
+  const int tiles2 = ((M + 255) / 256) * nn;
   if (M < 256 || tiles2 * 2 < num_sms || epi == EPI_ARGMAX) return 1;
+  // wave quantisation of whole tiles: the pair kernel is the faster per tile, but a 128-row tile
+  // grid can fill its waves much better (C2's QKV at T ~ 625: 140 tiles on 148 SMs in one wave
+  // vs 84 pair tiles on 74 pairs in two; measured 49 vs 68 us)
+  if (epi != EPI_ADD_F32) {
+    const int tiles1 = ((M + 127) / 128) * nn, u1 = num_sms, u2 = num_sms / 2;
+    const double e1 = (double)tiles1 / (double)(((tiles1 + u1 - 1) / u1) * u1);
+    const double e2 = (double)tiles2 / (double)(((tiles2 + u2 - 1) / u2) * u2);
+    if (e1 > e2 + 0.15) return 1;
+  }
   if (epi == EPI_STORE_BF16 || epi == EPI_QKV_ROPE) return 2;
   return g_cg1_rest && M < 4096 ? 1 : 2;
 }
@@ -701,8 +711,16 @@ const bool g_no_hybrid = [] {
 }();
 // Non-additive epilogues (QKV / SiLU / store) take the hybrid too when their fp32 workspace fits
 // (`ws_ok`): partial tiles then combine in ws and the last segment finishes the tile in-kernel.
+// Measured on B200 (profiles/r01/gemm_sched.txt): the in-kernel finish of workspace tiles costs
+// more than a memset + finish pass at C4's QKV (82 vs ~60 us), so it is opt-in
+// (GLLM_GEMM_SK_FIXUP=1) and only the residual-add epilogue takes the hybrid by default.
+const bool g_sk_fixup = [] {
+  const char* e = std::getenv("GLLM_GEMM_SK_FIXUP");
+  return e && e[0] == '1';
+}();
 int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms, bool ws_ok) {
   if (g_no_hybrid || cg != 2 || epi == EPI_ARGMAX || K / GEMM_BK < 8) return 0;
+  if (epi != EPI_ADD_F32 && !g_sk_fixup) return 0;
   const int units = num_sms / 2;
   const int ntiles = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
   if (epi != EPI_ADD_F32 && (!ws_ok || (size_t)M * N > GEMM_WS_ELEMS || ntiles * 2 > GEMM_MAX_SK_TILES)) return 0;
@@ -843,6 +861,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
       hybrid = true;
     }
   }
+  if (!g_sk_fixup) args.tile_ctr = nullptr;  // memset + finish pass (see hybrid_dp_tiles)
   if (args.streamk && epi != EPI_ADD_F32) {
     if (!args0.ws) return set_error(GLLM_EINVAL, "gemm: stream-K workspace required");
     if (!hybrid && args.tile_ctr && ntiles > GEMM_MAX_SK_TILES) args.tile_ctr = nullptr;  // legacy memset + finish

@@ -111,6 +111,33 @@ __device__ __forceinline__ float exp2_fma(float x) {
   return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
 }
 
+// packed fp32 pairs (sm_100 FFMA2 / FADD2)
+__device__ __forceinline__ uint64_t f2pack(float a, float b) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ void f2unpack(uint64_t v, float& a, float& b) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+}
+__device__ __forceinline__ uint64_t ffma2(uint64_t a, uint64_t b, uint64_t c) {
+  uint64_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+__device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+
+// Orders later uses of tcgen05.ld destination registers after the tcgen05.wait::ld that
+// precedes this call (the compiler sees no dependency between the wait and those registers).
+__device__ __forceinline__ void reg_fence(uint32_t (&r)[32]) {
+#pragma unroll
+  for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(r[i])::"memory");
+}
+
 // D[tmem] (+)= A[tmem] . B[smem]
 __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc, uint32_t idesc,
                                              uint32_t accumulate) {
@@ -314,28 +341,33 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::mbar_wait(&sfull[x], (uint32_t)(j & 1));
       ptx::tc_fence_after();
       const int kbase = j * WS_KT;
-      const bool diag = kbase + WS_KT - 1 > pos;  // keys past this row's position in this tile
-      // pass 1: row max of the raw scores
+      // causal masking only where some row of this warp ends inside the tile (warp-uniform, so
+      // the unmasked path carries no per-element compares)
+      const bool diag_w = __any_sync(0xffffffffu, kbase + WS_KT - 1 > pos);
+      // pass 1: row max of the raw scores; the next 32-column load is in flight while the
+      // current chunk is reduced (tcgen05.wait::ld covers every earlier load of the thread)
       float mx;
       {
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+        uint32_t sb[2][32];
+        ptx::tmem_ld_32x32b_x32(t_s, sb[0]);
+        ptx::tmem_ld_wait();
+        reg_fence(sb[0]);
 #pragma unroll
-        for (int h2 = 0; h2 < 2; ++h2) {
-          uint32_t r0[32], r1[32];
-          ptx::tmem_ld_32x32b_x32(t_s + h2 * 64, r0);
-          ptx::tmem_ld_32x32b_x32(t_s + h2 * 64 + 32, r1);
-          ptx::tmem_ld_wait();
-          if (diag) {
+        for (int cq = 0; cq < WS_KT / 32; ++cq) {
+          if (cq + 1 < WS_KT / 32) ptx::tmem_ld_32x32b_x32(t_s + (cq + 1) * 32, sb[(cq + 1) & 1]);
+          uint32_t(&r)[32] = sb[cq & 1];
+          if (diag_w) {
 #pragma unroll
-            for (int i = 0; i < 32; ++i) {
-              if (kbase + h2 * 64 + i > pos) r0[i] = __float_as_uint(-INFINITY);
-              if (kbase + h2 * 64 + 32 + i > pos) r1[i] = __float_as_uint(-INFINITY);
-            }
+            for (int i = 0; i < 32; ++i)
+              m4[i & 3] = fmaxf(m4[i & 3], kbase + cq * 32 + i > pos ? -INFINITY : __uint_as_float(r[i]));
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(r[i]));
           }
-#pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(r0[i]));
-            m4[(i + 2) & 3] = fmaxf(m4[(i + 2) & 3], __uint_as_float(r1[i]));
+          if (cq + 1 < WS_KT / 32) {
+            ptx::tmem_ld_wait();
+            reg_fence(sb[(cq + 1) & 1]);
           }
         }
         mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * sl2;
@@ -358,30 +390,43 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           tmem_st_x32(t_o + cb * 32, orr);
         }
       }
-      // pass 2: P = exp2(s * scale - m) as bf16 pairs over the consumed S columns
+      // pass 2: P = exp2(s * scale - m) as bf16 pairs over the consumed S columns (chunk cq's P
+      // lands in columns [16cq, 16cq + 16), already read); loads pipelined as in pass 1; the
+      // scale and the row sum run as packed f32x2 FFMA2 / FADD2 (half the FMA-pipe issues)
       float la = 0.f, lb = 0.f;
-#pragma unroll
-      for (int cq = 0; cq < WS_KT / 32; ++cq) {
-        uint32_t sr[32];
-        ptx::tmem_ld_32x32b_x32(t_s + cq * 32, sr);
+      {
+        const uint64_t sc2 = f2pack(sl2, sl2), nm2 = f2pack(-m_ref, -m_ref);
+        uint64_t l2 = f2pack(0.f, 0.f);
+        uint32_t sb[2][32];
+        ptx::tmem_ld_32x32b_x32(t_s, sb[0]);
         ptx::tmem_ld_wait();
-        uint32_t pw[16];
+        reg_fence(sb[0]);
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          const float x0 = fmaf(__uint_as_float(sr[2 * i]), sl2, -m_ref);
-          const float x1 = fmaf(__uint_as_float(sr[2 * i + 1]), sl2, -m_ref);
-          // EMU: one pair in four on the FMA pipe (MUFU and FMA pipes then finish together)
-          float p0 = (EMU && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
-          float p1 = (EMU && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
-          if (diag) {
-            if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
-            if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
+        for (int cq = 0; cq < WS_KT / 32; ++cq) {
+          if (cq + 1 < WS_KT / 32) ptx::tmem_ld_32x32b_x32(t_s + (cq + 1) * 32, sb[(cq + 1) & 1]);
+          const uint32_t(&sr)[32] = sb[cq & 1];
+          uint32_t pw[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            float x0, x1;
+            f2unpack(ffma2(f2pack(__uint_as_float(sr[2 * i]), __uint_as_float(sr[2 * i + 1])), sc2, nm2), x0, x1);
+            // EMU: one pair in four on the FMA pipe (A/B; measured slower at D = 128)
+            float p0 = (EMU && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
+            float p1 = (EMU && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
+            if (diag_w) {
+              if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
+              if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
+            }
+            l2 = fadd2(l2, f2pack(p0, p1));
+            pw[i] = ptx::pack_bf16(p0, p1);
           }
-          la += p0;
-          lb += p1;
-          pw[i] = ptx::pack_bf16(p0, p1);
+          tmem_st_x16(t_s + cq * 16, pw);
+          if (cq + 1 < WS_KT / 32) {
+            ptx::tmem_ld_wait();
+            reg_fence(sb[(cq + 1) & 1]);
+          }
         }
-        tmem_st_x16(t_s + cq * 16, pw);
+        f2unpack(l2, la, lb);
       }
       l += la + lb;
       tmem_st_wait();

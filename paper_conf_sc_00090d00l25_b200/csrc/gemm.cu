@@ -239,6 +239,18 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     ptx::mbar_wait(tfull_bar, parity);
     ptx::tc_fence_after();
   };
+  // While the MMAs of this tile run, pull the epilogue's other inputs into L2: the residual row
+  // segment (read-modify-write) or the row's RoPE table; one 128-B line per prefetch.
+  if (row_ok && !partial) {
+    if constexpr (EPI == EPI_ADD_F32) {
+      const float* xr = reinterpret_cast<const float*>(p.out) + (size_t)row * p.ldo + n_blk * GEMM_BN;
+      const int ncol = min(GEMM_BN, p.N - n_blk * GEMM_BN);
+      for (int c = 0; c < ncol; c += 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(xr + c));
+    } else if constexpr (EPI == EPI_QKV_ROPE) {
+      const float* cs = reinterpret_cast<const float*>(p.rope_cs + (size_t)row * (p.head_dim / 2));
+      for (int c = 0; c < p.head_dim; c += 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(cs + c));
+    }
+  }
   bool from_ws = false;  // this CTA finishes a stream-K tile from the workspace sums
   if (p.ws != nullptr && (partial || p.tile_ctr == nullptr)) {  // (legacy mode: every segment via ws)
     wait_acc();
@@ -615,6 +627,18 @@ __global__ void __launch_bounds__(256, 1)
 
 // Workspace mode: apply the non-additive epilogue to the fp32 sums in ws [M, N].
 // One thread per (row, 32-column chunk) of the OUTPUT space of the epilogue.
+__device__ __forceinline__ void ld_f32x32(const float* src, float (&v)[32]) {  // 8 x 16-B loads
+  const float4* s4 = reinterpret_cast<const float4*>(src);
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const float4 x = __ldg(s4 + q);
+    v[4 * q] = x.x;
+    v[4 * q + 1] = x.y;
+    v[4 * q + 2] = x.z;
+    v[4 * q + 3] = x.w;
+  }
+}
+
 template <int EPI>
 __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
   const int chunks_per_row = (EPI == EPI_SILU_MUL) ? p.N / 64 : p.N / 32;
@@ -626,26 +650,31 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
   if (p.zero_rows != nullptr && c == 0) p.zero_rows[row] = 0.f;
   if constexpr (EPI == EPI_STORE_BF16) {
     float v[32];
+    ld_f32x32(w + c * 32, v);
 #pragma unroll
-    for (int j = 0; j < 32; ++j) v[j] = w[c * 32 + j] * rs + (p.bias ? p.bias[c * 32 + j] : 0.f);
+    for (int j = 0; j < 32; ++j) v[j] = v[j] * rs + (p.bias ? p.bias[c * 32 + j] : 0.f);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, v);
   } else if constexpr (EPI == EPI_SILU_MUL) {
     const int n_blk = c / 4, cc = c % 4;  // output chunk -> (tile, chunk within the 128 gate columns)
     const float* g = w + n_blk * GEMM_BN + cc * 32;
     const float* u = g + GEMM_BN / 2;
-    float h[32];
+    float h[32], uv[32];
+    ld_f32x32(g, h);
+    ld_f32x32(u, uv);
 #pragma unroll
-    for (int j = 0; j < 32; ++j) h[j] = silu_f(g[j] * rs) * (u[j] * rs);
+    for (int j = 0; j < 32; ++j) h[j] = silu_f(h[j] * rs) * (uv[j] * rs);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, h);
   } else if constexpr (EPI == EPI_QKV_ROPE) {
     const int per_head = p.head_dim / 32, hpos = c % per_head;
     if (hpos >= per_head / 2) return;
     const int col1 = c * 32, half = p.head_dim / 2;
     float x1[32], x2[32];
+    ld_f32x32(w + col1, x1);
+    ld_f32x32(w + col1 + half, x2);
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
-      x1[j] = w[col1 + j] * rs + (p.bias ? p.bias[col1 + j] : 0.f);
-      x2[j] = w[col1 + half + j] * rs + (p.bias ? p.bias[col1 + half + j] : 0.f);
+      x1[j] = x1[j] * rs + (p.bias ? p.bias[col1 + j] : 0.f);
+      x2[j] = x2[j] * rs + (p.bias ? p.bias[col1 + half + j] : 0.f);
     }
     const int slot = p.slots[row];
     qkv_rope_store(p, row, col1, hpos * 32, x1, x2, slot / p.block_size, slot % p.block_size);

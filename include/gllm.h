@@ -210,6 +210,31 @@ GLLM_API int gllm_send_hidden(gllm_stage* st, const void* buf, int32_t num_token
 GLLM_API int gllm_recv_hidden(gllm_stage* st, void* buf, int32_t num_tokens, int32_t src, void* stream);
 GLLM_API int gllm_stage_sync(gllm_stage* st);
 
+/* Fused stage hand-off over peer memory (a12; PAPER.md L198, L204,
+ * L222): instead of an NCCL send/recv, stage s writes its output residual straight into a
+ * receive slot in stage s+1's device memory (NVLink peer stores, CUDA IPC mapping; on one GPU
+ * two processes share the device) from the last layer's residual-add GEMM epilogue, and raises
+ * the slot's flag with a system-scope release store after its last kernel.  Stage s+1's stream
+ * waits on that flag (cuStreamWaitValue32) and reads the slot as hidden_in.
+ * Slot reuse: micro-batch `tick` uses slot tick % depth.  With depth >= PP_depth the pipeline's
+ * own rule (at most PP_depth micro-batches in flight, batch k-PP retired before k is built, R1,
+ * L179) guarantees the receiver finished reading a slot before the sender overwrites it.
+ * Errors: EINVAL on bad arguments or a shape mismatch, ESTATE on the wrong stage role or a ring
+ * already created/opened, ECUDA on CUDA/IPC failures. */
+#define GLLM_PEER_HANDLE_BYTES 128
+/* Receiver (not the first stage): allocates depth slots of [max_tokens, hidden] fp32 plus depth
+ * 32-bit flags (zero) in one exportable allocation; writes the IPC handle (caller-owned, 128 B). */
+GLLM_API int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out);
+/* Sender (not the last stage): maps the receiver's ring from its handle. */
+GLLM_API int gllm_peer_ring_open(gllm_stage* st, const void* handle);
+/* Sender: the forward of a prepared batch with its output delivered to the receiver's slot for
+ * `tick` (hidden_out is the slot); flag = tick + 1 after the forward's last kernel. */
+GLLM_API int gllm_stage_forward_prepared_peer(gllm_stage* st, int32_t handle, const void* hidden_in,
+                                              int64_t tick, void* stream);
+/* Receiver: enqueues on `stream` a wait for the sender's release of `tick`; *slot_out = the
+ * device pointer of that slot (valid as hidden_in for forwards enqueued after the wait). */
+GLLM_API int gllm_peer_ring_recv(gllm_stage* st, int64_t tick, void* stream, void** slot_out);
+
 /* Introspection for parity tests (host outputs, synchronous). */
 /* Copies element range [row0, row0+nrows) x all columns of a logical weight
  * ("wq","wk","wv","wo","wg","wu","wd","bq","bk","bv","embed","lm_head") of

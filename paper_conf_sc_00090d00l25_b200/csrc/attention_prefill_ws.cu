@@ -8,8 +8,9 @@
 // both tiles share every K/V tile, and their softmax phases alternate with the other tile's MMAs
 // (ping-pong), so the tensor core and the SFU/FMA pipes run concurrently.  12 warps:
 //   warp 0      TMA producer: 128-key K and V tiles = 8 pages (16 x 64 SW128 boxes of the
-//               [kv_blocks*Hkv*16, D] page map) per tile, NS-stage ring, block table read a tile
-//               ahead; also owns the TMEM allocation (512 columns)
+//               [kv_blocks*Hkv*16, D] page map) per tile, NS-stage rings with separate K and V
+//               release (K slots free after the S MMAs, V slots after the PV MMAs), block table
+//               read a tile ahead; also owns the TMEM allocation (512 columns)
 //   warp 1      MMA issuer (one thread):  S_X = Q_X K_j^T  (M=128 N=128 K=D, both K-major)
 //                                          O_X += P_X V_j    (M=128 N=D K=128, P from TMEM, V MN-major)
 //               issue order per key tile j: PV_A(j), S_A(j+1), PV_B(j), [release stage], S_B(j+1),
@@ -50,8 +51,8 @@ struct WsSmem {
   static constexpr int K = Q + 2 * Q_TILE;
   static constexpr int V = K + WS_NS * KV_TILE;
   static constexpr int BAR = V + WS_NS * KV_TILE;
-  // barriers: q_full, kfull[NS], vfull[NS], kvempty[NS], sfull[2], pfull[2], ofull[2]; tmem slot
-  static constexpr int NBAR = 1 + 3 * WS_NS + 6;
+  // barriers: q_full, kfull[NS], vfull[NS], kempty[NS], vempty[NS], sfull[2], pfull[2], ofull[2]; tmem slot
+  static constexpr int NBAR = 1 + 4 * WS_NS + 6;
   static constexpr int BYTES = BAR + NBAR * 8 + 16 + 1024;  // + 1024-B alignment slack
 };
 
@@ -166,8 +167,9 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   uint64_t* q_full = bars;
   uint64_t* kfull = bars + 1;
   uint64_t* vfull = kfull + WS_NS;
-  uint64_t* kvempty = vfull + WS_NS;
-  uint64_t* sfull = kvempty + WS_NS;
+  uint64_t* kempty = vfull + WS_NS;   // K slot free: the last S MMA reading it completed
+  uint64_t* vempty = kempty + WS_NS;  // V slot free: the last PV MMA reading it completed
+  uint64_t* sfull = vempty + WS_NS;
   uint64_t* pfull = sfull + 2;
   uint64_t* ofull = pfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + L::NBAR);
@@ -193,7 +195,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     for (int s = 0; s < WS_NS; ++s) {
       ptx::mbar_init(&kfull[s], 1);
       ptx::mbar_init(&vfull[s], 1);
-      ptx::mbar_init(&kvempty[s], 1);
+      ptx::mbar_init(&kempty[s], 1);
+      ptx::mbar_init(&vempty[s], 1);
     }
     for (int x = 0; x < 2; ++x) {
       ptx::mbar_init(&sfull[x], 1);
@@ -214,38 +217,44 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
 
   if (warp == 0) {
-    // ---------------- TMA producer
+    // ---------------- TMA producer.  Loads in the order their slots free up: K(j) as soon as
+    // S_B(j-NS) (its slot's last reader) completes, V(j-1) once PV_B(j-1-NS) completes; so the
+    // next K tile streams in while the current tile's PV and softmax run.
     int bnext = 0;
     auto read_bt = [&](int j) {  // lanes 0..7: block ids of tile j's pages (past the sequence: its page 0)
       const int kb = j * PAGES + lane;
       return (lane < PAGES && j < n_kt) ? __ldg(bt + (kb < nblk_seq ? kb : 0)) : 0;
     };
+    auto load = [&](const CUtensorMap* map, uint64_t* full, uint32_t dst, const int (&bp)[PAGES]) {
+      ptx::mbar_arrive_expect_tx(full, L::KV_TILE);
+#pragma unroll
+      for (int p = 0; p < PAGES; ++p)
+#pragma unroll
+        for (int at = 0; at < ATOMS; ++at)
+          ptx::tma_load_2d(smem + dst + at * L::KV_ATOM + p * 2048, map, full, at * 64, (bp[p] * a.Hkv + kvh) * 16);
+    };
     bnext = read_bt(0);
+    int bprev[PAGES];
 #pragma unroll 1
-    for (int j = 0; j < n_kt; ++j) {
-      const int s = j % WS_NS;
+    for (int j = 0; j <= n_kt; ++j) {
       int bp[PAGES];
 #pragma unroll
       for (int p = 0; p < PAGES; ++p) bp[p] = __shfl_sync(0xffffffffu, bnext, p);
       bnext = read_bt(j + 1);
       if (lane == 0) {
-        if (j >= WS_NS) ptx::mbar_wait(&kvempty[s], (uint32_t)(((j / WS_NS) - 1) & 1));
-        const uint32_t kdst = L::K + s * L::KV_TILE, vdst = L::V + s * L::KV_TILE;
-        ptx::mbar_arrive_expect_tx(&kfull[s], L::KV_TILE);
-#pragma unroll
-        for (int p = 0; p < PAGES; ++p)
-#pragma unroll
-          for (int at = 0; at < ATOMS; ++at)
-            ptx::tma_load_2d(smem + kdst + at * L::KV_ATOM + p * 2048, &tmk, &kfull[s], at * 64,
-                             (bp[p] * a.Hkv + kvh) * 16);
-        ptx::mbar_arrive_expect_tx(&vfull[s], L::KV_TILE);
-#pragma unroll
-        for (int p = 0; p < PAGES; ++p)
-#pragma unroll
-          for (int at = 0; at < ATOMS; ++at)
-            ptx::tma_load_2d(smem + vdst + at * L::KV_ATOM + p * 2048, &tmv, &vfull[s], at * 64,
-                             (bp[p] * a.Hkv + kvh) * 16);
+        if (j >= 1) {  // V(j-1)
+          const int jv = j - 1, sv = jv % WS_NS;
+          if (jv >= WS_NS) ptx::mbar_wait(&vempty[sv], (uint32_t)(((jv / WS_NS) - 1) & 1));
+          load(&tmv, &vfull[sv], L::V + sv * L::KV_TILE, bprev);
+        }
+        if (j < n_kt) {  // K(j)
+          const int sk = j % WS_NS;
+          if (j >= WS_NS) ptx::mbar_wait(&kempty[sk], (uint32_t)(((j / WS_NS) - 1) & 1));
+          load(&tmk, &kfull[sk], L::K + sk * L::KV_TILE, bp);
+        }
       }
+#pragma unroll
+      for (int p = 0; p < PAGES; ++p) bprev[p] = bp[p];
       __syncwarp();
     }
   } else if (warp == 1) {
@@ -278,6 +287,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       wait_k(0);
       issue_s(0, 0);
       if (hasB) issue_s(1, 0);
+      ptx::umma_commit(&kempty[0]);  // K(0) is read by S_A(0), S_B(0) only
 #pragma unroll 1
       for (int j = 0; j < n_kt; ++j) {
         const int s = j % WS_NS;
@@ -300,7 +310,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           ptx::tc_fence_after();
           issue_pv(1, j);
         }
-        ptx::umma_commit(&kvempty[s]);  // stage s free once every MMA issued so far completes
+        ptx::umma_commit(&vempty[s]);  // V(j) free once the PVs issued so far complete
         if (hasB) {
           if (j + 1 < nB) {
             if (!k_next) wait_k(j + 1);
@@ -309,6 +319,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
             ptx::umma_commit(&ofull[1]);
           }
         }
+        if (j + 1 < n_kt) ptx::umma_commit(&kempty[(j + 1) % WS_NS]);  // every S of tile j+1 issued
       }
     }
   } else if (warp >= 4) {

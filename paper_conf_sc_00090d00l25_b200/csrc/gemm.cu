@@ -373,6 +373,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
             x.z += a4.z;
             x.w += a4.w;
             *reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + (size_t)(row0 + rr) * p.ldo + col) = x;
+            if (p.out_peer) *reinterpret_cast<float4*>(p.out_peer + (size_t)(row0 + rr) * p.ldo + col) = x;
             if (p.xb_out) {
               uint2 b;
               b.x = ptx::pack_bf16(x.x, x.y);
@@ -880,7 +881,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   args.units_per_cta = args.streamk ? (ntiles * nk + num_sms - 1) / num_sms : 0;
   args.dp_tiles = 0;
   bool hybrid = false;
-  if (cg == 2 && !args.xb_out && !args.ss_out) {  // partial tiles cannot produce the next norm's inputs
+  if (cg == 2 && !args.xb_out && !args.ss_out && !args.out_peer) {  // partial tiles: no fused outputs
     const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms, args0.ws && args0.tile_ctr);
     if (dp > 0) {
       const int ntiles2 = ((args.M + 255) / 256) * args.num_n_tiles, units = num_sms / 2;
@@ -898,6 +899,11 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
     args.ws = nullptr;
     args.tile_ctr = nullptr;
   }
+  static const bool dbg = std::getenv("GLLM_GEMM_DEBUG") != nullptr;
+  if (dbg)
+    std::fprintf(stderr, "[gemm] M=%d N=%d K=%d epi=%d cg=%d streamk=%d dp_tiles=%d per=%d ws=%d ctr=%d\n", args.M,
+                 args.N, args.K, (int)epi, cg, args.streamk, args.dp_tiles, args.units_per_cta, args.ws != nullptr,
+                 args.tile_ctr != nullptr);
   switch (epi) {
     case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, args, stream, num_sms, cg);
     case EPI_ADD_F32: return launch_e<EPI_ADD_F32>(a, b, args, stream, num_sms, cg);

@@ -50,6 +50,9 @@ struct GemmArgs {
   __nv_bfloat16* xb_out;
   float* ss_out;
   float* zero_rows;  // consumers: the n-tile-0 epilogue sets zero_rows[row] = 0 (resets the next ss_out)
+  // EPI_ADD_F32, whole tiles: the updated residual rows are also stored to out_peer [M, ldo] (the
+  // next pipeline stage's receive slot, NVLink peer memory) -- the fused stage hand-off (a12)
+  float* out_peer;
 };
 
 // true if launch_gemm would combine partial tiles (stream-K) for this shape -- then the ADD_F32

@@ -145,6 +145,15 @@ struct gllm_stage {
   int last_T = 0, last_launches = 0;
   bool profiling = false;
   bool prof_serial_attn = false;  // gllm_stage_set_profiling(st, 2): attribution pass, attention in series
+  // fused peer hand-off (a12, gllm_peer_*): receive ring owned here / the next stage's ring mapped here
+  float* ring = nullptr;
+  uint32_t* ring_flags = nullptr;
+  int ring_depth = 0;
+  void* peer_base = nullptr;  // IPC mapping of the next stage's ring
+  float* peer_ring = nullptr;
+  uint32_t* peer_flags = nullptr;
+  int peer_depth = 0;
+  size_t peer_slot_elems = 0;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> prof_ev;
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
@@ -262,6 +271,7 @@ void destroy(gllm_stage* st) {
   if (st->side) cudaStreamDestroy(st->side);
   if (st->ev_fork) cudaEventDestroy(st->ev_fork);
   if (st->ev_join) cudaEventDestroy(st->ev_join);
+  if (st->peer_base) cudaIpcCloseMemHandle(st->peer_base);
   cudaGetLastError();
   delete st;
 }
@@ -592,14 +602,15 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
 
 // Enqueues the stage forward of a prepared batch on `s`.
 int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidden_out, int32_t* sampled_out,
-                 cudaStream_t s) {
+                 cudaStream_t s, float* peer_out = nullptr) {
   const gllm_model_cfg& c = st->cfg;
   const int T = P.T, S = P.S, maxblk = P.maxblk, ns = P.ns, bs = st->bs;
   st->last_launches = 0;
   st->last_T = T;
   if (T == 0) return GLLM_OK;
   if (!st->is_first() && !hidden_in) return gllm::set_error(GLLM_EINVAL, "hidden_in required on stage > 0");
-  if (!st->is_last() && !hidden_out) return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
+  if (!st->is_last() && !hidden_out && !peer_out)
+    return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
   RC(ensure_parts(st, P.nparts));
   CK(cudaSetDevice(st->device));
   CK(cudaStreamWaitEvent(s, P.copied, 0));
@@ -662,7 +673,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     st->last_launches += 1;
   };
   const float inv_h = 1.0f / (float)H;
-  auto residual_gemm = [&](const CUtensorMap& ta, const CUtensorMap& tb, int K, float* ss_next) -> int {
+  auto residual_gemm = [&](const CUtensorMap& ta, const CUtensorMap& tb, int K, float* ss_next,
+                           float* out_peer) -> int {
     // ss_next was zeroed by the n-tile-0 epilogue of the preceding consumer GEMM (zero_rows)
     const bool sk = !fused || gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
     gllm::GemmArgs g{};
@@ -673,8 +685,11 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     g.ldo = H;
     g.xb_out = sk ? nullptr : st->y;
     g.ss_out = sk ? nullptr : ss_next;
+    g.out_peer = sk ? nullptr : out_peer;  // whole tiles store the new residual rows to the peer too
     st->last_launches += 1;
     RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms));
+    if (out_peer && sk)  // partial tiles reduce in place: copy the finished residual afterwards
+      CK(cudaMemcpyAsync(out_peer, x, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
     if (sk && fused) {  // partial tiles combine with reductions: recompute the statistics from x
       gllm::launch_rms_stats(x, st->y, ss_next, T, H, s);
       st->last_launches += 1;
@@ -755,7 +770,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     p_attn.close();
     {
       Prof p(st, s, C_O);
-      RC(residual_gemm(st->tm_attn, w.tm_o, qd, st->ss_b));
+      RC(residual_gemm(st->tm_attn, w.tm_o, qd, st->ss_b, nullptr));
     }
     standalone_norm();
     {
@@ -778,7 +793,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     }
     {
       Prof p(st, s, C_DOWN);
-      RC(residual_gemm(st->tm_act, w.tm_d, I, st->ss_a));
+      RC(residual_gemm(st->tm_act, w.tm_d, I, st->ss_a, li + 1 == st->layers.size() ? peer_out : nullptr));
     }
   }
   if (st->is_last() && ns > 0) {
@@ -1009,6 +1024,125 @@ int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed) {
   }
   CK(cudaDeviceSynchronize());
   return GLLM_OK;
+}
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- fused peer hand-off (a12)
+namespace {
+// ---- fused peer hand-off (a12): release flag written by one thread after the stage's last
+// kernel (stream order: every store of the forward, local and peer, is complete), system scope
+__global__ void peer_flag_kernel(uint32_t* flag, uint32_t value) {
+  __threadfence_system();
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(flag), "r"(value) : "memory");
+}
+
+using PfnWaitValue32 = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+PfnWaitValue32 wait_value32() {
+  static PfnWaitValue32 fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue32", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (PfnWaitValue32) nullptr;
+    return reinterpret_cast<PfnWaitValue32>(f);
+  }();
+  return fn;
+}
+
+struct PeerHandle {  // GLLM_PEER_HANDLE_BYTES
+  cudaIpcMemHandle_t mem;
+  int32_t depth, max_tokens, hidden, pad;
+};
+static_assert(sizeof(PeerHandle) <= GLLM_PEER_HANDLE_BYTES, "peer handle size");
+
+}  // namespace
+
+extern "C" {
+
+int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out) {
+  GLLM_TRY_BEGIN
+  if (!st || !handle_out || depth < 1) return gllm::set_error(GLLM_EINVAL, "peer ring: bad arguments");
+  if (st->is_first()) return gllm::set_error(GLLM_ESTATE, "peer ring: the first stage receives no hidden states");
+  if (st->ring) return gllm::set_error(GLLM_ESTATE, "peer ring already created");
+  CK(cudaSetDevice(st->device));
+  const size_t slot = (size_t)st->max_tokens * st->cfg.hidden;
+  const size_t bytes = (size_t)depth * slot * sizeof(float) + 256;
+  void* base = nullptr;
+  CK(cudaMalloc(&base, bytes));  // one plain allocation: exportable with cudaIpcGetMemHandle
+  CK(cudaMemset(base, 0, bytes));
+  st->allocs.push_back(base);
+  st->ring_flags = static_cast<uint32_t*>(base);  // [depth] flags in the first 256 B
+  st->ring = reinterpret_cast<float*>(static_cast<uint8_t*>(base) + 256);
+  st->ring_depth = depth;
+  PeerHandle h{};
+  CK(cudaIpcGetMemHandle(&h.mem, base));
+  h.depth = depth;
+  h.max_tokens = st->max_tokens;
+  h.hidden = st->cfg.hidden;
+  std::memset(handle_out, 0, GLLM_PEER_HANDLE_BYTES);
+  std::memcpy(handle_out, &h, sizeof(h));
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_peer_ring_open(gllm_stage* st, const void* handle) {
+  GLLM_TRY_BEGIN
+  if (!st || !handle) return gllm::set_error(GLLM_EINVAL, "peer ring open: null argument");
+  if (st->is_last()) return gllm::set_error(GLLM_ESTATE, "peer ring open: the last stage sends no hidden states");
+  if (st->peer_base) return gllm::set_error(GLLM_ESTATE, "peer ring already open");
+  PeerHandle h;
+  std::memcpy(&h, handle, sizeof(h));
+  if (h.depth < 1 || h.hidden != st->cfg.hidden || h.max_tokens < st->max_tokens)
+    return gllm::set_error(GLLM_EINVAL, "peer ring: shape mismatch (hidden %d vs %d, max_tokens %d vs %d)", h.hidden,
+                           st->cfg.hidden, h.max_tokens, st->max_tokens);
+  CK(cudaSetDevice(st->device));
+  void* base = nullptr;
+  CK(cudaIpcOpenMemHandle(&base, h.mem, cudaIpcMemLazyEnablePeerAccess));
+  st->peer_base = base;
+  st->peer_flags = static_cast<uint32_t*>(base);
+  st->peer_ring = reinterpret_cast<float*>(static_cast<uint8_t*>(base) + 256);
+  st->peer_depth = h.depth;
+  st->peer_slot_elems = (size_t)h.max_tokens * h.hidden;
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_stage_forward_prepared_peer(gllm_stage* st, int32_t handle, const void* hidden_in, int64_t tick,
+                                     void* stream) {
+  GLLM_TRY_BEGIN
+  if (!st || handle < RING || handle >= (int32_t)st->prep.size() || !st->prep[handle].in_use)
+    return gllm::set_error(GLLM_EINVAL, "bad prepared handle %d", handle);
+  if (!st->peer_base) return gllm::set_error(GLLM_ESTATE, "peer ring not open");
+  if (tick < 0) return gllm::set_error(GLLM_EINVAL, "negative tick");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const int slot = (int)(tick % st->peer_depth);
+  float* dst = st->peer_ring + (size_t)slot * st->peer_slot_elems;
+  RC(forward_impl(st, st->prep[handle], hidden_in, nullptr, nullptr, s, dst));
+  if (st->prep[handle].T > 0) {
+    peer_flag_kernel<<<1, 1, 0, s>>>(st->peer_flags + slot, (uint32_t)(tick + 1));
+    st->last_launches += 1;
+    CK(cudaGetLastError());
+  }
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_peer_ring_recv(gllm_stage* st, int64_t tick, void* stream, void** slot_out) {
+  GLLM_TRY_BEGIN
+  if (!st || !slot_out || tick < 0) return gllm::set_error(GLLM_EINVAL, "peer recv: bad arguments");
+  if (!st->ring) return gllm::set_error(GLLM_ESTATE, "peer ring not created");
+  PfnWaitValue32 wv = wait_value32();
+  if (!wv) return gllm::set_error(GLLM_ECUDA, "cuStreamWaitValue32 unavailable");
+  const int slot = (int)(tick % st->ring_depth);
+  CK(cudaSetDevice(st->device));
+  // (int32)(flag - (tick + 1)) >= 0: the sender released this slot for tick (or a later one)
+  const CUresult r = wv(reinterpret_cast<CUstream>(stream), reinterpret_cast<CUdeviceptr>(st->ring_flags + slot),
+                        (cuuint32_t)(tick + 1), CU_STREAM_WAIT_VALUE_GEQ);
+  if (r != CUDA_SUCCESS) return gllm::set_error(GLLM_ECUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+  *slot_out = st->ring + (size_t)slot * st->max_tokens * st->cfg.hidden;
+  return GLLM_OK;
+  GLLM_TRY_END
 }
 
 }  // extern "C"

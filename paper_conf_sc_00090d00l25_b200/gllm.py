@@ -106,6 +106,10 @@ def lib():
             "gllm_send_hidden": ([vp, vp, i32, i32, vp], C.c_int),
             "gllm_recv_hidden": ([vp, vp, i32, i32, vp], C.c_int),
             "gllm_stage_sync": ([vp], C.c_int),
+            "gllm_peer_ring_create": ([vp, i32, vp], C.c_int),
+            "gllm_peer_ring_open": ([vp, vp], C.c_int),
+            "gllm_stage_forward_prepared_peer": ([vp, i32, vp, i64, vp], C.c_int),
+            "gllm_peer_ring_recv": ([vp, i64, vp, C.POINTER(C.c_void_p)], C.c_int),
             "gllm_stage_read_weight": ([vp, i32, C.c_char_p, i64, i64, C.POINTER(C.c_float)], C.c_int),
             "gllm_stage_read_kv": ([vp, i32, _P32, i32, C.POINTER(C.c_float), C.POINTER(C.c_float)], C.c_int),
             "gllm_stage_read_slots": ([vp, _P32, i32], C.c_int),
@@ -330,6 +334,24 @@ class Stage:
     def comm_init(self, unique_id: bytes, rank: int, world: int):
         buf = C.create_string_buffer(unique_id, 128)
         _check(lib().gllm_comm_init(self.h, buf, rank, world))
+
+    # fused peer hand-off (a12): see include/gllm.h gllm_peer_*
+    def peer_ring_create(self, depth: int) -> bytes:
+        buf = C.create_string_buffer(128)
+        _check(lib().gllm_peer_ring_create(self.h, depth, buf))
+        return buf.raw
+
+    def peer_ring_open(self, handle: bytes):
+        buf = C.create_string_buffer(handle, 128)
+        _check(lib().gllm_peer_ring_open(self.h, buf))
+
+    def forward_prepared_peer(self, handle, tick, hidden_in=0, stream=0):
+        return _check(lib().gllm_stage_forward_prepared_peer(self.h, handle, hidden_in or None, tick, stream or None))
+
+    def peer_ring_recv(self, tick, stream=0) -> int:
+        out = C.c_void_p()
+        _check(lib().gllm_peer_ring_recv(self.h, tick, stream or None, C.byref(out)))
+        return out.value
 
     def send_hidden(self, ptr, num_tokens, dst, stream=0):
         _check(lib().gllm_send_hidden(self.h, ptr, num_tokens, dst, stream or None))

@@ -152,7 +152,10 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
-template <int D, bool EMU>
+// MODE 0: the kernel.  1: EMU (a quarter of the exponentials on the FMA pipe; A/B).  Timing
+// probes (GLLM_PREFILL_PROBE, wrong results, measurement only): 2 = no exp2 (P = the scaled
+// score), 3 = no softmax at all (P = whatever S left; only the load / MMA pipeline runs).
+template <int D, int MODE>
 __global__ void __launch_bounds__(WS_THREADS, 1)
     prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items,
                            const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
@@ -351,6 +354,12 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     for (int j = 0; j < nx; ++j) {
       ptx::mbar_wait(&sfull[x], (uint32_t)(j & 1));
       ptx::tc_fence_after();
+      if (MODE == 3) {
+        ptx::tc_fence_before();
+        ptx::mbar_arrive(&pfull[x]);
+        l = 1.f;
+        continue;
+      }
       const int kbase = j * WS_KT;
       // causal masking only where some row of this warp ends inside the tile (warp-uniform, so
       // the unmasked path carries no per-element compares)
@@ -422,8 +431,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
             float x0, x1;
             f2unpack(ffma2(f2pack(__uint_as_float(sr[2 * i]), __uint_as_float(sr[2 * i + 1])), sc2, nm2), x0, x1);
             // EMU: one pair in four on the FMA pipe (A/B; measured slower at D = 128)
-            float p0 = (EMU && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
-            float p1 = (EMU && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
+            float p0 = MODE == 2 ? x0 : (MODE == 1 && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
+            float p1 = MODE == 2 ? x1 : (MODE == 1 && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
             if (diag_w) {
               if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
               if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
@@ -478,22 +487,35 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   }
 }
 
-const bool g_prefill_emu = [] {
+const int g_prefill_mode = [] {
   const char* e = std::getenv("GLLM_PREFILL_EMU");
-  return e && e[0] == '1';
+  const char* p = std::getenv("GLLM_PREFILL_PROBE");
+  if (p && (p[0] == '2' || p[0] == '3')) return p[0] - '0';
+  return (e && e[0] == '1') ? 1 : 0;
 }();
 
-template <int D, bool EMU>
+template <int D, int MODE>
 int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
               int n_items, cudaStream_t s) {
   constexpr int bytes = WsSmem<D>::BYTES;
   static bool set = false;
   if (!set) {
-    cudaFuncSetAttribute(prefill_attn_ws_kernel<D, EMU>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(prefill_attn_ws_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  prefill_attn_ws_kernel<D, EMU><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
+  prefill_attn_ws_kernel<D, MODE><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
   return GLLM_OK;
+}
+
+template <int D>
+void launch_mode(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
+                 int n_items, cudaStream_t s) {
+  switch (g_prefill_mode) {
+    case 1: launch_ws<D, 1>(a, tmk, tmv, items, n_items, s); break;
+    case 2: launch_ws<D, 2>(a, tmk, tmv, items, n_items, s); break;
+    case 3: launch_ws<D, 3>(a, tmk, tmv, items, n_items, s); break;
+    default: launch_ws<D, 0>(a, tmk, tmv, items, n_items, s);
+  }
 }
 
 }  // namespace
@@ -505,11 +527,9 @@ int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const
   if (n_items <= 0) return GLLM_OK;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "prefill attention (ws): block size %d unsupported", a.bs);
   if (a.D == 128)
-    g_prefill_emu ? launch_ws<128, true>(a, tmk, tmv, items, n_items, s)
-                  : launch_ws<128, false>(a, tmk, tmv, items, n_items, s);
+    launch_mode<128>(a, tmk, tmv, items, n_items, s);
   else if (a.D == 64)
-    g_prefill_emu ? launch_ws<64, true>(a, tmk, tmv, items, n_items, s)
-                  : launch_ws<64, false>(a, tmk, tmv, items, n_items, s);
+    launch_mode<64>(a, tmk, tmv, items, n_items, s);
   else
     return set_error(GLLM_EINVAL, "prefill attention (ws): head_dim %d unsupported", a.D);
   cudaError_t e = cudaGetLastError();

@@ -340,9 +340,20 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       float ss[8];
 #pragma unroll
       for (int k = 0; k < 8; ++k) ss[k] = 0.f;
-      wait_acc();
-#pragma unroll 1
-      for (int c = 0; c < GEMM_BN / 32; ++c) {
+      // the residual rows of chunk c + 1 are loaded while chunk c is combined (two register
+      // buffers); chunk 0's are loaded before the accumulator is ready, under the mainloop
+      auto load_x = [&](int c, float4(&xv)[8]) {
+        const int col = n_blk * GEMM_BN + c * 32 + c4;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int rr = rsub + 4 * k;
+          xv[k] = (col < p.N && row0 + rr < p.M)
+                      ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.out) +
+                                                         (size_t)(row0 + rr) * p.ldo + col)
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+      };
+      auto combine = [&](int c, const float4(&xv)[8]) {
         ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
         ptx::tmem_ld_wait();
 #pragma unroll
@@ -353,15 +364,6 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
         __syncwarp();
         const int col = n_blk * GEMM_BN + c * 32 + c4;
         const bool col_ok = col < p.N;
-        float4 xv[8];
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const int rr = rsub + 4 * k;
-          xv[k] = (col_ok && row0 + rr < p.M)
-                      ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.out) +
-                                                         (size_t)(row0 + rr) * p.ldo + col)
-                      : make_float4(0.f, 0.f, 0.f, 0.f);
-        }
 #pragma unroll
         for (int k = 0; k < 8; ++k) {
           const int rr = rsub + 4 * k;
@@ -384,6 +386,16 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
           }
         }
         __syncwarp();
+      };
+      float4 xa[8], xb[8];
+      load_x(0, xa);
+      wait_acc();
+#pragma unroll 1
+      for (int c = 0; c < GEMM_BN / 32; c += 2) {
+        load_x(c + 1, xb);
+        combine(c, xa);
+        if (c + 2 < GEMM_BN / 32) load_x(c + 2, xa);
+        combine(c + 1, xb);
       }
       if (p.ss_out) {  // row rsub + 4k: its 32 columns of this tile are spread over 8 lanes
 #pragma unroll

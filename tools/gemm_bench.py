@@ -20,6 +20,9 @@ SHAPES = {
     # emulated PP stages at their window-mean T: C2 (PP=4, T ~ 625) and C3 (PP=8, T ~ 900)
     "C2": [(625, 7168, 5120, 0), (625, 5120, 5120, 1), (625, 27648, 5120, 2), (625, 5120, 13824, 1)],
     "C3": [(900, 7168, 5120, 0), (900, 5120, 5120, 1), (900, 55296, 5120, 2), (900, 5120, 27648, 1)],
+    # C3's O shape with the plain store epilogue, and with K cut to 512 / 1024 (prologue + epilogue
+    # dominated): separates the residual epilogue's cost from the mainloop's
+    "C3s": [(900, 5120, 5120, 0), (900, 5120, 512, 1), (900, 5120, 512, 0), (900, 5120, 1024, 1), (900, 5120, 1024, 0)],
     # the C1 O / down shapes with the plain bf16-store epilogue (isolates the residual epilogue)
     "C1s": [(2094, 4096, 4096, 0), (2094, 4096, 14336, 0)],
 }

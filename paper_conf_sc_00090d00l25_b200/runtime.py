@@ -100,15 +100,26 @@ class GpuExecutor:
         self.stage.release(h)
         self.keep.pop(h, None)
 
+    peer_in = False    # hidden_in arrives in this stage's peer ring (PeerTransport)
+    peer_out = False   # hidden_out goes straight into the next stage's peer ring
+
     def forward(self, h, k, T, is_first, is_last, ns):
         i = k & 1
+        cs = self.compute.cuda_stream
+        hin = 0
         if not is_first:
-            self.compute.wait_event(self.recv_ev[i])
-        if not is_last:
-            self.compute.wait_event(self.send_ev[i])   # send k-2 finished reading hout[i]
-        self.stage.forward_prepared(h, 0 if is_first else self.hin[i].data_ptr(),
-                                    0 if is_last else self.hout[i].data_ptr(),
-                                    self.samp[k & 3].data_ptr() if is_last else 0, self.compute.cuda_stream)
+            if self.peer_in:   # stream waits for the sender's release flag of tick k
+                hin = self.stage.peer_ring_recv(k, cs)
+            else:
+                self.compute.wait_event(self.recv_ev[i])
+                hin = self.hin[i].data_ptr()
+        if not is_last and self.peer_out:
+            self.stage.forward_prepared_peer(h, k, hin, cs)
+        else:
+            if not is_last:
+                self.compute.wait_event(self.send_ev[i])   # send k-2 finished reading hout[i]
+            self.stage.forward_prepared(h, hin, 0 if is_last else self.hout[i].data_ptr(),
+                                        self.samp[k & 3].data_ptr() if is_last else 0, cs)
         self.fwd_ev[i].record(self.compute)
         if is_last and ns:
             with self.torch.cuda.stream(self.compute):
@@ -139,6 +150,35 @@ class NcclTransport:
         ex.comm.wait_event(ex.fwd_ev[i])
         ex.stage.send_hidden(ex.hout[i].data_ptr(), T, self.rank + 1, ex.comm.cuda_stream)
         ex.send_ev[i].record(ex.comm)
+
+
+class PeerTransport:
+    """Fused hand-off over peer memory (include/gllm.h gllm_peer_*): stage s+1 exports a ring of
+    receive slots, stage s maps it and its last residual GEMM writes into the slot; the flags make
+    the hand-off stream-ordered, so recv/send are no-ops here.  Slot reuse is safe with
+    depth >= PP by R1 (batch k-PP retires before batch k is built); depth = 2 PP."""
+
+    def __init__(self, ex: GpuExecutor, rank, world, group, pp=None):
+        import torch
+        import torch.distributed as dist
+        self.ex, self.rank, self.world = ex, rank, world
+        depth = 2 * (pp or world)
+        # ring handles travel rank s+1 -> rank s over the (gloo) metadata group, in rank order
+        if rank > 0:
+            h = ex.stage.peer_ring_create(depth)
+            dist.send(torch.frombuffer(bytearray(h), dtype=torch.uint8), rank - 1, group=group)
+            ex.peer_in = True
+        if rank < world - 1:
+            t = torch.empty(128, dtype=torch.uint8)
+            dist.recv(t, rank + 1, group=group)
+            ex.stage.peer_ring_open(bytes(t.numpy().tobytes()))
+            ex.peer_out = True
+
+    def recv(self, k, T):
+        pass
+
+    def send(self, k, T):
+        pass
 
 
 class _NullTransport:

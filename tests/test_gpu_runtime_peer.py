@@ -1,0 +1,123 @@
+"""The pipeline runtime with the fused peer hand-off, end to end on one GPU: two ranks (stage 0:
+embedding + layer 0; stage 1: layer 1 + LM head of a 2-layer Llama-3-8B-shaped model) share
+cuda:0, exchange micro-batch metadata over gloo (L204) and hidden states through
+PeerTransport (gllm_peer_*, stream-ordered flags, no NCCL).  The greedy ids the last stage
+returns must agree with a one-process run of the same model on the same C1 stream prefix
+(same scheduler, PP_depth = 2 retire rule)."""
+import multiprocessing as mp
+import os
+import socket
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+TICKS = 40
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _setup(world):
+    import sys
+    sys.path.insert(0, ROOT)
+    import torch
+    from paper_conf_sc_00090d00l25_b200 import gllm
+    from workloads.configs import MODELS, SchedParams
+    from workloads.streams import make_stream
+    m = MODELS["C1"].with_layers(2)
+    sp = SchedParams(pp_depth=2, num_blocks=3000)
+    st = make_stream("C1", m.vocab, n=80)
+    max_tokens = sp.maxp + sp.max_seqs + 64
+    return torch, gllm, m, sp, st, max_tokens
+
+
+def _record(ex, store):
+    orig = ex.sampled
+
+    def sampled(k, ns):
+        ids = orig(k, ns)
+        store[int(k)] = np.asarray(ids).tolist()
+        return ids
+    ex.sampled = sampled
+
+
+def _peer_rank(rank, world, port, q):
+    torch, gllm, m, sp, st, max_tokens = _setup(world)
+    import torch.distributed as dist
+    from paper_conf_sc_00090d00l25_b200.runtime import GpuExecutor, PeerTransport, Pipeline, split_layers
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    lb, le = split_layers(m.n_layers, world)[rank]
+    stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
+    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden)
+    tr = PeerTransport(ex, rank, world, dist.group.WORLD)
+    sched = None
+    if rank == 0:
+        sched = gllm.Sched(sp)
+        sched.add_stream(st)
+    pipe = Pipeline(rank, world, ex, tr, sched, dist.group.WORLD)
+    got = {}
+    _record(ex, got)
+    for _ in range(TICKS):
+        pipe.tick()
+    pipe.drain()
+    torch.cuda.synchronize()
+    dist.barrier()
+    q.put((rank, got))
+    dist.destroy_process_group()
+    stage.close()
+
+
+def _reference(q):
+    torch, gllm, m, sp, st, max_tokens = _setup(1)
+    from paper_conf_sc_00090d00l25_b200.runtime import GpuExecutor, Pipeline
+    torch.cuda.set_device(0)
+    stage = gllm.Stage(m, 0, m.n_layers, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
+    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden)
+    sched = gllm.Sched(sp)
+    sched.add_stream(st)
+    pipe = Pipeline(0, 1, ex, None, sched, None, pp=2)
+    got = {}
+    _record(ex, got)
+    for _ in range(TICKS):
+        pipe.tick()
+    torch.cuda.synchronize()
+    q.put(("ref", got))
+    stage.close()
+
+
+@pytest.mark.timeout(900)
+def test_pipeline_runtime_with_peer_handoff_matches_one_process():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ref = ctx.Process(target=_reference, args=(q,))
+    ref.start()
+    tag, want = q.get(timeout=600)
+    ref.join(timeout=120)
+    assert tag == "ref" and ref.exitcode == 0
+    port = _free_port()
+    ps = [ctx.Process(target=_peer_rank, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    outs = dict(q.get(timeout=600) for _ in range(2))
+    for p in ps:
+        p.join(timeout=120)
+        assert p.exitcode == 0, f"rank exit code {p.exitcode}"
+    got = outs[1]                       # the last stage's sampled ids, by tick
+    common = sorted(set(want) & set(got))
+    assert len(common) >= TICKS - 4, (len(common), sorted(want)[:5], sorted(got)[:5])
+    n = agree = 0
+    for k in common:
+        assert len(got[k]) == len(want[k]), k
+        a, b = np.asarray(got[k]), np.asarray(want[k])
+        n += len(a)
+        agree += int((a == b).sum())
+    assert n > 100 and agree / n >= 0.98, (agree, n)

@@ -250,10 +250,14 @@ def run_ours(args):
         stage.fill_kv(0xC4)                   # warm-start decode set: cache pages hold O4 values
     tr = None
     if world > 1:
-        uid = [gllm.get_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(uid, 0)
-        stage.comm_init(uid[0], rank, world)
-        tr = NcclTransport(ex, rank, world)
+        if args.handoff == "peer":   # fused hand-off over NVLink peer memory (gllm_peer_*)
+            from paper_conf_sc_00090d00l25_b200.runtime import PeerTransport
+            tr = PeerTransport(ex, rank, world, meta)
+        else:
+            uid = [gllm.get_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, 0)
+            stage.comm_init(uid[0], rank, world)
+            tr = NcclTransport(ex, rank, world)
     sched = None
     stream = make_stream(args.config, m.vocab)
     if rank == 0:
@@ -405,6 +409,7 @@ def run_ours(args):
             "config": {**workload_config(args, sp), "layers_per_stage": le - lb,
                        "global_batch": round(tokens / args.steps, 1),
                        "token_budget": sp.maxp, "preroll_ticks": args.preroll,
+                       "handoff": args.handoff if N > 1 else None,
                        "window_ticks": [int(timed[0]["tick"]), int(timed[-1]["tick"])],
                        "l2": f"inputs > L2: every step streams all {le - lb} layers' weights (GBs >> 126 MB L2)"},
             "e2e": {"value": round(e2e_value, 1), "unit": UNIT, "h2d_bytes_per_step": int(h2d / args.steps),
@@ -544,6 +549,8 @@ def main():
     ap.add_argument("--stage", type=int, default=0, help="with --gpus 1 --pp N: which stage to run")
     ap.add_argument("--kv-blocks", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--handoff", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: stage hand-off over NCCL P2P (default) or the fused peer-memory path")
     args = ap.parse_args()
     if args.preroll is None:
         from workloads.configs import STREAMS

@@ -225,7 +225,8 @@ GLLM_API int gllm_stage_sync(gllm_stage* st);
 /* Receiver (not the first stage): allocates depth slots of [max_tokens, hidden] fp32 plus depth
  * 32-bit flags (zero) in one exportable allocation; writes the IPC handle (caller-owned, 128 B). */
 GLLM_API int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out);
-/* Sender (not the last stage): maps the receiver's ring from its handle. */
+/* Sender (not the last stage): maps the receiver's ring from its handle.  The receiver must live
+ * in another process (CUDA IPC handles cannot be opened by the exporting process): ECUDA. */
 GLLM_API int gllm_peer_ring_open(gllm_stage* st, const void* handle);
 /* Sender: the forward of a prepared batch with its output delivered to the receiver's slot for
  * `tick` (hidden_out is the slot); flag = tick + 1 after the forward's last kernel. */

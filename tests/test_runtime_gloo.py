@@ -104,7 +104,7 @@ def _worker(rank, world, port, ticks, q):
 
 def _bench_flow_worker(rank, world, port, q):
     """bench.py's multi-rank sequence: preroll ticks, drain, W+K batches scheduled up front and run
-    from prepared handles (twice: timed, then the attribution pass), bookkeeping reset, e2e serving
+    from prepared handles (three times: timed, profiled, attribution), bookkeeping reset, e2e serving
     ticks, drain."""
     import torch.distributed as dist
 
@@ -132,8 +132,9 @@ def _bench_flow_worker(rank, world, port, q):
     handles = [ex.prepare(a) for a in batches]
     for a, h in zip(batches, handles):
         pipe.run_batch(a, h)
-    for a, h in zip(batches, handles):   # bench's untimed attribution pass re-runs the same batches
-        pipe.run_batch(a, h)
+    for _ in range(2):   # bench's untimed profiled and attribution passes re-run the same batches
+        for a, h in zip(batches, handles):
+            pipe.run_batch(a, h)
     pipe.pending_samples.clear()
     pipe._expect.clear()
     # e2e leg: a fresh scheduler fast-forwarded to the value window replays the same ticks

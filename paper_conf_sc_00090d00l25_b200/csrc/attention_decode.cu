@@ -22,6 +22,7 @@
 #include "attention.cuh"
 #include "common.h"
 #include "ptx.cuh"
+#include "launch.cuh"
 
 namespace gllm {
 
@@ -65,6 +66,7 @@ __global__ void __launch_bounds__(WARPS * 32)
   const float sl2 = LOG2E_D * rsqrtf((float)D);
   const uint64_t pol = ptx::policy_evict_first();  // each page is read once per layer
 
+  pdl_trigger();
   if (lane == 0) {
     for (int s = 0; s < NST; ++s) ptx::mbar_init(&bar[s], 1);
     ptx::fence_barrier_init();
@@ -74,6 +76,7 @@ __global__ void __launch_bounds__(WARPS * 32)
     }
   }
   __syncwarp();
+  pdl_wait();  // work counter, Q rows, block table, KV pages: all produced by earlier kernels
 
   // ---- issue side of the page stream (warp-uniform state; lane 0 issues).  Global reads on
   // this path are issued a step before their value is needed: the next work item is claimed
@@ -351,7 +354,8 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
     int grid = per_sm * num_sms;
     const int need = (n_work + WARPS - 1) / WARPS;
     if (grid > need) grid = need;
-    decode_attn_tma_kernel<D, G, NST, WARPS><<<grid, WARPS * 32, Lay::BYTES, s>>>(a, items, n_work, ctr, tmk, tmv);
+    launch_pdl(decode_attn_tma_kernel<D, G, NST, WARPS>, dim3(grid), dim3(WARPS * 32), Lay::BYTES, s, 1, a, items,
+               n_work, ctr, tmk, tmv);
   }
   (void)merges;
   (void)n_merges;  // split rows are merged inside the kernel by their last split

@@ -28,6 +28,7 @@
 #include "attention.cuh"
 #include "common.h"
 #include "ptx.cuh"
+#include "launch.cuh"
 
 namespace gllm {
 
@@ -177,6 +178,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   uint64_t* ofull = pfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + L::NBAR);
 
+  pdl_trigger();
+  pdl_wait();
   const PrefillItem it = items[blockIdx.x];
   const int kvh = blockIdx.y;
   const int G = a.Hq / a.Hkv;
@@ -503,7 +506,7 @@ int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
     cudaFuncSetAttribute(prefill_attn_ws_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  prefill_attn_ws_kernel<D, MODE><<<dim3(n_items, a.Hkv), WS_THREADS, bytes, s>>>(a, items, tmk, tmv);
+  launch_pdl(prefill_attn_ws_kernel<D, MODE>, dim3(n_items, a.Hkv), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
   return GLLM_OK;
 }
 

@@ -25,6 +25,7 @@
 
 #include "common.h"
 #include "gemm.cuh"
+#include "launch.cuh"
 #include "ptx.cuh"
 
 namespace gllm {
@@ -497,6 +498,7 @@ __global__ void __launch_bounds__(256, 1)
   const int lane = threadIdx.x & 31;
   const uint32_t rank = CG == 2 ? cluster_rank() : 0;
   const bool leader = rank == 0;
+  pdl_trigger();
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tma_a);
     ptx::tma_prefetch(&tma_b);
@@ -520,6 +522,9 @@ __global__ void __launch_bounds__(256, 1)
     __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_ptr;
+  // A operand, residual, workspace, slots: produced by earlier kernels.  The producer thread waits
+  // after issuing the dependency-free weight tiles of its first ring fill (below).
+  if (warp != 0 || lane != 0) pdl_wait();
 
   const int num_m = (p.M + C::TILE_M - 1) / C::TILE_M;
   Jobs jobs;
@@ -531,13 +536,40 @@ __global__ void __launch_bounds__(256, 1)
       // ---------------- TMA producer (both CTAs of a pair load their halves)
       int stage = 0;
       uint32_t phase = 0;
+      int pre = 0;  // stages whose B tile (and expect_tx) went out before the wait
+      if (p.b_static) {
+        Jobs pj = jobs;
+        if (pj.next(tile, kb0, kb1)) {
+          const int b_row = (tile / num_m) * GEMM_BN + rank * C::B_ROWS;
+          pre = min(C::STAGES, kb1 - kb0);
+          for (int i = 0; i < pre; ++i) {  // fresh ring: every empty barrier passes
+            const int kb = kb0 + i;
+            if constexpr (CG == 1) {
+              ptx::mbar_arrive_expect_tx(&full[i], C::STAGE_BYTES);
+              ptx::tma_load_2d(sB + i * C::B_BYTES, &tma_b, &full[i], kb * GEMM_BK, b_row);
+              ptx::tma_load_2d(sB + i * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[i], kb * GEMM_BK,
+                               b_row + GEMM_B_BOX);
+            } else {
+              if (leader) ptx::mbar_arrive_expect_tx(&full[i], 2 * C::STAGE_BYTES);
+              tma_load_2d_cg2(sB + i * C::B_BYTES, &tma_b, &full[i], kb * GEMM_BK, b_row);
+            }
+          }
+        }
+      }
+      pdl_wait();
       while (jobs.next(tile, kb0, kb1)) {
         const int m_blk = tile % num_m, n_blk = tile / num_m;
         const int a_row = m_blk * C::TILE_M + rank * GEMM_BM;
         const int b_row = n_blk * GEMM_BN + rank * C::B_ROWS;
         for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&empty[stage], phase ^ 1);
-          if constexpr (CG == 1) {
+          if (pre > 0) {  // B and the expect_tx of this stage were issued before the wait
+            if constexpr (CG == 1)
+              ptx::tma_load_2d(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
+            else
+              tma_load_2d_cg2(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
+            --pre;
+          } else if constexpr (CG == 1) {
             ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
             ptx::tma_load_2d(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
             ptx::tma_load_2d(sB + stage * C::B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, b_row);
@@ -654,6 +686,8 @@ __device__ __forceinline__ void ld_f32x32(const float* src, float (&v)[32]) {  /
 
 template <int EPI>
 __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
+  pdl_trigger();
+  pdl_wait();
   const int chunks_per_row = (EPI == EPI_SILU_MUL) ? p.N / 64 : p.N / 32;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= p.M * chunks_per_row) return;
@@ -846,27 +880,13 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
     cudaError_t e = cudaMemsetAsync(args.ws, 0, (size_t)args.M * args.N * sizeof(float), stream);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm workspace memset: %s", cudaGetErrorString(e));
   }
-  if constexpr (CG == 1) {
-    gemm_tc_kernel<EPI, 1><<<grid, 256, C::SMEM_BYTES, stream>>>(a, b, args);
-  } else {
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(256);
-    cfg.dynamicSmemBytes = C::SMEM_BYTES;
-    cfg.stream = stream;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 2;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_tc_kernel<EPI, 2>, a, b, args);
-    if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (2-CTA) launch: %s", cudaGetErrorString(e));
+  {
+    cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, CG, a, b, args);
+    if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (%d-CTA) launch: %s", CG, cudaGetErrorString(e));
   }
   if (args.ws && !args.tile_ctr) {
     const int chunks = args.M * ((EPI == EPI_SILU_MUL) ? args.N / 64 : args.N / 32);
-    gemm_finish_kernel<EPI><<<(chunks + 255) / 256, 256, 0, stream>>>(args);
+    launch_pdl(gemm_finish_kernel<EPI>, dim3((chunks + 255) / 256), dim3(256), 0, stream, 1, args);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm launch: %s", cudaGetErrorString(e));

@@ -36,6 +36,9 @@ struct GemmArgs {
   // 2 = hybrid (CTA pairs, residual add only): whole tiles [0, dp_tiles) round robin, then
   // stream-K over the remaining tiles' k-blocks (units_per_cta per pair), partial tiles reduced.
   int streamk, units_per_cta, dp_tiles;
+  // B (the weights) is never written by a kernel on the stream: with PDL the producer issues the
+  // first ring fill's B tiles before griddepcontrol.wait (stage GEMMs only; gllm_op_gemm leaves 0)
+  int b_static;
   float* ws;
   // stream-K fixup counters (>= tiles ints).  Non-null: ws and tile_ctr are all zero on entry and
   // the kernel leaves them zero (the last segment of each tile finishes it in-kernel); null: ws

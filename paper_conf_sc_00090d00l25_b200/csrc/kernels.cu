@@ -5,6 +5,9 @@
 #include <cuda_bf16.h>
 
 #include "kernels.cuh"
+#include "launch.cuh"
+
+#include <cstdlib>
 
 namespace gllm {
 
@@ -61,6 +64,8 @@ __global__ void fill_kv_kernel(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, 
 __global__ void prep_kernel(const int32_t* __restrict__ positions, const int32_t* __restrict__ cu_q,
                             const int32_t* __restrict__ bt, int T, int S, int maxblk, int bs, int32_t* slots,
                             float2* cs, int half, double log2_theta) {
+  pdl_trigger();
+  pdl_wait();
   const int t = blockIdx.x;
   if (t >= T) return;
   const int pos = positions[t];
@@ -81,6 +86,8 @@ __global__ void prep_kernel(const int32_t* __restrict__ positions, const int32_t
 }
 
 __global__ void embed_kernel(const __nv_bfloat16* __restrict__ E, const int32_t* __restrict__ ids, float* x, int H) {
+  pdl_trigger();
+  pdl_wait();
   const int t = blockIdx.x;
   const __nv_bfloat16* row = E + (int64_t)ids[t] * H;
   float* out = x + (int64_t)t * H;
@@ -115,6 +122,8 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const float* __restrict__ 
                                                       __nv_bfloat16* y, const int32_t* __restrict__ rows, int H,
                                                       float eps) {
   __shared__ float red[8];
+  pdl_trigger();
+  pdl_wait();
   const int r = blockIdx.x;
   const int src = rows ? rows[r] : r;
   const float* xr = x + (int64_t)src * H;
@@ -141,6 +150,8 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const float* __restrict__ 
 __global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict__ x, __nv_bfloat16* xb, float* ss,
                                                         int H) {
   __shared__ float red[8];
+  pdl_trigger();
+  pdl_wait();
   const int r = blockIdx.x;
   const float* xr = x + (int64_t)r * H;
   __nv_bfloat16* yr = xb + (int64_t)r * H;
@@ -161,6 +172,8 @@ __global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict_
 
 __global__ void argmax_reduce_kernel(const float* __restrict__ pv, const int32_t* __restrict__ pi, int rows,
                                      int ntiles, int32_t* out) {
+  pdl_trigger();
+  pdl_wait();
   const int r = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
   const int l = threadIdx.x & 31;
   if (r >= rows) return;
@@ -193,6 +206,14 @@ int grid_for(int64_t n, int threads) {
 
 }  // namespace
 
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("GLLM_PDL");
+    return e != nullptr && e[0] == '1';
+  }();
+  return on;
+}
+
 void launch_init_bf16(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid, float scale,
                       int mode, int64_t row_offset, cudaStream_t s) {
   init_bf16_kernel<<<grid_for(rows * cols, 256), 256, 0, s>>>(dst, rows, cols, seed, tid, scale, mode, row_offset);
@@ -210,26 +231,26 @@ void launch_prep(const int32_t* positions, const int32_t* cu_q, const int32_t* b
                  int maxblk, int block_size, int32_t* slots, float2* rope_cs, int head_dim, float rope_theta,
                  cudaStream_t s) {
   if (T <= 0) return;
-  prep_kernel<<<T, 64, 0, s>>>(positions, cu_q, block_table, T, S, maxblk, block_size, slots, rope_cs,
-                               head_dim / 2, log2((double)rope_theta));
+  launch_pdl(prep_kernel, dim3(T), dim3(64), 0, s, 1, positions, cu_q, block_table, T, S, maxblk, block_size, slots, rope_cs,
+             head_dim / 2, log2((double)rope_theta));
 }
 void launch_embed(const __nv_bfloat16* E, const int32_t* ids, float* x, int T, int H, cudaStream_t s) {
   if (T <= 0) return;
-  embed_kernel<<<T, 128, 0, s>>>(E, ids, x, H);
+  launch_pdl(embed_kernel, dim3(T), dim3(128), 0, s, 1, E, ids, x, H);
 }
 void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int32_t* rows, int n, int H, float eps,
                     cudaStream_t s) {
   if (n <= 0) return;
-  rmsnorm_kernel<<<n, 256, 0, s>>>(x, g, y, rows, H, eps);
+  launch_pdl(rmsnorm_kernel, dim3(n), dim3(256), 0, s, 1, x, g, y, rows, H, eps);
 }
 void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s) {
   if (n <= 0) return;
-  rms_stats_kernel<<<n, 256, 0, s>>>(x, xb, ss, H);
+  launch_pdl(rms_stats_kernel, dim3(n), dim3(256), 0, s, 1, x, xb, ss, H);
 }
 void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,
                           cudaStream_t s) {
   if (rows <= 0) return;
-  argmax_reduce_kernel<<<(rows + 3) / 4, 128, 0, s>>>(part_val, part_idx, rows, ntiles, out);
+  launch_pdl(argmax_reduce_kernel, dim3((rows + 3) / 4), dim3(128), 0, s, 1, part_val, part_idx, rows, ntiles, out);
 }
 
 }  // namespace gllm

@@ -223,6 +223,7 @@ bool Prof::g_sync_debug = std::getenv("GLLM_SYNC_DEBUG") != nullptr;
 int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmEpi epi, int M, int N, int K,
          void* out, int ldo, const float* bias, cudaStream_t s) {
   gllm::GemmArgs g{};
+  g.b_static = 1;
   g.M = M;
   g.N = N;
   g.K = K;
@@ -678,6 +679,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     // ss_next was zeroed by the n-tile-0 epilogue of the preceding consumer GEMM (zero_rows)
     const bool sk = !fused || gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
     gllm::GemmArgs g{};
+  g.b_static = 1;
     g.M = T;
     g.N = H;
     g.K = K;
@@ -703,6 +705,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       // QKV projection with RoPE and the paged KV append fused into the epilogue (a5 + a6)
       Prof p(st, s, C_QKV);
       gllm::GemmArgs g{};
+  g.b_static = 1;
       g.M = T;
       g.N = nqkv;
       g.K = H;
@@ -776,6 +779,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     {
       Prof p(st, s, C_GU);
       gllm::GemmArgs g{};
+  g.b_static = 1;
       g.M = T;
       g.N = 2 * I;
       g.K = H;

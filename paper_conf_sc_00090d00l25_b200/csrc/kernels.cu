@@ -208,8 +208,8 @@ int grid_for(int64_t n, int threads) {
 
 bool pdl_enabled() {
   static const bool on = [] {
-    const char* e = std::getenv("GLLM_PDL");
-    return e != nullptr && e[0] == '1';
+    const char* e = std::getenv("GLLM_PDL");  // default on (A/B: profiles/r01/s4b)
+    return e == nullptr || e[0] != '0';
   }();
   return on;
 }

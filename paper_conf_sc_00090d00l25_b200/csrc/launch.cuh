@@ -8,8 +8,8 @@
 // before griddepcontrol.wait, which returns once every prerequisite grid has COMPLETED and its
 // memory is visible. Every thread that touches global memory executes the wait first, so the
 // ordering is the same as a plain stream; only launch latency and prologue overlap the
-// predecessor's tail. GLLM_PDL=1 enables it, GLLM_PDL=0 gives plain stream serialisation (the
-// device-side instructions are then no-ops).
+// predecessor's tail. On by default; GLLM_PDL=0 gives plain stream serialisation (the device-side
+// instructions are then no-ops).
 #pragma once
 #include <cuda_runtime.h>
 
@@ -20,7 +20,7 @@ namespace gllm {
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
-bool pdl_enabled();  // GLLM_PDL, read once per process (see kernels.cu for the default)
+bool pdl_enabled();  // GLLM_PDL (default on), read once per process
 
 // cudaLaunchKernelEx with the PDL attribute (when enabled) and an optional cluster shape.
 template <typename... KArgs, typename... Args>

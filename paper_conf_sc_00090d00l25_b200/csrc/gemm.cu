@@ -684,6 +684,14 @@ __device__ __forceinline__ void ld_f32x32(const float* src, float (&v)[32]) {  /
   }
 }
 
+// the finish pass leaves the workspace zero for the next stream-K launch (no memset launch, so the
+// PDL chain runs unbroken from the producing kernel into the GEMM)
+__device__ __forceinline__ void zero_f32x32(const float* p) {
+  float4* d = reinterpret_cast<float4*>(const_cast<float*>(p));
+#pragma unroll
+  for (int q = 0; q < 8; ++q) d[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
 template <int EPI>
 __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
   pdl_trigger();
@@ -698,6 +706,7 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
   if constexpr (EPI == EPI_STORE_BF16) {
     float v[32];
     ld_f32x32(w + c * 32, v);
+    zero_f32x32(w + c * 32);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] = v[j] * rs + (p.bias ? p.bias[c * 32 + j] : 0.f);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, v);
@@ -708,6 +717,8 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
     float h[32], uv[32];
     ld_f32x32(g, h);
     ld_f32x32(u, uv);
+    zero_f32x32(g);
+    zero_f32x32(u);
 #pragma unroll
     for (int j = 0; j < 32; ++j) h[j] = silu_f(h[j] * rs) * (uv[j] * rs);
     store_bf16x32(reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo + c * 32, h);
@@ -718,6 +729,8 @@ __global__ void __launch_bounds__(256) gemm_finish_kernel(const GemmArgs p) {
     float x1[32], x2[32];
     ld_f32x32(w + col1, x1);
     ld_f32x32(w + col1 + half, x2);
+    zero_f32x32(w + col1);
+    zero_f32x32(w + col1 + half);
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
       x1[j] = x1[j] * rs + (p.bias ? p.bias[col1 + j] : 0.f);
@@ -876,10 +889,6 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
     grid = (ntiles < units ? ntiles : units) * CG;
   }
   if (grid <= 0) return GLLM_OK;
-  if (args.ws && !args.tile_ctr) {
-    cudaError_t e = cudaMemsetAsync(args.ws, 0, (size_t)args.M * args.N * sizeof(float), stream);
-    if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm workspace memset: %s", cudaGetErrorString(e));
-  }
   {
     cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, CG, a, b, args);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (%d-CTA) launch: %s", CG, cudaGetErrorString(e));

@@ -42,7 +42,7 @@ struct GemmArgs {
   float* ws;
   // stream-K fixup counters (>= tiles ints).  Non-null: ws and tile_ctr are all zero on entry and
   // the kernel leaves them zero (the last segment of each tile finishes it in-kernel); null: ws
-  // is zeroed before and gemm_finish_kernel applies the epilogue after.
+  // is zero on entry too, and gemm_finish_kernel applies the epilogue and clears what it read.
   int* tile_ctr;
   // fused RMSNorm (a4).  Consumers (EPI_STORE_BF16 / EPI_QKV_ROPE / EPI_SILU_MUL) read the bf16
   // copy of the residual as A and scale each output row by r = rsqrt(row_ss[row] * inv_h + eps)

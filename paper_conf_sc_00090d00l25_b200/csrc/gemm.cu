@@ -672,11 +672,13 @@ __global__ void __launch_bounds__(256, 1)
 
 // Workspace mode: apply the non-additive epilogue to the fp32 sums in ws [M, N].
 // One thread per (row, 32-column chunk) of the OUTPUT space of the epilogue.
+// Plain (coherent) loads, not __ldg: the finish pass clears the same words after reading them, and
+// a read-only load may legally be reordered after those stores.
 __device__ __forceinline__ void ld_f32x32(const float* src, float (&v)[32]) {  // 8 x 16-B loads
   const float4* s4 = reinterpret_cast<const float4*>(src);
 #pragma unroll
   for (int q = 0; q < 8; ++q) {
-    const float4 x = __ldg(s4 + q);
+    const float4 x = s4[q];
     v[4 * q] = x.x;
     v[4 * q + 1] = x.y;
     v[4 * q + 2] = x.z;

@@ -1,7 +1,7 @@
 """Programmatic dependent launch (csrc/launch.cuh): the stage path must agree with the oracle with
-PDL on and off.  GLLM_PDL is read once per process, so each mode runs the parity cases that span
-the GEMM schedules (stream-K, hybrid, whole tiles), both attention kernels and the LM head in a
-child pytest process."""
+PDL on and off.  PDL is on by default, so the rest of the -m gpu suite covers it; GLLM_PDL is read
+once per process, so the PDL-off mode runs parity cases spanning the GEMM schedules (stream-K,
+whole tiles), both attention kernels and chunked prefill in a child pytest process."""
 import os
 import subprocess
 import sys
@@ -10,12 +10,12 @@ import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
-CASES = "c0_mixed_batch or c0b_chunked or gqa_bias or c1_stream_long_chunk or c3_long_prompt or c1_last_stage"
+CASES = "c0_mixed_batch or c0b_chunked or gqa_bias or c1_stream_long_chunk"
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("mode", ["0", "1"])
-def test_stage_parity_with_and_without_pdl(mode):
+@pytest.mark.parametrize("mode", ["0"])
+def test_stage_parity_without_pdl(mode):
     env = dict(os.environ, GLLM_PDL=mode)
     r = subprocess.run(
         [sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-p", "no:cacheprovider",

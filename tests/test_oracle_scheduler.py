@@ -318,3 +318,16 @@ def test_ctx_policy_invariants_and_long_prompts():
     s, total_p = _check_invariants(cfg, st, max_ticks=None)
     assert s.done() and total_p == sum(r.prompt_len for r in st.requests)
     assert sorted(s.free) == list(range(cfg.num_blocks))
+
+
+@pytest.mark.parametrize("name", ["w1_trace.txt", "p1_preempt_order.txt", "p2_preempt_inflight.txt",
+                                  "s1_sarathi.txt", "ws1_warm.txt"])
+def test_hand_worked_goldens(name):
+    # hand-worked traces (tests/golden/, derivations in their headers): preemption victim order and
+    # in-flight exclusion (R14, L127/L165/L325), Sarathi-Serve (L81/L125/L310), warm start (C4)
+    from oracle.scheduler import trace_bytes
+    from tests.golden_traces import CASES, compare
+    cfg, st = CASES[name]
+    s, batches = run(cfg, st)
+    compare([trace_bytes(b) for b in batches], name)
+    assert sorted(s.free) == list(range(cfg.num_blocks))

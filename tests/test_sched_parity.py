@@ -137,3 +137,18 @@ def test_ctx_policy_identical():
               make_stream("C1", 1000, n=100))
     with pytest.raises(gllm.GllmError):
         gllm.Sched(SchedParams(num_blocks=100, policy=4, attn_pairs_per_token=0))
+
+
+@pytest.mark.parametrize("name", ["w1_trace.txt", "p1_preempt_order.txt", "p2_preempt_inflight.txt",
+                                  "s1_sarathi.txt", "ws1_warm.txt"])
+def test_library_matches_hand_worked_goldens(name):
+    # the C++ scheduler against the hand-worked traces directly (not only against the oracle)
+    from tests.golden_traces import CASES, compare
+    cfg, st = CASES[name]
+    c = gllm.Sched(cfg)
+    c.add_stream(st)
+    traces = []
+    while not c.done():
+        c.build_batch()
+        traces.append(c.trace())
+    compare(traces, name)

@@ -219,7 +219,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     from paper_conf_sc_00090d00l25_b200 import gllm
-    from paper_conf_sc_00090d00l25_b200.runtime import (GpuExecutor, NcclTransport, Pipeline, pack_desc,
+    from paper_conf_sc_00090d00l25_b200.runtime import (GpuExecutor, NcclTransport, Pipeline, fill_warm, pack_desc,
                                                         split_layers, unpack_desc)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -242,12 +242,12 @@ def run_ours(args):
     lb, le = split_layers(m.n_layers, PP)[sidx]
     max_tokens = sp.maxp + -(-sp.max_seqs // PP) + 64
     stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=local)
-    ex = GpuExecutor(stage, dev, max_tokens, m.hidden)
+    ex = GpuExecutor(stage, dev, max_tokens, m.hidden, pp=PP)
     if emulate and sidx > 0:
         for b in ex.hin:
             b.normal_()                       # synthetic activations arriving from stage sidx-1
-    if args.config == "C4":
-        stage.fill_kv(0xC4)                   # warm-start decode set: cache pages hold O4 values
+    stream = make_stream(args.config, m.vocab)
+    fill_warm(stage, sp, stream.warm)         # C4 warm-start decode set: its cache pages hold the O4 values
     tr = None
     if world > 1:
         if args.handoff == "peer":   # fused hand-off over NVLink peer memory (gllm_peer_*)
@@ -259,7 +259,6 @@ def run_ours(args):
             stage.comm_init(uid[0], rank, world)
             tr = NcclTransport(ex, rank, world)
     sched = None
-    stream = make_stream(args.config, m.vocab)
     if rank == 0:
         sched = gllm.Sched(sp)
         sched.add_stream(stream)

@@ -152,6 +152,10 @@ GLLM_API int gllm_sched_done(const gllm_sched* s);
  * [3] preemptions so far, [4] finished requests, [5] requests admitted. */
 GLLM_API int gllm_sched_stats(const gllm_sched* s, int64_t* out6);
 
+/* Block ids of a running (not finished) request, in position order: *n receives the count;
+ * out: host int32 [cap].  EINVAL if the request is unknown or finished, or cap < *n. */
+GLLM_API int gllm_sched_seq_blocks(const gllm_sched* s, int64_t req_id, int32_t* out, int32_t cap, int32_t* n);
+
 /* Canonical little-endian int64 trace of the LAST built tick (layout in
  * DESIGN.md §3; identical to oracle.scheduler.trace_bytes).  *used receives
  * the byte count; EINVAL if cap is too small (then *used is the size needed). */
@@ -247,10 +251,16 @@ GLLM_API int gllm_stage_read_kv(gllm_stage* st, int32_t layer, const int32_t* sl
                        float* k_out, float* v_out);
 /* Device slot mapping produced by the last stage_forward, host int32 [num_tokens]. */
 GLLM_API int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n);
-/* Fills the KV cache of local layer `layer` (or all layers if layer < 0) with the
- * O4-style generator (warm start): element i of K (resp. V) of layer l has
- * tensor id 0xEE0000 + 2*l (+1 for V).  Used by benchmarks for warm decode state. */
-GLLM_API int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed);
+/* Warm start (C4's warm decode set): writes the cached K and V of
+ * positions [0, context_lens[i]) of warm request req_ids[i], for every local layer, through row i of
+ * block_table (host int32 [n_seqs * max_blocks], the blocks the scheduler gave the sequence, see
+ * gllm_sched_seq_blocks).  Values follow O4 with the model's weight seed: K (V) of request r,
+ * position p, layer l, kv head h, dim j is element ((r * 2^17 + p) * n_kv_heads + h) * head_dim + j
+ * of tensor 0xEE0000 + 2l (+1), scale sqrt(3), rounded to bf16 (oracle.weights.warm_kv holds the same
+ * values).  Host arrays are copied; synchronous.  EINVAL for contexts outside [1, 2^17], request ids
+ * outside the 40-bit index range, or block ids >= kv_blocks. */
+GLLM_API int gllm_stage_fill_warm_kv(gllm_stage* st, int32_t n_seqs, const int64_t* req_ids,
+                                     const int32_t* context_lens, const int32_t* block_table, int32_t max_blocks);
 
 /* Timing of the forwards since the previous call, from CUDA events recorded on each forward's own
  * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).  on = 2 also runs the

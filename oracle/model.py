@@ -140,6 +140,13 @@ class PagedCache:
             K[b][o] = k[t]
             V[b][o] = v[t]
 
+    def fill_warm(self, layer, blocks, k, v):
+        """Cached K/V of a warm sequence (O4 warm start): positions [0, len(k)) through its blocks."""
+        n = k.shape[0]
+        pos = np.arange(n)
+        slots = np.asarray(blocks, np.int64)[pos // self.bs] * self.bs + pos % self.bs
+        self.write(layer, slots, k.astype(self.dtype), v.astype(self.dtype))
+
     def gather(self, layer, blocks, n):
         """Keys/values of logical positions [0, n) through a block-table row."""
         K, V = self.k[layer], self.v[layer]

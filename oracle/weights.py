@@ -67,6 +67,42 @@ def gen(seed: int, t: int, n: int, scale: np.float32, start: int = 0) -> np.ndar
     return bf16_rne(x * np.float32(scale))
 
 
+# Warm-start KV (SURVEY.md §8(c) O4 last item; C4's warm decode set, §8(d)): K and V of warm request r at
+# position p, layer l, kv head h, dim j are element i = ((r * 2^17 + p) * Hkv + h) * D + j of tensor
+# T_WARM_K + 2 l (K) / T_WARM_K + 2 l + 1 (V), scale sqrt(3) (sigma 1, the size of a RoPE'd k of a
+# unit-rms input under 1/sqrt(H) weights).  Needs p < 2^17 and (r * 2^17 + p) * Hkv * D < 2^40.
+T_WARM_K = 0xEE0000
+WARM_POS_BITS = 17
+
+
+def warm_kv(seed: int, req_id: int, context_len: int, layer: int, n_kv_heads: int, head_dim: int):
+    """(K, V) [context_len, n_kv_heads, head_dim] of a warm sequence at one layer (fp32 holding bf16)."""
+    assert context_len <= (1 << WARM_POS_BITS)
+    per_pos = n_kv_heads * head_dim
+    start = (req_id << WARM_POS_BITS) * per_pos
+    assert start + context_len * per_pos <= (1 << 40)
+    s = scale_for("embed")
+    k = gen(seed, T_WARM_K + 2 * layer, context_len * per_pos, s, start)
+    v = gen(seed, T_WARM_K + 2 * layer + 1, context_len * per_pos, s, start)
+    return k.reshape(context_len, n_kv_heads, head_dim), v.reshape(context_len, n_kv_heads, head_dim)
+
+
+def gen_threads(seed: int, t: int, n: int, scale: np.float32, start: int = 0, chunk: int = 1 << 22) -> np.ndarray:
+    """`gen` over [start, start+n) in independent chunks on a thread pool (numpy releases the GIL in
+    its ufuncs); element for element identical to one `gen` call (counter-based)."""
+    if n <= chunk:
+        return gen(seed, t, n, scale, start)
+    from concurrent.futures import ThreadPoolExecutor
+    out = np.empty(n, np.float32)
+
+    def one(o):
+        m = min(chunk, n - o)
+        out[o:o + m] = gen(seed, t, m, scale, start + o)
+    with ThreadPoolExecutor() as ex:
+        list(ex.map(one, range(0, n, chunk)))
+    return out
+
+
 def layer_tid(layer: int, kind: str) -> int:
     return 1 + 16 * layer + KIND[kind]
 
@@ -82,7 +118,7 @@ class Weights:
     def _mat(self, t, rows, cols, scale):
         key = (t, rows, cols)
         if key not in self._cache:
-            self._cache[key] = gen(self.m.weight_seed, t, rows * cols, scale).reshape(rows, cols).astype(self.dtype)
+            self._cache[key] = gen_threads(self.m.weight_seed, t, rows * cols, scale).reshape(rows, cols).astype(self.dtype)
         return self._cache[key]
 
     def layer(self, l: int) -> dict:

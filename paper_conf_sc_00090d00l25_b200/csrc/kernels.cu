@@ -52,10 +52,26 @@ __global__ void fill_f32_kernel(float* dst, int64_t n, float v) {
     dst[i] = v;
 }
 
-__global__ void fill_kv_kernel(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, uint64_t seed, uint64_t tid) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    kc[i] = __float2bfloat16_rn(o4(seed, tid, (uint64_t)i, 1.7320508f));
-    vc[i] = __float2bfloat16_rn(o4(seed, tid + 1, (uint64_t)i, 1.7320508f));
+// Warm-start KV (O4): K / V of warm request r at position p, kv head h, dim j hold
+// element ((r * 2^17 + p) * Hkv + h) * D + j of tensor tid / tid + 1 (scale sqrt(3)), written through
+// the sequence's block table.  One CTA per (page, sequence); pages past the context are skipped.
+__global__ void fill_warm_kv_kernel(__nv_bfloat16* kc, __nv_bfloat16* vc, const int64_t* __restrict__ req_ids,
+                                    const int32_t* __restrict__ ctx, const int32_t* __restrict__ bt, int maxblk,
+                                    int Hkv, int D, int bs, uint64_t seed, uint64_t tid) {
+  const int seq = blockIdx.y, page = blockIdx.x;
+  const int n = ctx[seq];
+  const int p0 = page * bs;
+  if (p0 >= n) return;
+  const int np = min(bs, n - p0);
+  const int64_t blk = bt[(int64_t)seq * maxblk + page];
+  const uint64_t base = ((uint64_t)req_ids[seq] << 17);
+  const int per_pos = Hkv * D;
+  for (int e = threadIdx.x; e < np * per_pos; e += blockDim.x) {
+    const int o = e / per_pos, hd = e - o * per_pos, h = hd / D, j = hd - h * D;
+    const uint64_t i = (base + (uint64_t)(p0 + o)) * (uint64_t)per_pos + (uint64_t)hd;
+    const int64_t dst = ((blk * Hkv + h) * bs + o) * (int64_t)D + j;
+    kc[dst] = __float2bfloat16_rn(o4(seed, tid, i, 1.7320508f));
+    vc[dst] = __float2bfloat16_rn(o4(seed, tid + 1, i, 1.7320508f));
   }
 }
 
@@ -224,8 +240,11 @@ void launch_init_f32(float* dst, int64_t n, uint64_t seed, uint64_t tid, float s
 void launch_fill_f32(float* dst, int64_t n, float v, cudaStream_t s) {
   fill_f32_kernel<<<grid_for(n, 256), 256, 0, s>>>(dst, n, v);
 }
-void launch_fill_kv(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, uint64_t seed, uint64_t tid, cudaStream_t s) {
-  fill_kv_kernel<<<grid_for(n, 256), 256, 0, s>>>(kc, vc, n, seed, tid);
+void launch_fill_warm_kv(__nv_bfloat16* kc, __nv_bfloat16* vc, const int64_t* req_ids, const int32_t* ctx,
+                         const int32_t* bt, int n_seqs, int maxblk, int Hkv, int D, int bs, uint64_t seed,
+                         uint64_t tid, cudaStream_t s) {
+  if (n_seqs == 0 || maxblk == 0) return;
+  fill_warm_kv_kernel<<<dim3(maxblk, n_seqs), 256, 0, s>>>(kc, vc, req_ids, ctx, bt, maxblk, Hkv, D, bs, seed, tid);
 }
 void launch_prep(const int32_t* positions, const int32_t* cu_q, const int32_t* block_table, int T, int S,
                  int maxblk, int block_size, int32_t* slots, float2* rope_cs, int head_dim, float rope_theta,

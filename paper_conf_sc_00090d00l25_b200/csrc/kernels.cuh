@@ -37,7 +37,10 @@ void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H
 void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,
                           cudaStream_t s);
 
-// warm KV fill (benchmarks): element i of K / V of a layer gets the O4 value of tensor id tid / tid+1
-void launch_fill_kv(__nv_bfloat16* kc, __nv_bfloat16* vc, int64_t n, uint64_t seed, uint64_t tid, cudaStream_t s);
+// warm-start KV (O4): positions [0, ctx[i]) of warm request req_ids[i] through block-table row i,
+// K / V of one layer from tensor ids tid / tid + 1 (device arrays)
+void launch_fill_warm_kv(__nv_bfloat16* kc, __nv_bfloat16* vc, const int64_t* req_ids, const int32_t* ctx,
+                         const int32_t* bt, int n_seqs, int maxblk, int Hkv, int D, int bs, uint64_t seed,
+                         uint64_t tid, cudaStream_t s);
 
 }  // namespace gllm

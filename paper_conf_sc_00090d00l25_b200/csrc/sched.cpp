@@ -238,11 +238,14 @@ void preempt(gllm_sched* s, Req* v) {
     if (it != s->readyq.end()) s->readyq.erase(it);
   }
   s->wp -= v->prefill_len - v->sched_prompt;
+  // a victim still waiting (partially prefilled, not in flight) keeps its valid queue entry; a
+  // decode-phase victim's entry (if any) is stale and waitq_insert re-validates it
+  const bool valid_entry = v->in_waitq && v->waiting();
   s->release(v);
   v->prefill_len = v->orig_len + v->gen;
   v->sched_prompt = v->done_prompt = 0;
   s->wp += v->prefill_len;
-  s->waitq_insert(v);
+  if (!valid_entry) s->waitq_insert(v);
   s->preemptions += 1;
 }
 
@@ -560,6 +563,21 @@ int gllm_sched_stats(const gllm_sched* s, int64_t* out6) {
   out6[4] = s->finished;
   out6[5] = s->admitted_total;
   return GLLM_OK;
+}
+
+int gllm_sched_seq_blocks(const gllm_sched* s, int64_t req_id, int32_t* out, int32_t cap, int32_t* n) {
+  GLLM_TRY_BEGIN
+  if (!s || !n || (cap > 0 && !out)) return gllm::set_error(GLLM_EINVAL, "null argument");
+  for (const auto& r : s->storage) {
+    if (r->id != req_id) continue;
+    if (r->finished) break;
+    *n = (int32_t)r->blocks.size();
+    if (*n > cap) return gllm::set_error(GLLM_EINVAL, "seq_blocks: cap %d < %d blocks", cap, *n);
+    std::memcpy(out, r->blocks.data(), r->blocks.size() * sizeof(int32_t));
+    return GLLM_OK;
+  }
+  return gllm::set_error(GLLM_EINVAL, "seq_blocks: request %lld not running", (long long)req_id);
+  GLLM_TRY_END
 }
 
 int gllm_sched_trace(gllm_sched* s, void* buf, size_t cap, size_t* used) {

@@ -612,8 +612,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
   if (!st->is_first() && !hidden_in) return gllm::set_error(GLLM_EINVAL, "hidden_in required on stage > 0");
   if (!st->is_last() && !hidden_out && !peer_out)
     return gllm::set_error(GLLM_EINVAL, "hidden_out required before the last stage");
+  CK(cudaSetDevice(st->device));  // before ensure_parts: its buffers belong to the stage's device
   RC(ensure_parts(st, P.nparts));
-  CK(cudaSetDevice(st->device));
   CK(cudaStreamWaitEvent(s, P.copied, 0));
   Prof p_total(st, s, C_TOTAL);
   uint8_t* m = P.dev;
@@ -1017,17 +1017,48 @@ int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n) {
   return GLLM_OK;
 }
 
-int gllm_stage_fill_kv(gllm_stage* st, int32_t layer, uint64_t seed) {
-  if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
-  cudaSetDevice(st->device);
-  const size_t n = (size_t)st->kv_blocks * st->cfg.n_kv_heads * st->bs * st->cfg.head_dim;
-  for (int l = st->lb; l < st->le; ++l) {
-    if (layer >= 0 && l != layer) continue;
-    LayerW& w = st->layers[l - st->lb];
-    gllm::launch_fill_kv(w.kc, w.vc, n, seed, 0xEE0000ull + 2 * (uint64_t)l, 0);
+int gllm_stage_fill_warm_kv(gllm_stage* st, int32_t n_seqs, const int64_t* req_ids, const int32_t* context_lens,
+                            const int32_t* block_table, int32_t max_blocks) {
+  GLLM_TRY_BEGIN
+  if (!st || n_seqs < 0 || max_blocks < 0 || (n_seqs && (!req_ids || !context_lens || !block_table)))
+    return gllm::set_error(GLLM_EINVAL, "fill_warm_kv: bad arguments");
+  if (n_seqs == 0) return GLLM_OK;
+  const int Hkv = st->cfg.n_kv_heads, D = st->cfg.head_dim, bs = st->bs;
+  for (int i = 0; i < n_seqs; ++i) {
+    const int n = context_lens[i];
+    if (n < 1 || n > (1 << 17) || (n + bs - 1) / bs > max_blocks)
+      return gllm::set_error(GLLM_EINVAL, "fill_warm_kv: seq %d context %d", i, n);
+    if (req_ids[i] < 0 || ((uint64_t)(req_ids[i] + 1) << 17) * (uint64_t)(Hkv * D) > (1ull << 40))
+      return gllm::set_error(GLLM_EINVAL, "fill_warm_kv: request id %lld out of the O4 index range", (long long)req_ids[i]);
+    for (int j = 0; j < (n + bs - 1) / bs; ++j) {
+      const int b = block_table[(size_t)i * max_blocks + j];
+      if (b < 0 || b >= st->kv_blocks) return gllm::set_error(GLLM_EINVAL, "fill_warm_kv: block id %d", b);
+    }
   }
-  CK(cudaDeviceSynchronize());
+  CK(cudaSetDevice(st->device));
+  int64_t* d_req = nullptr;
+  int32_t *d_ctx = nullptr, *d_bt = nullptr;
+  const size_t bt_n = (size_t)n_seqs * max_blocks;
+  CK(cudaMalloc(&d_req, n_seqs * sizeof(int64_t)));
+  cudaError_t e = cudaMalloc(&d_ctx, n_seqs * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&d_bt, bt_n * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMemcpy(d_req, req_ids, n_seqs * sizeof(int64_t), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d_ctx, context_lens, n_seqs * sizeof(int32_t), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d_bt, block_table, bt_n * sizeof(int32_t), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) {
+    for (int l = st->lb; l < st->le; ++l) {
+      LayerW& w = st->layers[l - st->lb];
+      gllm::launch_fill_warm_kv(w.kc, w.vc, d_req, d_ctx, d_bt, n_seqs, max_blocks, Hkv, D, bs, st->cfg.weight_seed,
+                                0xEE0000ull + 2 * (uint64_t)l, 0);
+    }
+    e = cudaDeviceSynchronize();
+  }
+  cudaFree(d_req);
+  cudaFree(d_ctx);
+  cudaFree(d_bt);
+  if (e != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "fill_warm_kv: %s", cudaGetErrorString(e));
   return GLLM_OK;
+  GLLM_TRY_END
 }
 
 }  // extern "C"

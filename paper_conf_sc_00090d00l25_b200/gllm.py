@@ -113,7 +113,8 @@ def lib():
             "gllm_stage_read_weight": ([vp, i32, C.c_char_p, i64, i64, C.POINTER(C.c_float)], C.c_int),
             "gllm_stage_read_kv": ([vp, i32, _P32, i32, C.POINTER(C.c_float), C.POINTER(C.c_float)], C.c_int),
             "gllm_stage_read_slots": ([vp, _P32, i32], C.c_int),
-            "gllm_stage_fill_kv": ([vp, i32, u64], C.c_int),
+            "gllm_stage_fill_warm_kv": ([vp, i32, C.POINTER(C.c_int64), _P32, _P32, i32], C.c_int),
+            "gllm_sched_seq_blocks": ([vp, i64, _P32, i32, _P32], C.c_int),
             "gllm_stage_set_profiling": ([vp, i32], C.c_int),
             "gllm_stage_last_timing": ([vp, C.POINTER(C.c_float), i32], C.c_int),
             "gllm_stage_last_launches": ([vp, _P32], C.c_int),
@@ -204,6 +205,14 @@ class Sched:
         out = (C.c_int64 * 6)()
         _check(lib().gllm_sched_stats(self.h, out))
         return dict(zip(["tick", "running", "free_blocks", "preemptions", "finished", "admitted"], list(out)))
+
+    def seq_blocks(self, req_id) -> np.ndarray:
+        n = C.c_int32()
+        rc = lib().gllm_sched_seq_blocks(self.h, req_id, None, 0, C.byref(n))
+        out = np.zeros(max(n.value, 1), np.int32)
+        if rc != 0:
+            _check(lib().gllm_sched_seq_blocks(self.h, req_id, _p32(out), out.shape[0], C.byref(n)))
+        return out[: n.value]
 
     def trace(self) -> bytes:
         used = C.c_size_t()
@@ -327,8 +336,15 @@ class Stage:
         _check(lib().gllm_stage_read_slots(self.h, _p32(out), n))
         return out
 
-    def fill_kv(self, seed, layer=-1):
-        _check(lib().gllm_stage_fill_kv(self.h, layer, seed))
+    def fill_warm_kv(self, req_ids, context_lens, block_table):
+        """gllm_stage_fill_warm_kv: block_table int32 [n, max_blocks] (rows -1 padded)."""
+        rid = np.ascontiguousarray(req_ids, dtype=np.int64)
+        ctx = np.ascontiguousarray(context_lens, dtype=np.int32)
+        bt = np.ascontiguousarray(block_table, dtype=np.int32)
+        n = int(rid.shape[0])
+        mb = int(bt.shape[1]) if bt.ndim == 2 else 0
+        _check(lib().gllm_stage_fill_warm_kv(self.h, n, rid.ctypes.data_as(C.POINTER(C.c_int64)), _p32(ctx),
+                                             _p32(bt), mb))
 
     # pipeline hand-off (NCCL P2P)
     def comm_init(self, unique_id: bytes, rank: int, world: int):

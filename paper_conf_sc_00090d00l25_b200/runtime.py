@@ -33,6 +33,22 @@ def split_layers(n_layers: int, world: int):
     return out
 
 
+def fill_warm(stage, sched_cfg, warm) -> None:
+    """Warm-start KV of a warm decode set (C4, O4 values): the blocks each warm sequence holds are
+    those the scheduler allocates at add_warm (lowest first, in list order, before any request), so a
+    scheduler holding only the warm set reproduces them on every rank."""
+    if not warm:
+        return
+    s = gllm.Sched(sched_cfg)
+    for w in warm:
+        s.add_warm(w.req_id, w.context_len, w.remaining_out, w.token_ids)
+    rows = [s.seq_blocks(w.req_id) for w in warm]
+    bt = np.full((len(rows), max(len(r) for r in rows)), -1, np.int32)
+    for i, r in enumerate(rows):
+        bt[i, :len(r)] = r
+    stage.fill_warm_kv([w.req_id for w in warm], [w.context_len for w in warm], bt)
+
+
 def pack_desc(d) -> np.ndarray:
     """Flatten a BatchDesc (or its to_numpy() dict) into one int32 buffer for the broadcast."""
     a = d.to_numpy() if hasattr(d, "to_numpy") else d
@@ -72,7 +88,7 @@ def unpack_desc(buf: np.ndarray) -> dict:
 class GpuExecutor:
     """Product executor: a gllm.Stage on this rank's GPU; buffers are torch CUDA tensors."""
 
-    def __init__(self, stage: "gllm.Stage", device, max_tokens, hidden):
+    def __init__(self, stage: "gllm.Stage", device, max_tokens, hidden, pp=1):
         import torch
         self.torch = torch
         self.stage = stage
@@ -81,10 +97,14 @@ class GpuExecutor:
         self.comm = torch.cuda.Stream(device=device)
         self.hin = [torch.empty((max_tokens, hidden), dtype=torch.float32, device=device) for _ in range(2)]
         self.hout = [torch.empty((max_tokens, hidden), dtype=torch.float32, device=device) for _ in range(2)]
-        self.samp = [torch.empty((max(stage.max_seqs, 1),), dtype=torch.int32, device=device) for _ in range(4)]
+        # sampled ids of batch k are read PP-1 (last stage, world > 1) or PP (one-GPU emulation) ticks
+        # later, so the ring holds more than PP batches
+        self.nsamp = max(4, 2 * pp + 2)
+        self.samp = [torch.empty((max(stage.max_seqs, 1),), dtype=torch.int32, device=device)
+                     for _ in range(self.nsamp)]
         self.samp_host = [torch.empty((max(stage.max_seqs, 1),), dtype=torch.int32, pin_memory=True)
-                          for _ in range(4)]
-        self.samp_ev = [torch.cuda.Event() for _ in range(4)]
+                          for _ in range(self.nsamp)]
+        self.samp_ev = [torch.cuda.Event() for _ in range(self.nsamp)]
         self.fwd_ev = [torch.cuda.Event() for _ in range(2)]
         self.recv_ev = [torch.cuda.Event() for _ in range(2)]
         self.send_ev = [torch.cuda.Event() for _ in range(2)]
@@ -118,17 +138,20 @@ class GpuExecutor:
         else:
             if not is_last:
                 self.compute.wait_event(self.send_ev[i])   # send k-2 finished reading hout[i]
+            j = k % self.nsamp
             self.stage.forward_prepared(h, hin, 0 if is_last else self.hout[i].data_ptr(),
-                                        self.samp[k & 3].data_ptr() if is_last else 0, cs)
+                                        self.samp[j].data_ptr() if is_last else 0, cs)
         self.fwd_ev[i].record(self.compute)
         if is_last and ns:
+            j = k % self.nsamp
             with self.torch.cuda.stream(self.compute):
-                self.samp_host[k & 3][:ns].copy_(self.samp[k & 3][:ns], non_blocking=True)
-            self.samp_ev[k & 3].record(self.compute)
+                self.samp_host[j][:ns].copy_(self.samp[j][:ns], non_blocking=True)
+            self.samp_ev[j].record(self.compute)
 
     def sampled(self, k, ns) -> np.ndarray:
-        self.samp_ev[k & 3].synchronize()
-        return self.samp_host[k & 3][:ns].numpy().copy()
+        j = k % self.nsamp
+        self.samp_ev[j].synchronize()
+        return self.samp_host[j][:ns].numpy().copy()
 
 
 class NcclTransport:

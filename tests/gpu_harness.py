@@ -5,7 +5,7 @@ import torch
 
 from oracle import model as om
 from oracle.scheduler import Scheduler
-from oracle.weights import Weights
+from oracle.weights import Weights, warm_kv
 from paper_conf_sc_00090d00l25_b200 import gllm
 
 TOL_HIDDEN = 2e-2   # north_star: max relative error 2e-2 (reading: per-row inf-norm, stage-local)
@@ -36,6 +36,12 @@ class GpuRun:
         self.stage = gllm.Stage(shape, lb, le, kv_blocks or sched_cfg.num_blocks, mt,
                                 max_seqs or min(sched_cfg.max_seqs, mt))
         self.dev = torch.device("cuda", 0)
+        if stream.warm:   # warm-start KV (O4) through the blocks the C++ scheduler gave each sequence
+            rows = [self.sched.seq_blocks(w.req_id) for w in stream.warm]
+            bt = np.full((len(rows), max(len(r) for r in rows)), -1, np.int32)
+            for i, r in enumerate(rows):
+                bt[i, :len(r)] = r
+            self.stage.fill_warm_kv([w.req_id for w in stream.warm], [w.context_len for w in stream.warm], bt)
 
     def step(self, hidden_in=None):
         d = self.sched.build_batch()
@@ -67,6 +73,11 @@ class OracleRun:
         self.sched = Scheduler(sched_cfg, stream.requests, stream.warm)
         self.W = Weights(shape, dtype=dtype)
         self.cache = om.PagedCache(shape, sched_cfg.block_size, dtype)
+        by_id = {r.req_id: r for r in self.sched.admitted}
+        for w in stream.warm:   # the same O4 warm K/V in the oracle's own cache
+            for l in range(self.lb, self.le):
+                k, v = warm_kv(shape.weight_seed, w.req_id, w.context_len, l, shape.n_kv_heads, shape.head_dim)
+                self.cache.fill_warm(l, by_id[w.req_id].blocks, k, v)
 
     def step(self, hidden_in=None, hin_fn=None):
         b = self.sched.build_batch()

@@ -17,7 +17,7 @@ pytestmark = pytest.mark.gpu
 GQA_GPU = ModelShape("gqa-bias-gpu", 2, 256, 4, 2, 64, 512, 512, 1e-5, 10000.0, True, 77)
 
 
-def _run_pair(shape, cfg, stream, lb=0, le=None, max_ticks=None, kv_blocks=None, check_kv=True):
+def _run_pair(shape, cfg, stream, lb=0, le=None, max_ticks=None, kv_blocks=None, check_kv=True, tick_hook=None):
     g = GpuRun(shape, cfg, stream, lb, le, kv_blocks=kv_blocks)
     o = OracleRun(shape, cfg, stream, lb, le)
     n_rows, errs, greedy = 0, [], []
@@ -28,6 +28,8 @@ def _run_pair(shape, cfg, stream, lb=0, le=None, max_ticks=None, kv_blocks=None,
         gb = g.step(ob.get("hidden_in"))
         ticks += 1
         b = ob["batch"]
+        if tick_hook is not None:
+            tick_hook(g, o, b)
         d = gb["desc"]
         assert np.array_equal(d["slot_mapping"], b.slot_mapping)
         if b.num_tokens == 0:
@@ -185,3 +187,65 @@ def test_invalid_batch_is_einval_not_ub():
     with pytest.raises(gllm.GllmError) as ei:
         g.stage.forward(desc, 0, x.data_ptr(), 0, 0)
     assert ei.value.code == -1
+
+
+def _warm_kv_bit_exact(g, o, shape, warm, layers, n_seq=4):
+    # the warm cache itself: GPU bf16 pages == the oracle's O4 values, bit for bit, through the blocks
+    from oracle.weights import warm_kv
+    blocks = {r.req_id: r.blocks for r in o.sched.admitted}
+    for w in warm[:n_seq]:
+        pos = np.arange(w.context_len)
+        bl = np.asarray(blocks[w.req_id], np.int64)
+        slots = (bl[pos // 16] * 16 + pos % 16).astype(np.int32)
+        for l in layers:
+            k, v = g.stage.read_kv(l, slots)
+            kr, vr = warm_kv(shape.weight_seed, w.req_id, w.context_len, l, shape.n_kv_heads, shape.head_dim)
+            assert np.array_equal(k, kr) and np.array_equal(v, vr), (w.req_id, l)
+
+
+def test_c4_warm_start_decode_near_full_kv_last_stage():
+    # C4 (Llama-3-70B shapes: H 8192, I 28672, GQA group 8) warm start as the bench runs it, scaled to
+    # 64 warm decode sequences with contexts U[1536, 2560] whose O4 warm K/V fill >= 90% of the pool,
+    # plus the C4 arrivals (prefill throttled near KV_thresh, Eq.3 UT term / L165).  Last stage: two
+    # layers + final norm + the 128256-wide LM head, so the greedy ids are checked too.
+    m = MODELS["C4"].with_layers(4)
+    full = make_stream("C4", m.vocab, n=12)
+    warm = full.warm[:64]
+    used = sum(-(-w.context_len // 16) for w in warm)
+    nb = int(used / 0.92)
+    st = Stream("C4w", full.requests, warm)
+    cfg = SCHED["C4"].with_(num_blocks=nb, pp_depth=2)
+    kv, ctx = [], []
+
+    def hook(g, o, b):
+        if b.tick == 0:
+            _warm_kv_bit_exact(g, o, m, warm, (2, 3))
+        kv.append(o.sched.kv_used() / nb)
+        ctx.extend(int(x) for x in b.kv_len[len(b.chunks):])
+    n, errs, greedy = _run_pair(m, cfg, st, lb=2, le=4, max_ticks=6, kv_blocks=nb, check_kv=True, tick_hook=hook)
+    assert min(kv) >= 0.9, kv
+    assert max(ctx) >= 2400 and len(ctx) >= 6 * 32, (max(ctx), len(ctx))
+    assert errs.max() <= TOL_HIDDEN, errs.max()
+    assert len(greedy) >= 6 * 32 and greedy.mean() >= 0.99, (len(greedy), greedy.mean())
+
+
+def test_c3_long_context_decode_stage_local():
+    # C3 (Qwen2.5-32B shapes, GQA group 5, q/k/v bias): 40 decode rows at the C3 window's ~4.8k-token
+    # contexts (decode ctx ~4.8k), warm-started from O4 K/V, all in one micro-batch
+    # (PP=1): long split-KV decode work items merged across splits, vs the oracle, one middle layer.
+    from workloads.streams import WarmSeq
+    m = MODELS["C3"].with_layers(4)
+    rng = np.random.default_rng(33)
+    ctxs = rng.integers(4096, 5633, size=40)
+    warm = [WarmSeq(i, int(c), 3, rng.integers(0, m.vocab, size=int(c) + 3).astype(np.int32))
+            for i, c in enumerate(ctxs)]
+    nb = sum(-(-int(c) // 16) for c in ctxs) + 64
+    st = Stream("C3w", [], warm)
+    cfg = SCHED["C3"].with_(num_blocks=nb, pp_depth=1)
+
+    def hook(g, o, b):
+        if b.tick == 0:
+            _warm_kv_bit_exact(g, o, m, warm, (1,), n_seq=2)
+    n, errs, _ = _run_pair(m, cfg, st, lb=1, le=2, max_ticks=2, kv_blocks=nb, check_kv=True, tick_hook=hook)
+    assert n == 80
+    assert errs.max() <= TOL_HIDDEN, errs.max()

@@ -57,7 +57,7 @@ def _peer_rank(rank, world, port, q):
     torch.cuda.set_device(0)
     lb, le = split_layers(m.n_layers, world)[rank]
     stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
-    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden)
+    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden, pp=world)
     tr = PeerTransport(ex, rank, world, dist.group.WORLD)
     sched = None
     if rank == 0:
@@ -81,7 +81,7 @@ def _reference(q):
     from paper_conf_sc_00090d00l25_b200.runtime import GpuExecutor, Pipeline
     torch.cuda.set_device(0)
     stage = gllm.Stage(m, 0, m.n_layers, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
-    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden)
+    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden, pp=2)
     sched = gllm.Sched(sp)
     sched.add_stream(st)
     pipe = Pipeline(0, 1, ex, None, sched, None, pp=2)

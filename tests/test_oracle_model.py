@@ -200,3 +200,34 @@ def test_chunk_sizes_gqa_bias(chunk):
 def test_fp32_paged_equals_fp32_dense():
     n = _check_stage_equals_dense(MODELS["C0"], make_stream("C0", 512), SCHED["C0"], dtype=np.float32)
     assert n > 0
+
+
+def test_warm_start_decode_reads_the_warm_cache():
+    # A warm sequence's first decode (pos = context_len) attends the O4 warm K/V of positions
+    # [0, context_len) plus its own new key: stage_forward through the paged cache (blocks from the
+    # scheduler's warm allocation) == the same layer computed on dense concatenated arrays.
+    from oracle.weights import warm_kv
+    from workloads.streams import WarmSeq
+    shape = GQA.with_layers(1)
+    W = Weights(shape, dtype=np.float64)
+    ids = np.arange(200, dtype=np.int32) % shape.vocab
+    warm = [WarmSeq(0, 37, 3, ids[:40]), WarmSeq(1, 64, 2, ids[:66]), WarmSeq(2, 5, 2, ids[:7])]
+    cfg = SchedParams(pp_depth=1, num_blocks=32, block_size=16)
+    s = Scheduler(cfg, [], warm)
+    cache = om.PagedCache(shape, 16, np.float64)
+    for r in s.admitted:
+        k, v = warm_kv(shape.weight_seed, r.req_id, r.orig_len, 0, shape.n_kv_heads, shape.head_dim)
+        cache.fill_warm(0, r.blocks, k, v)
+    b = s.build_batch()
+    assert [p for (_, p) in b.decodes] == [37, 64, 5]
+    out = om.stage_forward(shape, W, cache, b, 0, 1)
+    w = W.layer(0)
+    for t, (rid, p) in enumerate(b.decodes):
+        x = W.embed_rows(ids[p:p + 1])
+        h = om.rmsnorm(x, w["g1"], shape.rms_eps)
+        q, k, v = om._qkv(shape, w, h, np.array([p]))
+        kw, vw = warm_kv(shape.weight_seed, rid, p, 0, shape.n_kv_heads, shape.head_dim)
+        kk, vv = np.concatenate([kw, k]), np.concatenate([vw, v])
+        a = om.attention(q, kk, vv, np.array([p]), np.arange(p + 1)).reshape(1, shape.q_dim)
+        ref = om._mlp(shape, w, x + a @ w["wo"].T)
+        assert np.max(np.abs(out["hidden"][t] - ref[0])) / np.max(np.abs(ref)) < 1e-12

@@ -47,3 +47,30 @@ def test_embedding_rows_match_full_table():
     full = gen(m.weight_seed, 0xFFFFF0, m.vocab * m.hidden, scale_for("embed")).reshape(m.vocab, m.hidden)
     ids = np.array([3, 511, 3, 0, 17])
     assert np.array_equal(W.embed_rows(ids), full[ids])
+
+
+def test_warm_kv_index_layout_and_counter_property():
+    # O4 warm start: element ((r*2^17 + p)*Hkv + h)*D + j of tensor 0xEE0000 + 2l (+1 V)
+    from oracle.weights import T_WARM_K, warm_kv
+    seed, Hkv, D = 1004, 8, 128
+    k, v = warm_kv(seed, 5, 40, 3, Hkv, D)
+    assert k.shape == (40, Hkv, D) and v.shape == (40, Hkv, D)
+    # a longer context extends the same values (counter-based: position p never depends on the length)
+    k2, v2 = warm_kv(seed, 5, 100, 3, Hkv, D)
+    assert np.array_equal(k2[:40], k) and np.array_equal(v2[:40], v)
+    # element (p=17, h=6, j=99) is counter (5*2^17 + 17)*1024 + 6*128 + 99 of the layer's K tensor
+    i = (5 * 2 ** 17 + 17) * Hkv * D + 6 * D + 99
+    assert k[17, 6, 99] == gen(seed, T_WARM_K + 6, 1, scale_for("embed"), start=i)[0]
+    assert v[17, 6, 99] == gen(seed, T_WARM_K + 7, 1, scale_for("embed"), start=i)[0]
+    # different request / layer / K vs V streams are decorrelated; sigma = 1, bf16 exact
+    kk, _ = warm_kv(seed, 6, 40, 3, Hkv, D)
+    kl, _ = warm_kv(seed, 5, 40, 4, Hkv, D)
+    for a, b in ((k, kk), (k, kl), (k, v)):
+        assert abs(np.corrcoef(a.ravel(), b.ravel())[0, 1]) < 0.02
+    assert abs(k.std() - 1.0) < 0.02 and np.array_equal(bf16_rne(k), k)
+
+
+def test_threaded_generation_equals_one_shot():
+    from oracle.weights import gen_threads
+    s = scale_for("proj", 512)
+    assert np.array_equal(gen_threads(7, 9, 3_000_001, s, start=11, chunk=1 << 18), gen(7, 9, 3_000_001, s, start=11))

@@ -33,8 +33,7 @@ def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_
     lb, le = split_layers(m.n_layers, pp)[stage_idx]
     max_tokens = max(sp.maxp, sp.token_budget) + sp.max_seqs + 64
     st = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs)
-    if config == "C4":
-        st.fill_kv(0xC4)
+    fill_warm(st, sp, make_stream(config, m.vocab).warm)
     s = gllm.Sched(sp)
     s.add_stream(make_stream(config, m.vocab))
     dev = torch.device("cuda")

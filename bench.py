@@ -257,6 +257,10 @@ def run_ours(args):
             uid = [gllm.get_unique_id() if rank == 0 else None]
             dist.broadcast_object_list(uid, 0)
             stage.comm_init(uid[0], rank, world)
+            nccl_info = stage.comm_size()
+            print(f"[bench] rank {rank}: NCCL communicator nranks={nccl_info[0]} rank={nccl_info[1]}",
+                  file=sys.stderr, flush=True)
+            assert nccl_info == (world, rank), nccl_info
             tr = NcclTransport(ex, rank, world)
     sched = None
     if rank == 0:
@@ -561,8 +565,9 @@ def main():
     ap.add_argument("--stage", type=int, default=0, help="with --gpus 1 --pp N: which stage to run")
     ap.add_argument("--kv-blocks", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--handoff", default="nccl", choices=["nccl", "peer"],
-                    help="N > 1: stage hand-off over NCCL P2P (default) or the fused peer-memory path")
+    ap.add_argument("--handoff", default="peer", choices=["nccl", "peer"],
+                    help="N > 1: the fused peer-memory hand-off (default; flags + slot credits over NVLink) or "
+                         "NCCL P2P send/recv")
     args = ap.parse_args()
     if args.preroll is None:
         from workloads.configs import STREAMS

@@ -210,6 +210,8 @@ GLLM_API int gllm_stage_release(gllm_stage* st, int32_t handle);
  * device buffer to/from rank dst/src on `stream`. */
 GLLM_API int gllm_get_unique_id(void* out128);
 GLLM_API int gllm_comm_init(gllm_stage* st, const void* nccl_unique_id, int32_t rank, int32_t world);
+/* The communicator's size and this stage's rank in it (ncclCommCount / ncclCommUserRank). */
+GLLM_API int gllm_comm_size(gllm_stage* st, int32_t* nranks, int32_t* rank);
 GLLM_API int gllm_send_hidden(gllm_stage* st, const void* buf, int32_t num_tokens, int32_t dst, void* stream);
 GLLM_API int gllm_recv_hidden(gllm_stage* st, void* buf, int32_t num_tokens, int32_t src, void* stream);
 GLLM_API int gllm_stage_sync(gllm_stage* st);
@@ -220,24 +222,35 @@ GLLM_API int gllm_stage_sync(gllm_stage* st);
  * two processes share the device) from the last layer's residual-add GEMM epilogue, and raises
  * the slot's flag with a system-scope release store after its last kernel.  Stage s+1's stream
  * waits on that flag (cuStreamWaitValue32) and reads the slot as hidden_in.
- * Slot reuse: micro-batch `tick` uses slot tick % depth.  With depth >= PP_depth the pipeline's
- * own rule (at most PP_depth micro-batches in flight, batch k-PP retired before k is built, R1,
- * L179) guarantees the receiver finished reading a slot before the sender overwrites it.
+ * Slot reuse is flow-controlled, independent of host timing: micro-batch `tick` uses slot
+ * tick % depth; the receiver's stage-entry kernel (the one pass that reads the slot) releases a
+ * credit for the slot (credit = tick + 1, system-scope release store from its last CTA into the
+ * sender's memory) and the sender's stream waits for credit >= tick - depth + 1 before it
+ * enqueues the forward that overwrites the slot.  Both waits are on local memory; both signals
+ * are remote stores.  Set-up order: receiver gllm_peer_ring_create -> sender gllm_peer_ring_open
+ * (returns the credit handle) -> receiver gllm_peer_credit_open.  The credits are mandatory: a
+ * sender whose receiver never opened them stalls at tick `depth`.
  * Errors: EINVAL on bad arguments or a shape mismatch, ESTATE on the wrong stage role or a ring
  * already created/opened, ECUDA on CUDA/IPC failures. */
 #define GLLM_PEER_HANDLE_BYTES 128
-/* Receiver (not the first stage): allocates depth slots of [max_tokens, hidden] fp32 plus depth
- * 32-bit flags (zero) in one exportable allocation; writes the IPC handle (caller-owned, 128 B). */
+/* Receiver (not the first stage): allocates depth (1..64) slots of [max_tokens, hidden] fp32 plus
+ * depth 32-bit flags (zero) in one exportable allocation; writes the IPC handle (caller-owned, 128 B). */
 GLLM_API int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out);
-/* Sender (not the last stage): maps the receiver's ring from its handle.  The receiver must live
- * in another process (CUDA IPC handles cannot be opened by the exporting process): ECUDA. */
-GLLM_API int gllm_peer_ring_open(gllm_stage* st, const void* handle);
+/* Sender (not the last stage): maps the receiver's ring from its handle and allocates the slot
+ * credits (depth 32-bit flags, zero) in its own memory; writes their IPC handle to
+ * credit_handle_out (caller-owned, 128 B).  The receiver must live in another process (CUDA IPC
+ * handles cannot be opened by the exporting process): ECUDA. */
+GLLM_API int gllm_peer_ring_open(gllm_stage* st, const void* handle, void* credit_handle_out);
+/* Receiver: maps the sender's slot credits (handle from gllm_peer_ring_open). */
+GLLM_API int gllm_peer_credit_open(gllm_stage* st, const void* credit_handle);
 /* Sender: the forward of a prepared batch with its output delivered to the receiver's slot for
- * `tick` (hidden_out is the slot); flag = tick + 1 after the forward's last kernel. */
+ * `tick` (hidden_out is the slot); waits on the slot's credit first (tick >= depth); flag =
+ * tick + 1 after the forward's last kernel. */
 GLLM_API int gllm_stage_forward_prepared_peer(gllm_stage* st, int32_t handle, const void* hidden_in,
                                               int64_t tick, void* stream);
 /* Receiver: enqueues on `stream` a wait for the sender's release of `tick`; *slot_out = the
- * device pointer of that slot (valid as hidden_in for forwards enqueued after the wait). */
+ * device pointer of that slot.  The next forward on this stage whose hidden_in is that slot reads
+ * it in its first kernel and releases the slot's credit. */
 GLLM_API int gllm_peer_ring_recv(gllm_stage* st, int64_t tick, void* stream, void** slot_out);
 
 /* Introspection for parity tests (host outputs, synchronous). */

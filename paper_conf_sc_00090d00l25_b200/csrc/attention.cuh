@@ -37,23 +37,15 @@ struct AttnArgs {
   int* part_ctr;       // [nparts * Hkv] split arrival counters (persistent decode kernel; kept zero)
 };
 
-// flattened (token, group-head) rows per prefill work item
-int prefill_rows_per_item();
-int launch_prefill_attention(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
-// same work items on tcgen05 (S and O in TMEM); the default prefill path
-int launch_prefill_attention_tc(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
 // warp-specialised tcgen05 prefill (attention_prefill_ws.cu), the default: items of
 // prefill_ws_rows_per_item() rows (two 128-row Q tiles); K/V pages by TMA through the decode page maps
 int prefill_ws_rows_per_item();
 int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
                                 const PrefillItem* items, int n_items, cudaStream_t s);
-int launch_decode_attention(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
-                            int n_merges, cudaStream_t s);
 // persistent warp-worker decode kernel fed by TMA (attention_decode.cu), the default; `tmk` /
 // `tmv` map the layer's K / V cache as [kv_blocks*Hkv*16, D] bf16 with 16 x 64 SW128 boxes;
 // `ctr` = 2 device ints, zero before the first launch (the kernel leaves them zero)
 bool decode_tma_supported(int D, int G);
-void set_decode_warps(int warps);
 int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
                                 const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
                                 int num_sms, cudaStream_t s);

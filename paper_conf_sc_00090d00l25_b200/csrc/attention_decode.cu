@@ -335,8 +335,6 @@ __global__ void __launch_bounds__(WARPS * 32)
   }
 }
 
-int g_dec_warps = 0;  // GLLM_DECODE_WARPS (A/B): warps per CTA, 4 (default) or 8
-
 template <int D, int G, int NST, int WARPS>
 int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items,
              int n_items, const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
@@ -365,9 +363,6 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
 template <int D, int G>
 int launch_g(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items, int n_items,
              const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
-  if (g_dec_warps == 8) return launch_t<D, G, 3, 8>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-  if (g_dec_warps == 2) return launch_t<D, G, 4, 2>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-  if (g_dec_warps == 3) return launch_t<D, G, 4, 3>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
   return launch_t<D, G, 3, 4>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
 }
 
@@ -387,8 +382,6 @@ int launch_d(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
 }  // namespace
 
 bool decode_tma_supported(int D, int G) { return (D == 64 || D == 128) && (G == 1 || G == 2 || G == 4 || G == 5 || G == 8); }
-
-void set_decode_warps(int w) { g_dec_warps = w; }
 
 int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
                                 const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,

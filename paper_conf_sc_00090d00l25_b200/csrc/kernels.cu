@@ -163,8 +163,9 @@ __global__ void __launch_bounds__(256) rmsnorm_kernel(const float* __restrict__ 
   }
 }
 
-__global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict__ x, __nv_bfloat16* xb, float* ss,
-                                                        int H) {
+__global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict__ x, float* x_copy,
+                                                        __nv_bfloat16* xb, float* ss, int H, uint32_t* rel_flag,
+                                                        uint32_t rel_val, unsigned* rel_ctr) {
   __shared__ float red[8];
   pdl_trigger();
   pdl_wait();
@@ -174,6 +175,7 @@ __global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict_
   float acc = 0.f;
   for (int c = threadIdx.x * 4; c < H; c += 256 * 4) {
     const float4 v = *reinterpret_cast<const float4*>(xr + c);
+    if (x_copy) *reinterpret_cast<float4*>(x_copy + (int64_t)r * H + c) = v;  // hand-off copy-in
     acc += v.x * v.x + v.y * v.y + v.z * v.z + v.w * v.w;
     uint2 o;
     __nv_bfloat162 a = __floats2bfloat162_rn(v.x, v.y);
@@ -182,8 +184,19 @@ __global__ void __launch_bounds__(256) rms_stats_kernel(const float* __restrict_
     o.y = *reinterpret_cast<uint32_t*>(&b);
     *reinterpret_cast<uint2*>(yr + c) = o;
   }
-  acc = block_sum<256>(acc, red);
-  if (threadIdx.x == 0) ss[r] = acc;
+  acc = block_sum<256>(acc, red);  // (its __syncthreads also orders every thread's reads of the row)
+  if (threadIdx.x == 0) {
+    ss[r] = acc;
+    if (rel_flag) {
+      // peer-ring credit: the last CTA to finish reading the input slot hands it back to the sender
+      __threadfence();
+      if (atomicAdd(rel_ctr, 1u) == gridDim.x - 1) {
+        *rel_ctr = 0;  // kept zero for the next release (stream order)
+        __threadfence_system();
+        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(rel_flag), "r"(rel_val) : "memory");
+      }
+    }
+  }
 }
 
 __global__ void argmax_reduce_kernel(const float* __restrict__ pv, const int32_t* __restrict__ pi, int rows,
@@ -262,9 +275,10 @@ void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int3
   if (n <= 0) return;
   launch_pdl(rmsnorm_kernel, dim3(n), dim3(256), 0, s, 1, x, g, y, rows, H, eps);
 }
-void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s) {
+void launch_rms_stats(const float* x, float* x_copy, __nv_bfloat16* xb, float* ss, int n, int H, uint32_t* rel_flag,
+                      uint32_t rel_val, unsigned* rel_ctr, cudaStream_t s) {
   if (n <= 0) return;
-  launch_pdl(rms_stats_kernel, dim3(n), dim3(256), 0, s, 1, x, xb, ss, H);
+  launch_pdl(rms_stats_kernel, dim3(n), dim3(256), 0, s, 1, x, x_copy, xb, ss, H, rel_flag, rel_val, rel_ctr);
 }
 void launch_argmax_reduce(const float* part_val, const int32_t* part_idx, int rows, int ntiles, int32_t* out,
                           cudaStream_t s) {

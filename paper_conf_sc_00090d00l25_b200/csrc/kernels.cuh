@@ -28,8 +28,11 @@ void launch_rmsnorm(const float* x, const float* g, __nv_bfloat16* y, const int3
                     cudaStream_t s);
 
 // Fused-RMSNorm statistics (a4): xb[r] = bf16(x[r]) and ss[r] = sum(x[r]^2) (fp32); the
-// consumer GEMM scales its output rows by rsqrt(ss/H + eps).
-void launch_rms_stats(const float* x, __nv_bfloat16* xb, float* ss, int n, int H, cudaStream_t s);
+// consumer GEMM scales its output rows by rsqrt(ss/H + eps).  x_copy (optional) receives x (the
+// stage-entry hand-off copy-in); rel_flag (optional): once every CTA has read its rows, the last one
+// stores rel_val there with st.release.sys (peer-ring slot credit); rel_ctr = one zeroed counter.
+void launch_rms_stats(const float* x, float* x_copy, __nv_bfloat16* xb, float* ss, int n, int H, uint32_t* rel_flag,
+                      uint32_t rel_val, unsigned* rel_ctr, cudaStream_t s);
 
 // (RoPE + paged K/V append run in the QKV GEMM epilogue, gemm.cu EPI_QKV_ROPE.)
 

@@ -67,6 +67,8 @@ struct NcclApi {
   decltype(&ncclSend) send = nullptr;
   decltype(&ncclRecv) recv = nullptr;
   decltype(&ncclGetErrorString) error_string = nullptr;
+  decltype(&ncclCommCount) comm_count = nullptr;
+  decltype(&ncclCommUserRank) user_rank = nullptr;
   bool ok = false;
 };
 NcclApi& nccl() {
@@ -83,7 +85,10 @@ NcclApi& nccl() {
     a.send = reinterpret_cast<decltype(a.send)>(dlsym(h, "ncclSend"));
     a.recv = reinterpret_cast<decltype(a.recv)>(dlsym(h, "ncclRecv"));
     a.error_string = reinterpret_cast<decltype(a.error_string)>(dlsym(h, "ncclGetErrorString"));
-    a.ok = a.get_unique_id && a.comm_init_rank && a.comm_destroy && a.send && a.recv && a.error_string;
+    a.comm_count = reinterpret_cast<decltype(a.comm_count)>(dlsym(h, "ncclCommCount"));
+    a.user_rank = reinterpret_cast<decltype(a.user_rank)>(dlsym(h, "ncclCommUserRank"));
+    a.ok = a.get_unique_id && a.comm_init_rank && a.comm_destroy && a.send && a.recv && a.error_string &&
+           a.comm_count && a.user_rank;
     return a;
   }();
   return api;
@@ -124,12 +129,6 @@ struct gllm_stage {
   float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T), kept zero
   int* sk_ctr = nullptr;     // stream-K fixup tile counters, kept zero
   float *ss_a = nullptr, *ss_b = nullptr;  // fused-RMSNorm row statistics (sum of squares of x)
-  float* ones = nullptr;                   // unit norm gains for the standalone RMSNorm path
-  bool fused_norm = true;
-  bool prefill_mma_sync = false;           // GLLM_PREFILL_MMA=1: mma.sync prefill kernel (A/B)
-  bool prefill_ws = true;                  // warp-specialised tcgen05 prefill (GLLM_PREFILL_WS=0: v1, A/B)
-  bool attn_overlap = true;                // GLLM_ATTN_SERIAL=1: prefill and decode attention in series (A/B)
-  bool decode_v1 = false;                  // GLLM_DECODE_V1=1: the per-CTA cp.async decode kernel (A/B)
   int* dec_ctr = nullptr;                  // persistent decode kernel: work counter + done counter
   float* part_val = nullptr;
   int32_t* part_idx = nullptr;
@@ -154,6 +153,16 @@ struct gllm_stage {
   uint32_t* peer_flags = nullptr;
   int peer_depth = 0;
   size_t peer_slot_elems = 0;
+  // slot credits (consumer -> producer): the sender owns credit[depth] (exported), the receiver maps
+  // it and releases credit[tick % depth] = tick + 1 once its stage-entry kernel has read the slot
+  uint32_t* credit = nullptr;       // sender: local credit flags
+  void* credit_peer_base = nullptr; // receiver: IPC mapping of the previous stage's credit flags
+  uint32_t* credit_peer = nullptr;
+  int credit_depth = 0;
+  unsigned* release_ctr = nullptr;  // receiver: CTA arrival counter of the releasing kernel (kept zero)
+  const void* pending_slot = nullptr;  // receiver: slot armed by gllm_peer_ring_recv for the next forward
+  uint32_t* pending_flag = nullptr;
+  uint32_t pending_value = 0;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> prof_ev;
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_used = 0;
@@ -161,7 +170,6 @@ struct gllm_stage {
   bool timing_pending = false;
 
   bool is_first() const { return lb == 0; }
-  bool use_prefill_ws() const { return prefill_ws && !prefill_mma_sync; }
   bool is_last() const { return le == cfg.n_layers; }
   int qd() const { return cfg.n_heads * cfg.head_dim; }
   int kd() const { return cfg.n_kv_heads * cfg.head_dim; }
@@ -273,6 +281,7 @@ void destroy(gllm_stage* st) {
   if (st->ev_fork) cudaEventDestroy(st->ev_fork);
   if (st->ev_join) cudaEventDestroy(st->ev_join);
   if (st->peer_base) cudaIpcCloseMemHandle(st->peer_base);
+  if (st->credit_peer_base) cudaIpcCloseMemHandle(st->credit_peer_base);
   cudaGetLastError();
   delete st;
 }
@@ -421,22 +430,17 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = st->dalloc(&st->slots, R)) ||
       // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
       (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)) || (rc = st->dalloc(&st->ss_a, R)) ||
-      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->ones, H)) || (rc = st->dalloc(&st->dec_ctr, 2)) ||
+      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->dec_ctr, 2)) || (rc = st->dalloc(&st->release_ctr, 1)) ||
       (rc = st->dalloc(&st->sk_ctr, gllm::GEMM_MAX_SK_TILES)))
     return fail(rc);
   CK(cudaMemsetAsync(st->gemm_ws, 0, gllm::GEMM_WS_ELEMS * sizeof(float), s0));
   CK(cudaMemsetAsync(st->sk_ctr, 0, gllm::GEMM_MAX_SK_TILES * sizeof(int), s0));
   CK(cudaMemsetAsync(st->dec_ctr, 0, 2 * sizeof(int), s0));
+  CK(cudaMemsetAsync(st->release_ctr, 0, sizeof(unsigned), s0));
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
-  gllm::launch_fill_f32(st->ones, H, 1.0f, s0);
-  if (const char* e = std::getenv("GLLM_UNFUSED_NORM")) st->fused_norm = e[0] != '1';
-  if (const char* e = std::getenv("GLLM_PREFILL_MMA")) st->prefill_mma_sync = e[0] == '1';
-  if (const char* e = std::getenv("GLLM_PREFILL_WS")) st->prefill_ws = e[0] != '0';
-  if (block_size != 16) st->prefill_ws = false;
-  if (const char* e = std::getenv("GLLM_ATTN_SERIAL")) st->attn_overlap = e[0] != '1';
-  if (const char* e = std::getenv("GLLM_DECODE_V1")) st->decode_v1 = e[0] == '1';
-  if (const char* e = std::getenv("GLLM_DECODE_WARPS")) gllm::set_decode_warps(std::atoi(e));
-  if (!gllm::decode_tma_supported(D, cfg->n_heads / Hkv) || block_size != 16) st->decode_v1 = true;
+  if (!gllm::decode_tma_supported(D, cfg->n_heads / Hkv))
+    return fail(gllm::set_error(GLLM_EINVAL, "decode attention: head_dim %d / GQA group %d unsupported", D,
+                                cfg->n_heads / Hkv));
   CK(cudaMemsetAsync(st->attn, 0, R * qd * sizeof(bf16), s0));
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
@@ -445,10 +449,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     return fail(rc);
   for (int i = 0; i < RING; ++i)
     if ((rc = new_slot(st)) < 0) return fail(rc);
-  int prio_lo = 0, prio_hi = 0;
-  cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-  const char* sp = std::getenv("GLLM_SIDE_PRIO");  // A/B: prefill attention stream at the highest priority
-  if (cudaStreamCreateWithPriority(&st->side, cudaStreamNonBlocking, (sp && sp[0] == '1') ? prio_hi : 0) != cudaSuccess ||
+  if (cudaStreamCreateWithFlags(&st->side, cudaStreamNonBlocking) != cudaSuccess ||
       cudaEventCreateWithFlags(&st->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
       cudaEventCreateWithFlags(&st->ev_join, cudaEventDisableTiming) != cudaSuccess)
     return fail(gllm::set_error(GLLM_ECUDA, "side stream / events"));
@@ -515,7 +516,7 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   for (int i = 0; i < NP; ++i) {
     const int n = d->cu_q[i + 1] - d->cu_q[i];
     const int rows = n * G, s0 = d->kv_len[i] - n;
-    const int rpi = st->use_prefill_ws() ? gllm::prefill_ws_rows_per_item() : gllm::prefill_rows_per_item();
+    const int rpi = gllm::prefill_ws_rows_per_item();
     for (int r0 = 0; r0 < rows; r0 += rpi) {
       const int last = std::min(r0 + rpi - 1, rows - 1) / G;
       pcost.push_back({(s0 + last + 64) / 64, (int)pitems.size()});
@@ -537,7 +538,7 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
     // longer than the average per-warp work are split; a split is at least 16 pages)
     const int64_t target = 8LL * st->num_sms;  // CTAs (v1) / warp workers (persistent kernel)
     int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
-    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(st->decode_v1 ? 32 : 16, per));
+    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(16, per));
   }
   std::vector<gllm::DecodeItem> ditems;
   std::vector<gllm::MergeItem> merges;
@@ -637,8 +638,6 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     Prof p(st, s, C_OTHER);
     gllm::launch_embed(st->embed, d_ids, x, T, H, s);
     st->last_launches += 1;
-  } else if (hidden_in != x) {
-    CK(cudaMemcpyAsync(x, hidden_in, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
   }
   gllm::AttnArgs aa{};
   aa.q = st->qkv;
@@ -659,27 +658,28 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
   // Fused RMSNorm (a4): y holds bf16(x) and ss_a / ss_b the per-row sum of squares of x; the
   // consumer GEMMs (QKV, gate_up) scale their rows by rsqrt(ss/H + eps) in the epilogue and the
   // residual-add GEMMs (O, down) produce y and ss for the next norm.  Only the stage entry (and a
-  // stream-K residual GEMM) needs the standalone statistics pass.
-  // (GLLM_UNFUSED_NORM=1 selects standalone RMSNorm kernels instead -- kept for A/B measurement.)
-  const bool fused = st->fused_norm;
-  if (fused) {
+  // stream-K residual GEMM) needs the standalone statistics pass.  On stages after the first that
+  // pass also moves hidden_in into the residual buffer (the hand-off copy-in, one read of the
+  // input), and when hidden_in is a peer-ring slot its last CTA releases the slot's credit to the
+  // sending stage.
+  {
     Prof p(st, s, C_NORM);
-    gllm::launch_rms_stats(x, st->y, st->ss_a, T, H, s);
+    const float* src = st->is_first() ? x : static_cast<const float*>(hidden_in);
+    uint32_t* rel = nullptr;
+    if (!st->is_first() && hidden_in == st->pending_slot && st->pending_flag) rel = st->pending_flag;
+    gllm::launch_rms_stats(src, src != x ? x : nullptr, st->y, st->ss_a, T, H, rel, st->pending_value,
+                           st->release_ctr, s);
+    st->pending_slot = nullptr;
+    st->pending_flag = nullptr;
     st->last_launches += 1;
   }
-  auto standalone_norm = [&]() {
-    if (fused) return;
-    Prof p(st, s, C_NORM);
-    gllm::launch_rmsnorm(x, st->ones, st->y, nullptr, T, H, c.rms_eps, s);
-    st->last_launches += 1;
-  };
   const float inv_h = 1.0f / (float)H;
   auto residual_gemm = [&](const CUtensorMap& ta, const CUtensorMap& tb, int K, float* ss_next,
                            float* out_peer) -> int {
     // ss_next was zeroed by the n-tile-0 epilogue of the preceding consumer GEMM (zero_rows)
-    const bool sk = !fused || gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
+    const bool sk = gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
     gllm::GemmArgs g{};
-  g.b_static = 1;
+    g.b_static = 1;
     g.M = T;
     g.N = H;
     g.K = K;
@@ -692,20 +692,19 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms));
     if (out_peer && sk)  // partial tiles reduce in place: copy the finished residual afterwards
       CK(cudaMemcpyAsync(out_peer, x, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
-    if (sk && fused) {  // partial tiles combine with reductions: recompute the statistics from x
-      gllm::launch_rms_stats(x, st->y, ss_next, T, H, s);
+    if (sk) {  // partial tiles combine with reductions: recompute the statistics from x
+      gllm::launch_rms_stats(x, nullptr, st->y, ss_next, T, H, nullptr, 0, nullptr, s);
       st->last_launches += 1;
     }
     return GLLM_OK;
   };
   for (size_t li = 0; li < st->layers.size(); ++li) {
     LayerW& w = st->layers[li];
-    standalone_norm();
     {
       // QKV projection with RoPE and the paged KV append fused into the epilogue (a5 + a6)
       Prof p(st, s, C_QKV);
       gllm::GemmArgs g{};
-  g.b_static = 1;
+      g.b_static = 1;
       g.M = T;
       g.N = nqkv;
       g.K = H;
@@ -723,25 +722,23 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.block_size = bs;
       g.ws = st->gemm_ws;
       g.tile_ctr = st->sk_ctr;
-  g.tile_ctr = st->sk_ctr;
-      g.row_ss = fused ? st->ss_a : nullptr;
+      g.row_ss = st->ss_a;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
-      g.zero_rows = fused ? st->ss_b : nullptr;  // reset for the O GEMM's statistics
+      g.zero_rows = st->ss_b;  // reset for the O GEMM's statistics
       st->last_launches += 1;
       RC(gllm::launch_gemm(st->tm_y, w.tm_qkv, gllm::EPI_QKV_ROPE, g, s, st->num_sms));
     }
     aa.kc = w.kc;
     aa.vc = w.vc;
     auto decode = [&](cudaStream_t ds) -> int {
-      st->last_launches += (P.n_mi && st->decode_v1) ? 2 : 1;  // the persistent kernel merges in place
-      if (st->decode_v1) return gllm::launch_decode_attention(aa, d_di, P.n_di, d_mi, P.n_mi, ds);
+      st->last_launches += 1;  // the persistent kernel merges split rows in place
       return gllm::launch_decode_attention_tma(aa, w.tm_kc, w.tm_vc, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
                                                st->num_sms, ds);
     };
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.
-    const bool overlap = st->attn_overlap && !st->prof_serial_attn && P.n_pi > 0 && P.n_di > 0;
+    const bool overlap = !st->prof_serial_attn && P.n_pi > 0 && P.n_di > 0;
     Prof p_attn(st, s, C_ATTN);  // span of the attention step (prefill || decode), on the main stream
     if (P.n_pi > 0) {
       cudaStream_t ps = overlap ? st->side : s;
@@ -751,11 +748,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       }
       {
         Prof p(st, ps, C_PREFILL);
-        if (st->use_prefill_ws())
-          RC(gllm::launch_prefill_attention_ws(aa, w.tm_kc, w.tm_vc, d_pi, P.n_pi, ps));
-        else
-          RC(st->prefill_mma_sync ? gllm::launch_prefill_attention(aa, d_pi, P.n_pi, ps)
-                                  : gllm::launch_prefill_attention_tc(aa, d_pi, P.n_pi, ps));
+        RC(gllm::launch_prefill_attention_ws(aa, w.tm_kc, w.tm_vc, d_pi, P.n_pi, ps));
       }
       if (overlap) CK(cudaEventRecord(st->ev_join, ps));
       st->last_launches += 1;
@@ -775,11 +768,10 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       Prof p(st, s, C_O);
       RC(residual_gemm(st->tm_attn, w.tm_o, qd, st->ss_b, nullptr));
     }
-    standalone_norm();
     {
       Prof p(st, s, C_GU);
       gllm::GemmArgs g{};
-  g.b_static = 1;
+      g.b_static = 1;
       g.M = T;
       g.N = 2 * I;
       g.K = H;
@@ -787,11 +779,10 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.ldo = I;
       g.ws = st->gemm_ws;
       g.tile_ctr = st->sk_ctr;
-  g.tile_ctr = st->sk_ctr;
-      g.row_ss = fused ? st->ss_b : nullptr;
+      g.row_ss = st->ss_b;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
-      g.zero_rows = fused ? st->ss_a : nullptr;  // reset for the down GEMM's statistics
+      g.zero_rows = st->ss_a;  // reset for the down GEMM's statistics
       st->last_launches += 1;
       RC(gllm::launch_gemm(st->tm_y, w.tm_gu, gllm::EPI_SILU_MUL, g, s, st->num_sms));
     }
@@ -917,6 +908,18 @@ int gllm_comm_init(gllm_stage* st, const void* uid, int32_t rank, int32_t world)
   std::memcpy(&id, uid, sizeof(id));
   ncclResult_t r = nccl().comm_init_rank(&st->comm, world, id, rank);
   if (r != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclCommInitRank: %s", nccl().error_string(r));
+  return GLLM_OK;
+}
+
+int gllm_comm_size(gllm_stage* st, int32_t* nranks, int32_t* rank) {
+  if (!st || !nranks || !rank) return gllm::set_error(GLLM_EINVAL, "null argument");
+  if (!st->comm) return gllm::set_error(GLLM_ESTATE, "comm_size: no communicator");
+  int n = 0, r = 0;
+  ncclResult_t e = nccl().comm_count(st->comm, &n);
+  if (e == ncclSuccess) e = nccl().user_rank(st->comm, &r);
+  if (e != ncclSuccess) return gllm::set_error(GLLM_ENCCL, "ncclCommCount/UserRank: %s", nccl().error_string(e));
+  *nranks = n;
+  *rank = r;
   return GLLM_OK;
 }
 
@@ -1097,7 +1100,7 @@ extern "C" {
 
 int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out) {
   GLLM_TRY_BEGIN
-  if (!st || !handle_out || depth < 1) return gllm::set_error(GLLM_EINVAL, "peer ring: bad arguments");
+  if (!st || !handle_out || depth < 1 || depth > 64) return gllm::set_error(GLLM_EINVAL, "peer ring: bad arguments");
   if (st->is_first()) return gllm::set_error(GLLM_ESTATE, "peer ring: the first stage receives no hidden states");
   if (st->ring) return gllm::set_error(GLLM_ESTATE, "peer ring already created");
   CK(cudaSetDevice(st->device));
@@ -1121,9 +1124,9 @@ int gllm_peer_ring_create(gllm_stage* st, int32_t depth, void* handle_out) {
   GLLM_TRY_END
 }
 
-int gllm_peer_ring_open(gllm_stage* st, const void* handle) {
+int gllm_peer_ring_open(gllm_stage* st, const void* handle, void* credit_handle_out) {
   GLLM_TRY_BEGIN
-  if (!st || !handle) return gllm::set_error(GLLM_EINVAL, "peer ring open: null argument");
+  if (!st || !handle || !credit_handle_out) return gllm::set_error(GLLM_EINVAL, "peer ring open: null argument");
   if (st->is_last()) return gllm::set_error(GLLM_ESTATE, "peer ring open: the last stage sends no hidden states");
   if (st->peer_base) return gllm::set_error(GLLM_ESTATE, "peer ring already open");
   PeerHandle h;
@@ -1139,6 +1142,20 @@ int gllm_peer_ring_open(gllm_stage* st, const void* handle) {
   st->peer_ring = reinterpret_cast<float*>(static_cast<uint8_t*>(base) + 256);
   st->peer_depth = h.depth;
   st->peer_slot_elems = (size_t)h.max_tokens * h.hidden;
+  // the slot credits live here (the waiter's memory, like the ready flags on the receiver's side);
+  // the receiver maps them with gllm_peer_credit_open and releases each slot after reading it
+  void* cb = nullptr;
+  CK(cudaMalloc(&cb, 256));
+  CK(cudaMemset(cb, 0, 256));
+  st->allocs.push_back(cb);
+  st->credit = static_cast<uint32_t*>(cb);
+  PeerHandle ch{};
+  CK(cudaIpcGetMemHandle(&ch.mem, cb));
+  ch.depth = h.depth;
+  ch.max_tokens = h.max_tokens;
+  ch.hidden = h.hidden;
+  std::memset(credit_handle_out, 0, GLLM_PEER_HANDLE_BYTES);
+  std::memcpy(credit_handle_out, &ch, sizeof(ch));
   return GLLM_OK;
   GLLM_TRY_END
 }
@@ -1152,6 +1169,15 @@ int gllm_stage_forward_prepared_peer(gllm_stage* st, int32_t handle, const void*
   if (tick < 0) return gllm::set_error(GLLM_EINVAL, "negative tick");
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const int slot = (int)(tick % st->peer_depth);
+  if (tick >= st->peer_depth && st->prep[handle].T > 0) {
+    // the slot last carried tick - depth: wait until the receiver has read it (credit >= tick - depth + 1)
+    PfnWaitValue32 wv = wait_value32();
+    if (!wv) return gllm::set_error(GLLM_ECUDA, "cuStreamWaitValue32 unavailable");
+    CK(cudaSetDevice(st->device));
+    const CUresult r = wv(reinterpret_cast<CUstream>(s), reinterpret_cast<CUdeviceptr>(st->credit + slot),
+                          (cuuint32_t)(tick - st->peer_depth + 1), CU_STREAM_WAIT_VALUE_GEQ);
+    if (r != CUDA_SUCCESS) return gllm::set_error(GLLM_ECUDA, "cuStreamWaitValue32 (credit) failed (%d)", (int)r);
+  }
   float* dst = st->peer_ring + (size_t)slot * st->peer_slot_elems;
   RC(forward_impl(st, st->prep[handle], hidden_in, nullptr, nullptr, s, dst));
   if (st->prep[handle].T > 0) {
@@ -1176,6 +1202,29 @@ int gllm_peer_ring_recv(gllm_stage* st, int64_t tick, void* stream, void** slot_
                         (cuuint32_t)(tick + 1), CU_STREAM_WAIT_VALUE_GEQ);
   if (r != CUDA_SUCCESS) return gllm::set_error(GLLM_ECUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
   *slot_out = st->ring + (size_t)slot * st->max_tokens * st->cfg.hidden;
+  if (st->credit_peer) {  // the next forward reading this slot releases its credit (rms_stats' last CTA)
+    st->pending_slot = *slot_out;
+    st->pending_flag = st->credit_peer + slot;
+    st->pending_value = (uint32_t)(tick + 1);
+  }
+  return GLLM_OK;
+  GLLM_TRY_END
+}
+
+int gllm_peer_credit_open(gllm_stage* st, const void* credit_handle) {
+  GLLM_TRY_BEGIN
+  if (!st || !credit_handle) return gllm::set_error(GLLM_EINVAL, "peer credit open: null argument");
+  if (!st->ring) return gllm::set_error(GLLM_ESTATE, "peer credit open: create the receive ring first");
+  if (st->credit_peer_base) return gllm::set_error(GLLM_ESTATE, "peer credits already open");
+  PeerHandle h;
+  std::memcpy(&h, credit_handle, sizeof(h));
+  if (h.depth != st->ring_depth || h.hidden != st->cfg.hidden)
+    return gllm::set_error(GLLM_EINVAL, "peer credit: depth %d / hidden %d do not match the ring", h.depth, h.hidden);
+  CK(cudaSetDevice(st->device));
+  void* base = nullptr;
+  CK(cudaIpcOpenMemHandle(&base, h.mem, cudaIpcMemLazyEnablePeerAccess));
+  st->credit_peer_base = base;
+  st->credit_peer = static_cast<uint32_t*>(base);
   return GLLM_OK;
   GLLM_TRY_END
 }

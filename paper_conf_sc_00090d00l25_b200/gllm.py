@@ -103,11 +103,13 @@ def lib():
             "gllm_stage_release": ([vp, i32], C.c_int),
             "gllm_get_unique_id": ([vp], C.c_int),
             "gllm_comm_init": ([vp, vp, i32, i32], C.c_int),
+            "gllm_comm_size": ([vp, _P32, _P32], C.c_int),
             "gllm_send_hidden": ([vp, vp, i32, i32, vp], C.c_int),
             "gllm_recv_hidden": ([vp, vp, i32, i32, vp], C.c_int),
             "gllm_stage_sync": ([vp], C.c_int),
             "gllm_peer_ring_create": ([vp, i32, vp], C.c_int),
-            "gllm_peer_ring_open": ([vp, vp], C.c_int),
+            "gllm_peer_ring_open": ([vp, vp, vp], C.c_int),
+            "gllm_peer_credit_open": ([vp, vp], C.c_int),
             "gllm_stage_forward_prepared_peer": ([vp, i32, vp, i64, vp], C.c_int),
             "gllm_peer_ring_recv": ([vp, i64, vp, C.POINTER(C.c_void_p)], C.c_int),
             "gllm_stage_read_weight": ([vp, i32, C.c_char_p, i64, i64, C.POINTER(C.c_float)], C.c_int),
@@ -357,9 +359,16 @@ class Stage:
         _check(lib().gllm_peer_ring_create(self.h, depth, buf))
         return buf.raw
 
-    def peer_ring_open(self, handle: bytes):
+    def peer_ring_open(self, handle: bytes) -> bytes:
+        """Maps the receiver's ring; returns the handle of this sender's slot credits."""
         buf = C.create_string_buffer(handle, 128)
-        _check(lib().gllm_peer_ring_open(self.h, buf))
+        out = C.create_string_buffer(128)
+        _check(lib().gllm_peer_ring_open(self.h, buf, out))
+        return out.raw
+
+    def peer_credit_open(self, credit_handle: bytes):
+        buf = C.create_string_buffer(credit_handle, 128)
+        _check(lib().gllm_peer_credit_open(self.h, buf))
 
     def forward_prepared_peer(self, handle, tick, hidden_in=0, stream=0):
         return _check(lib().gllm_stage_forward_prepared_peer(self.h, handle, hidden_in or None, tick, stream or None))
@@ -368,6 +377,12 @@ class Stage:
         out = C.c_void_p()
         _check(lib().gllm_peer_ring_recv(self.h, tick, stream or None, C.byref(out)))
         return out.value
+
+    def comm_size(self):
+        """(nranks, rank) of this stage's NCCL communicator."""
+        n, r = C.c_int32(), C.c_int32()
+        _check(lib().gllm_comm_size(self.h, C.byref(n), C.byref(r)))
+        return n.value, r.value
 
     def send_hidden(self, ptr, num_tokens, dst, stream=0):
         _check(lib().gllm_send_hidden(self.h, ptr, num_tokens, dst, stream or None))

@@ -177,25 +177,34 @@ class NcclTransport:
 
 class PeerTransport:
     """Fused hand-off over peer memory (include/gllm.h gllm_peer_*): stage s+1 exports a ring of
-    receive slots, stage s maps it and its last residual GEMM writes into the slot; the flags make
-    the hand-off stream-ordered, so recv/send are no-ops here.  Slot reuse is safe with
-    depth >= PP by R1 (batch k-PP retires before batch k is built); depth = 2 PP."""
+    receive slots, stage s maps it and its last residual GEMM writes into the slot; ready flags
+    (sender -> receiver) and slot credits (receiver -> sender) make the hand-off stream-ordered and
+    flow-controlled on the devices, so recv/send are no-ops here.  depth = 2 PP slots.
+
+    Handle exchange over the (gloo) metadata group: rank s+1 sends its ring handle to rank s; rank s
+    maps it and sends back the handle of its slot credits, which rank s+1 maps."""
 
     def __init__(self, ex: GpuExecutor, rank, world, group, pp=None):
         import torch
         import torch.distributed as dist
         self.ex, self.rank, self.world = ex, rank, world
         depth = 2 * (pp or world)
-        # ring handles travel rank s+1 -> rank s over the (gloo) metadata group, in rank order
+
+        def send(b: bytes, dst):
+            dist.send(torch.frombuffer(bytearray(b), dtype=torch.uint8), dst, group=group)
+
+        def recv(src) -> bytes:
+            t = torch.empty(128, dtype=torch.uint8)
+            dist.recv(t, src, group=group)
+            return bytes(t.numpy().tobytes())
         if rank > 0:
-            h = ex.stage.peer_ring_create(depth)
-            dist.send(torch.frombuffer(bytearray(h), dtype=torch.uint8), rank - 1, group=group)
+            send(ex.stage.peer_ring_create(depth), rank - 1)
             ex.peer_in = True
         if rank < world - 1:
-            t = torch.empty(128, dtype=torch.uint8)
-            dist.recv(t, rank + 1, group=group)
-            ex.stage.peer_ring_open(bytes(t.numpy().tobytes()))
+            send(ex.stage.peer_ring_open(recv(rank + 1)), rank + 1)
             ex.peer_out = True
+        if rank > 0:
+            ex.stage.peer_credit_open(recv(rank - 1))
 
     def recv(self, k, T):
         pass

@@ -6,7 +6,12 @@ The sender's last residual-add GEMM epilogue stores its output rows straight int
 ring slot and raises the slot flag; the receiver's stream waits on the flag and reads the slot as
 hidden_in.  The receiver's hidden states and greedy ids must match the oracle's two-layer forward
 (north_star bars), tick by tick over the C0 stream and a C1-shaped prefix (stream-K and whole-tile
-schedules of the last GEMM)."""
+schedules of the last GEMM).
+
+The free-running variant removes the lockstep: the sender enqueues every tick back to back with a
+2-slot ring while the receiver sleeps before each tick, so only the slot credits (the receiver's
+stage-entry kernel releases each slot; the sender's stream waits for the credit before overwriting)
+keep the sender from overwriting slots the receiver has not read."""
 import multiprocessing as mp
 import os
 
@@ -29,7 +34,7 @@ def _cases():
     }
 
 
-def _sender(case, q_handle, q_desc, q_done):
+def _sender(case, lockstep, q_handle, q_credit, q_desc, q_done):
     import sys
     sys.path.insert(0, ROOT)
     import torch
@@ -39,7 +44,7 @@ def _sender(case, q_handle, q_desc, q_done):
     stage = gllm.Stage(m, 0, 1, cfg.num_blocks, mt, min(cfg.max_seqs, mt))
     sched = gllm.Sched(cfg)
     sched.add_stream(st)
-    stage.peer_ring_open(q_handle.get(timeout=120))
+    q_credit.put(stage.peer_ring_open(q_handle.get(timeout=120)))
     s = torch.cuda.current_stream().cuda_stream
     for k in range(ticks):
         d = sched.build_batch()
@@ -48,13 +53,19 @@ def _sender(case, q_handle, q_desc, q_done):
         if d.num_tokens:
             h = stage.prepare(d, s)
             stage.forward_prepared_peer(h, int(a["tick"]), 0, s)
-            torch.cuda.synchronize()
-            stage.release(h)
-        assert q_done.get(timeout=300) == k    # lockstep: the receiver consumed tick k
+            if lockstep:
+                torch.cuda.synchronize()
+            stage.release(h)   # (a prepared slot is reused only after its forward completed)
+        if lockstep:
+            assert q_done.get(timeout=300) == k    # the receiver consumed tick k
+    torch.cuda.synchronize()
+    if not lockstep:
+        for k in range(ticks):   # keep the credit memory alive until the receiver is done
+            assert q_done.get(timeout=600) == k
     stage.close()
 
 
-def _receiver(case, q_handle, q_desc, q_done, q_out):
+def _receiver(case, lockstep, q_handle, q_credit, q_desc, q_done, q_out):
     import sys
     sys.path.insert(0, ROOT)
     import torch
@@ -62,10 +73,14 @@ def _receiver(case, q_handle, q_desc, q_done, q_out):
     m, cfg, _, depth, mt, ticks = _cases()[case]
     stage = gllm.Stage(m, 1, 2, cfg.num_blocks, mt, min(cfg.max_seqs, mt))
     q_handle.put(stage.peer_ring_create(depth))
+    stage.peer_credit_open(q_credit.get(timeout=120))
     dev = torch.device("cuda", 0)
     s = torch.cuda.current_stream().cuda_stream
     for k in range(ticks):
         a = q_desc.get(timeout=300)
+        if not lockstep:
+            import time
+            time.sleep(0.3)      # let the sender run ahead by more than the ring depth
         T = int(a["num_tokens"])
         res = {"tick": int(a["tick"]), "T": T}
         if T:
@@ -85,14 +100,14 @@ def _receiver(case, q_handle, q_desc, q_done, q_out):
 
 
 @pytest.mark.timeout(900)
-@pytest.mark.parametrize("case", ["C0", "C1"])
-def test_peer_handoff_two_processes_one_gpu(case):
+@pytest.mark.parametrize("case,lockstep", [("C0", True), ("C1", True), ("C1", False)])
+def test_peer_handoff_two_processes_one_gpu(case, lockstep):
     from tests.gpu_harness import OracleRun, TOL_HIDDEN, greedy_ok, row_rel_err
     m, cfg, (sname, n), depth, mt, ticks = _cases()[case]
     ctx = mp.get_context("spawn")
-    q_handle, q_desc, q_done, q_out = ctx.Queue(), ctx.Queue(), ctx.Queue(), ctx.Queue()
-    ps = [ctx.Process(target=_sender, args=(case, q_handle, q_desc, q_done)),
-          ctx.Process(target=_receiver, args=(case, q_handle, q_desc, q_done, q_out))]
+    q_handle, q_credit, q_desc, q_done, q_out = ctx.Queue(), ctx.Queue(), ctx.Queue(), ctx.Queue(), ctx.Queue()
+    ps = [ctx.Process(target=_sender, args=(case, lockstep, q_handle, q_credit, q_desc, q_done)),
+          ctx.Process(target=_receiver, args=(case, lockstep, q_handle, q_credit, q_desc, q_done, q_out))]
     for p in ps:
         p.start()
     outs = [q_out.get(timeout=600) for _ in range(ticks)]

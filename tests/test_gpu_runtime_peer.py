@@ -3,7 +3,11 @@ embedding + layer 0; stage 1: layer 1 + LM head of a 2-layer Llama-3-8B-shaped m
 cuda:0, exchange micro-batch metadata over gloo (L204) and hidden states through
 PeerTransport (gllm_peer_*, stream-ordered flags, no NCCL).  The greedy ids the last stage
 returns must agree with a one-process run of the same model on the same C1 stream prefix
-(same scheduler, PP_depth = 2 retire rule)."""
+(same scheduler, PP_depth = 2 retire rule).
+
+With two or more visible GPUs the same run is repeated with the stages on cuda:0 and cuda:1, over
+the peer hand-off (NVLink peer stores) and over NCCL P2P (gllm_send_hidden / recv_hidden,
+NcclTransport); with one GPU those cases skip (NCCL rejects two ranks on one device)."""
 import multiprocessing as mp
 import os
 import socket
@@ -47,18 +51,27 @@ def _record(ex, store):
     ex.sampled = sampled
 
 
-def _peer_rank(rank, world, port, q):
+def _peer_rank(rank, world, port, q, transport="peer", gpus=1):
     torch, gllm, m, sp, st, max_tokens = _setup(world)
     import torch.distributed as dist
-    from paper_conf_sc_00090d00l25_b200.runtime import GpuExecutor, PeerTransport, Pipeline, split_layers
+    from paper_conf_sc_00090d00l25_b200.runtime import (GpuExecutor, NcclTransport, PeerTransport, Pipeline,
+                                                        split_layers)
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    torch.cuda.set_device(0)
+    dev = rank if gpus > 1 else 0
+    torch.cuda.set_device(dev)
     lb, le = split_layers(m.n_layers, world)[rank]
-    stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
-    ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden, pp=world)
-    tr = PeerTransport(ex, rank, world, dist.group.WORLD)
+    stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=dev)
+    ex = GpuExecutor(stage, torch.device("cuda", dev), max_tokens, m.hidden, pp=world)
+    if transport == "peer":
+        tr = PeerTransport(ex, rank, world, dist.group.WORLD)
+    else:
+        uid = [gllm.get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, 0)
+        stage.comm_init(uid[0], rank, world)
+        assert stage.comm_size() == (world, rank)
+        tr = NcclTransport(ex, rank, world)
     sched = None
     if rank == 0:
         sched = gllm.Sched(sp)
@@ -95,7 +108,11 @@ def _reference(q):
 
 
 @pytest.mark.timeout(900)
-def test_pipeline_runtime_with_peer_handoff_matches_one_process():
+@pytest.mark.parametrize("transport,gpus", [("peer", 1), ("peer", 2), ("nccl", 2)])
+def test_pipeline_runtime_handoff_matches_one_process(transport, gpus):
+    import torch
+    if torch.cuda.device_count() < gpus:
+        pytest.skip(f"needs {gpus} GPUs")
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     ref = ctx.Process(target=_reference, args=(q,))
@@ -104,7 +121,7 @@ def test_pipeline_runtime_with_peer_handoff_matches_one_process():
     ref.join(timeout=120)
     assert tag == "ref" and ref.exitcode == 0
     port = _free_port()
-    ps = [ctx.Process(target=_peer_rank, args=(r, 2, port, q)) for r in range(2)]
+    ps = [ctx.Process(target=_peer_rank, args=(r, 2, port, q, transport, gpus)) for r in range(2)]
     for p in ps:
         p.start()
     outs = dict(q.get(timeout=600) for _ in range(2))

@@ -450,8 +450,27 @@ def run_ours(args):
 
 
 # ---------------------------------------------------------------------------- oracle (CPU)
-def _oracle_layer_time(m, a, W, layers=1):
-    """Time `layers` decoder layers of the oracle on batch `a` (full width); returns seconds."""
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def _blas_threads():
+    try:
+        from threadpoolctl import threadpool_info
+        return max((p.get("num_threads", 1) for p in threadpool_info()), default=os.cpu_count())
+    except Exception:
+        return os.cpu_count()
+
+
+def _oracle_layer_time(m, a, W, layer=0):
+    """Wall time of ONE decoder layer of oracle.model.stage_forward on batch `a` at full width (the
+    embedding rows are the stage input; no LM head).  Returns seconds, measured."""
     from oracle import model as om
 
     class B:
@@ -461,48 +480,53 @@ def _oracle_layer_time(m, a, W, layers=1):
         setattr(b, k, np.asarray(a[k]))
     b.num_tokens = int(a["num_tokens"])
     cache = om.PagedCache(m, 16, np.float32)
-    # KV of earlier ticks: the oracle cache starts empty in this bounded sample; seed the pages the
-    # batch reads (values do not change the oracle's cost)
-    rng = np.random.default_rng(0)
-    shape = (16, m.n_kv_heads, m.head_dim)
-    for l in range(layers):
-        K, V = cache.k.setdefault(l, {}), cache.v.setdefault(l, {})
-        for row, n in zip(np.asarray(a["block_table"]), np.asarray(a["kv_len"])):
-            for blk in row[: -(-int(n) // 16)]:
-                if int(blk) not in K:
-                    K[int(blk)] = rng.standard_normal(shape).astype(np.float32)
-                    V[int(blk)] = rng.standard_normal(shape).astype(np.float32)
-    for l in range(layers):
-        W.layer(l)  # generate weights outside the timed region
+    # the pages this batch reads from earlier ticks: the O4 warm-KV values of each sequence (the oracle's
+    # arithmetic does not depend on them; they make the sample self-contained)
+    from oracle.weights import warm_kv
+    for i, (row, n) in enumerate(zip(np.asarray(a["block_table"]), np.asarray(a["kv_len"]))):
+        k, v = warm_kv(m.weight_seed, i, int(n), layer, m.n_kv_heads, m.head_dim)
+        cache.fill_warm(layer, row, k, v)
+    W.layer(layer)  # weights generated outside the timed region
+    x = W.embed_rows(b.token_ids)
     t0 = time.perf_counter()
-    # oracle.model.stage_forward over layers [0, layers): embedding + decoder layers, no LM head
-    om.stage_forward(m, W, cache, b, 0, layers)
+    om.stage_forward(m, W, cache, b, layer, layer + 1, hidden_in=x)
     return time.perf_counter() - t0
 
 
+def _layer_flops(m, T):
+    return 2.0 * T * (m.hidden * (m.q_dim + 2 * m.kv_dim) + m.q_dim * m.hidden + 3 * m.hidden * m.intermediate)
+
+
 def cpu_baseline(args, m, a, n_layers=None, with_lm_head=True):
-    """The oracle on a bounded sample: 1 decoder layer of the batch, scaled to the stage's layers."""
+    """The oracle as it stands on a bounded sample: ONE decoder layer of the first timed tick's whole
+    batch, timed for real with all BLAS threads and with one thread, then expressed in the metric's
+    unit for the stage (time x layers, + the LM head's FLOP share)."""
     from oracle.weights import Weights
-    try:
-        from threadpoolctl import threadpool_info
-        threads = max((p.get("num_threads", 1) for p in threadpool_info()), default=os.cpu_count())
-    except Exception:
-        threads = os.cpu_count()
     n_layers = n_layers or m.n_layers
     W = Weights(m)
-    sec = _oracle_layer_time(m, a, W, 1)
     T = int(a["num_tokens"])
-    layer_flops = 2.0 * T * (m.hidden * (m.q_dim + 2 * m.kv_dim) + m.q_dim * m.hidden + 3 * m.hidden * m.intermediate)
-    lm_flops = 2.0 * int(np.asarray(a["sample_idx"]).shape[0]) * m.hidden * m.vocab if with_lm_head else 0.0
-    est = sec * (n_layers + lm_flops / layer_flops)
-    return {"value": round(T / est, 2), "unit": UNIT, "cores": int(threads), "kind": "oracle",
-            "sample": f"oracle fp32 forward of 1 of {n_layers} decoder layers on the first timed tick "
-                      f"(T={T}), {sec:.2f} s, scaled by layers" + (" + LM-head FLOP share" if with_lm_head else ""),
-            "host_cpus": os.cpu_count()}
+    lm = (2.0 * int(np.asarray(a["sample_idx"]).shape[0]) * m.hidden * m.vocab if with_lm_head else 0.0)
+    scale = n_layers + lm / _layer_flops(m, T)
+    sec = _oracle_layer_time(m, a, W)
+    sec1 = None
+    try:
+        from threadpoolctl import threadpool_limits
+        with threadpool_limits(limits=1):
+            sec1 = _oracle_layer_time(m, a, W)
+    except Exception:
+        pass
+    return {"value": round(T / (sec * scale), 2), "unit": UNIT, "cores": int(_blas_threads()), "kind": "oracle",
+            "sample": f"measured: oracle fp32 forward of 1 decoder layer on the first timed tick's whole batch "
+                      f"(T={T}): {sec:.2f} s on {_blas_threads()} threads; value = T / (that time x {scale:.2f} "
+                      f"layer-equivalents of the stage)",
+            "one_thread": ({"value": round(T / (sec1 * scale), 3), "layer_s": round(sec1, 2)} if sec1 else None),
+            "layer_s": round(sec, 3), "cpu_model": _cpu_model(), "host_cpus": os.cpu_count()}
 
 
 def run_reference(args):
-    """--impl reference: the oracle as it stands on the host cores, K bounded-sample steps."""
+    """--impl reference: the oracle as it stands on the host cores.  Each step is a bounded sample of
+    that tick's workload: one decoder layer over the tick's whole batch, timed for real; ms_per_step
+    is that measured time, `value` expresses it for the whole model (x layers + LM-head share)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -517,37 +541,34 @@ def run_reference(args):
         s.build_batch()
     W = Weights(m)
     W.layer(0)
-    tot_tokens, tot_sec = 0, 0.0
-    sample_desc = None
+    tot_tokens, tot_equiv, tot_meas = 0, 0.0, 0.0
+    t_start = time.perf_counter()
     for i in range(args.warmup + args.steps):
         b = s.build_batch()
         a = dict(token_ids=b.token_ids, positions=b.positions, slot_mapping=b.slot_mapping, cu_q=b.cu_q,
                  kv_len=b.kv_len, block_table=b.block_table, sample_idx=b.sample_idx, num_tokens=b.num_tokens)
-        if b.num_tokens == 0:
+        if b.num_tokens == 0 or i < args.warmup:   # (the oracle has nothing to warm up)
             continue
-        # bounded sample: the first 256 tokens' sequences would change the workload; instead time
-        # one decoder layer of the batch and scale to the whole model (as cpu_baseline)
-        sec = _oracle_layer_time(m, a, W, 1)
+        sec = _oracle_layer_time(m, a, W)
         T = b.num_tokens
-        layer_flops = 2.0 * T * (m.hidden * (m.q_dim + 2 * m.kv_dim) + m.q_dim * m.hidden + 3 * m.hidden * m.intermediate)
-        lm_flops = 2.0 * len(b.sample_idx) * m.hidden * m.vocab
-        est = sec * (m.n_layers + lm_flops / layer_flops)
+        scale = m.n_layers + 2.0 * len(b.sample_idx) * m.hidden * m.vocab / _layer_flops(m, T)
         if i >= args.warmup:
             tot_tokens += T
-            tot_sec += est
-            sample_desc = f"per step: oracle fp32 forward of 1 of {m.n_layers} layers on that tick's batch, scaled"
-    try:
-        from threadpoolctl import threadpool_info
-        threads = max((p.get("num_threads", 1) for p in threadpool_info()), default=os.cpu_count())
-    except Exception:
-        threads = os.cpu_count()
-    v = tot_tokens / tot_sec if tot_sec > 0 else 0.0
+            tot_meas += sec
+            tot_equiv += sec * scale
+    wall = time.perf_counter() - t_start
+    v = tot_tokens / tot_equiv if tot_equiv > 0 else 0.0
+    sample = (f"per step: the oracle's fp32 forward of 1 of {m.n_layers} decoder layers over that tick's whole batch, "
+              f"measured ({tot_meas / max(args.steps, 1):.2f} s/step); value = tokens / (measured time x layers + "
+              f"LM-head share)")
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 2), "unit": UNIT, "n_gpus": N,
-           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_sec / max(args.steps, 1) * 1e3, 1),
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot_meas / max(args.steps, 1) * 1e3, 1),
+           "ms_per_step_model_equivalent": round(tot_equiv / max(args.steps, 1) * 1e3, 1),
+           "wall_s": round(wall, 1),
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
            "config": workload_config(args, sp),
-           "cpu_baseline": {"value": round(v, 2), "unit": UNIT, "cores": int(threads), "kind": "oracle",
-                            "sample": sample_desc},
+           "cpu_baseline": {"value": round(v, 2), "unit": UNIT, "cores": int(_blas_threads()), "kind": "oracle",
+                            "sample": sample, "cpu_model": _cpu_model()},
            "e2e": {"value": round(v, 2), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out))
 

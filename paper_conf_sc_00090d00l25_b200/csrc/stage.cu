@@ -532,13 +532,32 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   const int ND = S - NP;
   int split_pages = 1 << 30;
   if (ND > 0) {
-    // split long contexts so that the decode grid has >= ~8 CTAs per SM of work; a split is
-    // at least 32 pages (512 keys) so the merge pass stays negligible
-    // (persistent kernel: one warp worker's fair share -- 8 resident warps per SM -- so only rows
-    // longer than the average per-warp work are split; a split is at least 16 pages)
-    const int64_t target = 8LL * st->num_sms;  // CTAs (v1) / warp workers (persistent kernel)
-    int64_t per = (total_pages * c.n_kv_heads + target - 1) / target;
-    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>(16, per));
+    // Split long rows into equal-length key ranges so that the (row split, kv head) work units fill
+    // the persistent decode kernel's warp workers (8 per SM) in k >= 2 rounds: total units <= k x
+    // workers, with the split length u (pages) as small as that allows (>= 8 pages, so the in-place
+    // merge of a row's partials stays a few % of its bytes).  Longest-first claiming then balances
+    // to within about one unit (C3 window: ~14 rows x 300 pages; a fixed fair-share split left
+    // half the warps idle for a second, tail-sized unit).
+    const int64_t W = 8LL * st->num_sms;
+    const int64_t total = total_pages * c.n_kv_heads;
+    int max_pages = 1;
+    for (int i = NP; i < S; ++i) max_pages = std::max(max_pages, (d->kv_len[i] + bs - 1) / bs);
+    const double F = (double)total / (double)W;
+    const int64_t k = std::max<int64_t>(2, (int64_t)std::ceil(F / 32.0));
+    auto units = [&](int u) {
+      int64_t n = 0;
+      for (int i = NP; i < S; ++i) n += ((d->kv_len[i] + bs - 1) / bs + u - 1) / u;
+      return n * c.n_kv_heads;
+    };
+    int lo = std::max(8, (int)(F / (double)k)), hi = std::max(lo, max_pages);
+    while (lo < hi) {  // smallest u in [lo, max_pages] with units(u) <= k * W (units is non-increasing in u)
+      const int mid = lo + (hi - lo) / 2;
+      if (units(mid) <= k * W)
+        hi = mid;
+      else
+        lo = mid + 1;
+    }
+    split_pages = lo;
   }
   std::vector<gllm::DecodeItem> ditems;
   std::vector<gllm::MergeItem> merges;

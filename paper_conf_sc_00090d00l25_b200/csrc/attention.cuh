@@ -46,6 +46,7 @@ int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const
 // `tmv` map the layer's K / V cache as [kv_blocks*Hkv*16, D] bf16 with 16 x 64 SW128 boxes;
 // `ctr` = 2 device ints, zero before the first launch (the kernel leaves them zero)
 bool decode_tma_supported(int D, int G);
+int decode_workers(int num_sms);  // warp workers of the persistent decode kernel
 int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
                                 const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
                                 int num_sms, cudaStream_t s);

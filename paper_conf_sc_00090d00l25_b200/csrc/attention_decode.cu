@@ -280,37 +280,60 @@ __global__ void __launch_bounds__(WARPS * 32)
         if (prev == c_nsplit - 1) {
           __threadfence();
           if (lane == 0) a.part_ctr[(size_t)first * Hkv + c_kvh] = 0;  // ready for the next launch
-          // lane owns elements lane + 32k of the G x D output; all loads of one split are
-          // independent (issued together), so the merge costs ~nsplit L2 round trips
+          // Merge of the row's nsplit partials, latency-tolerant: (1) lane l reduces the (max, sum)
+          // statistics of splits l, l + 32, ... (independent loads), combined across the warp in a
+          // fixed order; (2) lane l owns output elements l + 32k and accumulates the splits' O
+          // rows four splits per step, so four independent loads per element are in flight
+          // (a dependent L2 round trip per split made long rows' merges dominate small batches).
           constexpr int PER = G * D / 32;
           const int t = a.cu_q[c_seq];
-          float M[G], Ls[G], acc[PER];
+          const size_t pbase = (size_t)first * Hkv + c_kvh;  // split sp's (G, D) block: (pbase + sp*Hkv)*G
+          float M[G], Ls[G];
+#pragma unroll
+          for (int h = 0; h < G; ++h) M[h] = -INFINITY;
+          for (int sp = lane; sp < c_nsplit; sp += 32) {
+#pragma unroll
+            for (int h = 0; h < G; ++h) M[h] = fmaxf(M[h], __ldcg(a.part_ml + ((pbase + (size_t)sp * Hkv) * G + h) * 2));
+          }
 #pragma unroll
           for (int h = 0; h < G; ++h) {
-            M[h] = -INFINITY;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) M[h] = fmaxf(M[h], __shfl_xor_sync(0xffffffffu, M[h], o));
             Ls[h] = 0.f;
           }
-#pragma unroll
-          for (int k = 0; k < PER; ++k) acc[k] = 0.f;
-          for (int sp = 0; sp < c_nsplit; ++sp) {
-            const size_t b0 = ((size_t)(first + sp) * Hkv + c_kvh) * G;
-#pragma unroll
-            for (int h = 0; h < G; ++h) M[h] = fmaxf(M[h], __ldcg(a.part_ml + (b0 + h) * 2));
-          }
-          for (int sp = 0; sp < c_nsplit; ++sp) {
-            const size_t b0 = ((size_t)(first + sp) * Hkv + c_kvh) * G;
-            float f[G];
+          for (int sp = lane; sp < c_nsplit; sp += 32) {
 #pragma unroll
             for (int h = 0; h < G; ++h) {
-              const float2 ml = __ldcg(reinterpret_cast<const float2*>(a.part_ml + (b0 + h) * 2));
-              f[h] = exp2f(ml.x - M[h]);
-              Ls[h] += ml.y * f[h];
+              const float2 ml = __ldcg(reinterpret_cast<const float2*>(a.part_ml + ((pbase + (size_t)sp * Hkv) * G + h) * 2));
+              Ls[h] += ml.y * exp2f(ml.x - M[h]);
+            }
+          }
+#pragma unroll
+          for (int h = 0; h < G; ++h)
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) Ls[h] += __shfl_xor_sync(0xffffffffu, Ls[h], o);
+          float acc[PER];
+#pragma unroll
+          for (int k = 0; k < PER; ++k) acc[k] = 0.f;
+          constexpr int QU = PER >= 32 ? 2 : 4;  // splits per step (register budget at G = 8)
+          for (int sp0 = 0; sp0 < c_nsplit; sp0 += QU) {
+            float v[QU][PER], f[QU][G];
+#pragma unroll
+            for (int q = 0; q < QU; ++q) {
+              const int sp = min(sp0 + q, c_nsplit - 1);
+              const size_t b0 = (pbase + (size_t)sp * Hkv) * G;
+#pragma unroll
+              for (int h = 0; h < G; ++h) {
+                const float mm = __ldcg(a.part_ml + (b0 + h) * 2);
+                f[q][h] = sp0 + q < c_nsplit ? exp2f(mm - M[h]) : 0.f;
+              }
+#pragma unroll
+              for (int k = 0; k < PER; ++k) v[q][k] = __ldcg(a.part_o + b0 * D + lane + 32 * k);
             }
 #pragma unroll
-            for (int k = 0; k < PER; ++k) {
-              const int idx = lane + 32 * k;
-              acc[k] += __ldcg(a.part_o + b0 * D + idx) * f[idx / D];
-            }
+            for (int q = 0; q < QU; ++q)
+#pragma unroll
+              for (int k = 0; k < PER; ++k) acc[k] += v[q][k] * f[q][(lane + 32 * k) / D];
           }
 #pragma unroll
           for (int k = 0; k < PER; ++k) {
@@ -363,6 +386,8 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
 template <int D, int G>
 int launch_g(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items, int n_items,
              const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
+  // 3-slot page ring x 4 warps, 2 CTAs per SM (profiles/r02/decode_split_ab.txt: 6 slots x 4 warps at
+  // 1 CTA per SM is 15-25% slower -- the per-page mma.sync work of fewer warps limits it)
   return launch_t<D, G, 3, 4>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
 }
 
@@ -380,6 +405,10 @@ int launch_d(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
 }
 
 }  // namespace
+
+int decode_workers(int num_sms) {  // warp workers of the persistent decode kernel (host split policy)
+  return 8 * num_sms;  // 2 CTAs of 4 warps per SM
+}
 
 bool decode_tma_supported(int D, int G) { return (D == 64 || D == 128) && (G == 1 || G == 2 || G == 4 || G == 5 || G == 8); }
 

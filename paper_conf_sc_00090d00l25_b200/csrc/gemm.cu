@@ -18,6 +18,7 @@
 //   warps 4-7: epilogue (warp 4+i reads TMEM lanes 32i..32i+31)
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -92,6 +93,28 @@ __device__ __forceinline__ void umma_commit_cg2(uint64_t* bar) {
       "h"((uint16_t)3)
       : "memory");
 }
+// distributed shared memory: the address of `addr` in cluster CTA `rank`, and a 16-byte load there
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ float4 ld_dsmem_v4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(addr)
+               : "memory");
+  return v;
+}
+// cluster split-K: each CTA's fp32 partial tile [128 rows][256 cols] in its own SMEM, row stride 260
+// floats (conflict-free 16-byte accesses when thread = row)
+constexpr int CL_STRIDE = GEMM_BN + 4;
+struct ClSrc {
+  uint32_t part;  // local SMEM address of the partial tile (0: not cluster split-K)
+  int S, r;       // cluster size, this CTA's rank
+};
+
 // arrive on the leader CTA's copy of a barrier (from either CTA of the pair)
 __device__ __forceinline__ void mbar_arrive_leader(uint64_t* bar) {
   asm volatile(
@@ -144,6 +167,14 @@ struct Jobs {
     u1 = min(total, u + per);
   }
   __device__ bool next(int& tile, int& kb0, int& kb1) {
+    if (mode == 3) {  // cluster split-K: one (tile, k range) per CTA; unit = the CTA index
+      if (it++ > 0) return false;
+      const int S = per, r = unit % S;
+      tile = unit / S;
+      kb0 = r * nk / S;
+      kb1 = (r + 1) * nk / S;
+      return true;
+    }
     if (mode == 0 || (mode == 2 && unit + it * nunits < dp_tiles)) {
       tile = unit + it * nunits;
       ++it;
@@ -232,8 +263,21 @@ __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: 
 template <int EPI>
 __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
                                               uint64_t* tfull_bar, uint32_t parity, float* stg, int tile,
-                                              int contrib, int* fix_flag) {
+                                              int contrib, int* fix_flag, ClSrc cl = ClSrc{0u, 1, 0}) {
   const bool row_ok = row < p.M;
+  const bool from_cl = cl.part != 0u;  // cluster split-K: sums of the cluster's partial tiles (DSMEM)
+  // column chunks (32 wide) this CTA finishes: all, or (cluster split-K) its share of the tile's
+  // epilogue units -- a chunk, or a rotate-half / gate-up chunk pair
+  auto own = [&](int c) {
+    if (!from_cl) return true;
+    int unit = c;
+    if constexpr (EPI == EPI_QKV_ROPE) {
+      const int per_head = p.head_dim / 32;
+      unit = (c / per_head) * (per_head / 2) + c % per_head;
+    }
+    return unit % cl.S == cl.r;
+  };
+  const uint32_t cl_row = cl.part + (uint32_t)((threadIdx.x & 127) * CL_STRIDE * 4);
   const float rs = (EPI == EPI_ADD_F32 || EPI == EPI_ARGMAX) ? 1.0f : row_scale(p, row);
   uint32_t r[32];
   auto wait_acc = [&]() {
@@ -253,7 +297,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     }
   }
   bool from_ws = false;  // this CTA finishes a stream-K tile from the workspace sums
-  if (p.ws != nullptr && (partial || p.tile_ctr == nullptr)) {  // (legacy mode: every segment via ws)
+  if (!from_cl && p.ws != nullptr && (partial || p.tile_ctr == nullptr)) {  // (legacy mode: every segment via ws)
     wait_acc();
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
@@ -274,11 +318,30 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     if (threadIdx.x == 128) p.tile_ctr[tile] = 0;
     from_ws = true;
   }
-  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && (!partial || from_ws)) p.zero_rows[row] = 0.f;
+  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && (!partial || from_ws) && cl.r == 0) p.zero_rows[row] = 0.f;
   float* wrow = p.ws + (size_t)(row_ok ? row : 0) * p.N + n_blk * GEMM_BN;
   // accumulator columns [col, col + 32) of this tile's row: from TMEM or (finisher) from ws,
   // re-zeroing ws behind the read
   auto ld = [&](int col, uint32_t(&v)[32]) {
+    if (from_cl) {  // fixed rank order: deterministic sums
+      float f[32];
+#pragma unroll
+      for (int q = 0; q < 32; ++q) f[q] = 0.f;
+      for (int src = 0; src < cl.S; ++src) {
+        const uint32_t a = mapa_u32(cl_row + col * 4, (uint32_t)src);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+          const float4 x = ld_dsmem_v4(a + 16 * q);
+          f[4 * q] += x.x;
+          f[4 * q + 1] += x.y;
+          f[4 * q + 2] += x.z;
+          f[4 * q + 3] += x.w;
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 32; ++q) v[q] = __float_as_uint(f[q]);
+      return;
+    }
     if (!from_ws) {
       ptx::tmem_ld_32x32b_x32(tbase + col, v);
       return;
@@ -300,16 +363,17 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     }
   };
   auto ld_wait = [&]() {
-    if (!from_ws) ptx::tmem_ld_wait();
+    if (!from_ws && !from_cl) ptx::tmem_ld_wait();
   };
   auto wait_src = [&]() {
-    if (!from_ws) wait_acc();
+    if (!from_ws && !from_cl) wait_acc();
   };
   if constexpr (EPI == EPI_STORE_BF16) {
     wait_src();
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out);
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
+      if (!own(c)) continue;
       ld(c * 32, r);
       ld_wait();
       const int col0 = n_blk * GEMM_BN + c * 32;
@@ -355,8 +419,8 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
         }
       };
       auto combine = [&](int c, const float4(&xv)[8]) {
-        ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
-        ptx::tmem_ld_wait();
+        ld(c * 32, r);
+        ld_wait();
 #pragma unroll
         for (int q = 0; q < 8; ++q)  // row `lane` of the chunk (stride 36 floats: conflict-free v4)
           *reinterpret_cast<float4*>(stg + lane * 36 + 4 * q) =
@@ -389,14 +453,30 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
         __syncwarp();
       };
       float4 xa[8], xb[8];
-      load_x(0, xa);
-      wait_acc();
+      if (from_cl) {  // this CTA's chunks of the tile, summed over the cluster
+        int c = 0;
+        while (c < GEMM_BN / 32 && !own(c)) ++c;
+        if (c < GEMM_BN / 32) load_x(c, xa);
 #pragma unroll 1
-      for (int c = 0; c < GEMM_BN / 32; c += 2) {
-        load_x(c + 1, xb);
-        combine(c, xa);
-        if (c + 2 < GEMM_BN / 32) load_x(c + 2, xa);
-        combine(c + 1, xb);
+        while (c < GEMM_BN / 32) {
+          int cn = c + 1;
+          while (cn < GEMM_BN / 32 && !own(cn)) ++cn;
+          if (cn < GEMM_BN / 32) load_x(cn, xb);
+          combine(c, xa);
+#pragma unroll
+          for (int k = 0; k < 8; ++k) xa[k] = xb[k];
+          c = cn;
+        }
+      } else {
+        load_x(0, xa);
+        wait_acc();
+#pragma unroll 1
+        for (int c = 0; c < GEMM_BN / 32; c += 2) {
+          load_x(c + 1, xb);
+          combine(c, xa);
+          if (c + 2 < GEMM_BN / 32) load_x(c + 2, xa);
+          combine(c + 1, xb);
+        }
       }
       if (p.ss_out) {  // row rsub + 4k: its 32 columns of this tile are spread over 8 lanes
 #pragma unroll
@@ -416,6 +496,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
     uint32_t u[32];
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 64; ++c) {
+      if (!own(c)) continue;
       ld(c * 32, r);                // gate columns
       ld(GEMM_BN / 2 + c * 32, u);  // up columns
       ld_wait();
@@ -438,7 +519,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
       const int hpos = c % per_head;
-      if (hpos >= per_head / 2) continue;
+      if (hpos >= per_head / 2 || !own(c)) continue;
       ld(c * 32, r);
       ld((c + per_head / 2) * 32, u);
       ld_wait();
@@ -496,6 +577,7 @@ __global__ void __launch_bounds__(256, 1)
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const bool skc = p.streamk == 3;  // cluster split-K (CG = 1 kernel launched in clusters of split_s)
   const uint32_t rank = CG == 2 ? cluster_rank() : 0;
   const bool leader = rank == 0;
   pdl_trigger();
@@ -516,7 +598,7 @@ __global__ void __launch_bounds__(256, 1)
   }
   if (warp == 2) tmem_alloc_cg<CG>(tmem_ptr, TMEM_COLS);
   ptx::tc_fence_before();
-  if constexpr (CG == 2)
+  if (CG == 2 || skc)
     cluster_sync_all();
   else
     __syncthreads();
@@ -528,7 +610,7 @@ __global__ void __launch_bounds__(256, 1)
 
   const int num_m = (p.M + C::TILE_M - 1) / C::TILE_M;
   Jobs jobs;
-  jobs.init(p, blockIdx.x / CG, gridDim.x / CG, num_m);
+  jobs.init(p, skc ? (int)blockIdx.x : (int)blockIdx.x / CG, gridDim.x / CG, num_m);
   int tile, kb0, kb1;
 
   if (warp == 0) {
@@ -630,6 +712,27 @@ __global__ void __launch_bounds__(256, 1)
         if (acc == 0) acc_phase ^= 1;
       }
     }
+  } else if (warp >= 4 && skc) {
+    // ---------------- cluster split-K: this CTA's partial tile -> its SMEM (the operand ring is
+    // idle: every stage was consumed by the MMAs the tfull commit covers)
+    if (jobs.next(tile, kb0, kb1)) {
+      ptx::mbar_wait(&tfull[0], 0);
+      ptx::tc_fence_after();
+      const int rl = (warp - 4) * 32 + lane;
+      const uint32_t tb = tmem_base + ((uint32_t)((warp - 4) * 32) << 16);
+      float* dst = reinterpret_cast<float*>(sA) + rl * CL_STRIDE;
+      uint32_t r[32];
+#pragma unroll 1
+      for (int c = 0; c < GEMM_BN / 32; ++c) {
+        ptx::tmem_ld_32x32b_x32(tb + c * 32, r);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          *reinterpret_cast<float4*>(dst + c * 32 + 4 * q) =
+              make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]), __uint_as_float(r[4 * q + 2]),
+                          __uint_as_float(r[4 * q + 3]));
+      }
+    }
   } else if (warp >= 4) {
     // ---------------- epilogue warps (each CTA drains its own 128 rows)
     const int ew = warp - 4;
@@ -659,11 +762,32 @@ __global__ void __launch_bounds__(256, 1)
       if (acc == 0) acc_phase ^= 1;
     }
   }
-  ptx::tc_fence_before();
-  if constexpr (CG == 2)
+  if (skc) {
+    // every partial of the cluster is in SMEM: each CTA reduces its share of the tile's column
+    // chunks over DSMEM (rank order) and runs the epilogue; the second cluster barrier keeps every
+    // CTA's SMEM alive until the last remote read
     cluster_sync_all();
-  else
-    __syncthreads();
+    if (warp >= 4) {
+      Jobs ej;
+      ej.init(p, blockIdx.x, gridDim.x, num_m);
+      if (ej.next(tile, kb0, kb1)) {
+        const int ew = warp - 4;
+        const int m_blk = tile % num_m, n_blk = tile / num_m;
+        const int row = m_blk * C::TILE_M + ew * 32 + lane;
+        epilogue_tile<EPI>(p, tmem_base + ((uint32_t)(ew * 32) << 16), row, n_blk, false, &tfull[0], 0,
+                           stg + ew * C::STG_FLOATS, tile, 1, fix_flag,
+                           ClSrc{ptx::smem_u32(sA), p.split_s, (int)cluster_rank()});
+      }
+    }
+    ptx::tc_fence_before();
+    cluster_sync_all();
+  } else {
+    ptx::tc_fence_before();
+    if constexpr (CG == 2)
+      cluster_sync_all();
+    else
+      __syncthreads();
+  }
   if (warp == 2) {
     ptx::tc_fence_after();
     tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
@@ -820,10 +944,22 @@ int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms, bool ws_o
   return ntiles - tail;
 }
 
+// Cluster split-K (Jobs mode 3) for small-T, few-tile GEMMs (weight streaming, e.g. C4's QKV / O /
+// down at T ~ 128): one M tile, tiles x S <= SMs with S = the k-split per tile (2..8, at most the
+// epilogue's units per tile: 8 chunks, or 4 chunk pairs for RoPE / SiLU).  Returns S (0 = not used).
+int skc_split(int M, int N, int K, int epi, int num_sms) {
+  if (M > GEMM_BM || epi == EPI_ARGMAX) return 0;
+  const int ntiles = (N + GEMM_BN - 1) / GEMM_BN, nk = K / GEMM_BK;
+  const int cap = (epi == EPI_SILU_MUL || epi == EPI_QKV_ROPE) ? 4 : 8;
+  const int S = std::min(std::min(cap, num_sms / std::max(ntiles, 1)), nk / 4);
+  return S >= 2 ? S : 0;
+}
+
 }  // namespace
 
 bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms) {
   if (M <= 0) return false;
+  if (!g_force_cg && skc_split(M, N, K, epi, num_sms)) return false;  // whole tiles, reduced in-cluster
   const int cg = choose_cg(M, N, epi, num_sms);
   if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms, false) > 0;
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
@@ -881,7 +1017,9 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
   const int num_m = (args.M + C::TILE_M - 1) / C::TILE_M;
   const int ntiles = num_m * args.num_n_tiles;
   int grid;
-  if (args.streamk == 1) {
+  if (args.streamk == 3) {
+    grid = ntiles * args.split_s;
+  } else if (args.streamk == 1) {
     const int total = ntiles * (args.K / GEMM_BK);
     grid = (total + args.units_per_cta - 1) / args.units_per_cta;
   } else if (args.streamk == 2) {
@@ -892,7 +1030,8 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
   }
   if (grid <= 0) return GLLM_OK;
   {
-    cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, CG, a, b, args);
+    const int cluster = args.streamk == 3 ? args.split_s : CG;
+    cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, cluster, a, b, args);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (%d-CTA) launch: %s", CG, cudaGetErrorString(e));
   }
   if (args.ws && !args.tile_ctr) {
@@ -923,6 +1062,15 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   args.streamk = cg == 1 ? choose_streamk(args.M, args.N, ntiles, nk, epi, num_sms) : 0;
   args.units_per_cta = args.streamk ? (ntiles * nk + num_sms - 1) / num_sms : 0;
   args.dp_tiles = 0;
+  args.split_s = 0;
+  if (cg == 1 && !g_force_cg) {
+    const int S = skc_split(args.M, args.N, args.K, epi, num_sms);
+    if (S > 0) {  // cluster split-K replaces stream-K: no workspace, no atomics, no finish pass
+      args.streamk = 3;
+      args.split_s = S;
+      args.units_per_cta = S;
+    }
+  }
   bool hybrid = false;
   if (cg == 2 && !args.xb_out && !args.ss_out && !args.out_peer) {  // partial tiles: no fused outputs
     const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms, args0.ws && args0.tile_ctr);
@@ -935,7 +1083,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
     }
   }
   if (!g_sk_fixup) args.tile_ctr = nullptr;  // memset + finish pass (see hybrid_dp_tiles)
-  if (args.streamk && epi != EPI_ADD_F32) {
+  if (args.streamk && args.streamk != 3 && epi != EPI_ADD_F32) {
     if (!args0.ws) return set_error(GLLM_EINVAL, "gemm: stream-K workspace required");
     if (!hybrid && args.tile_ctr && ntiles > GEMM_MAX_SK_TILES) args.tile_ctr = nullptr;  // legacy memset + finish
   } else {

@@ -35,7 +35,11 @@ struct GemmArgs {
   // into the fp32 workspace `ws` [M, N], finished by gemm_finish_kernel.
   // 2 = hybrid (CTA pairs, residual add only): whole tiles [0, dp_tiles) round robin, then
   // stream-K over the remaining tiles' k-blocks (units_per_cta per pair), partial tiles reduced.
-  int streamk, units_per_cta, dp_tiles;
+  // 3 = cluster split-K (CG=1, M <= 128, few tiles): each tile's k-blocks are split evenly over a
+  // cluster of split_s CTAs; partial accumulators meet in shared memory and every CTA reduces its
+  // share of the tile's column chunks over DSMEM in fixed rank order and runs the epilogue
+  // (no atomics, no workspace, no finish pass; deterministic).
+  int streamk, units_per_cta, dp_tiles, split_s;
   // B (the weights) is never written by a kernel on the stream: with PDL the producer issues the
   // first ring fill's B tiles before griddepcontrol.wait (stage GEMMs only; gllm_op_gemm leaves 0)
   int b_static;

@@ -532,32 +532,16 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
   const int ND = S - NP;
   int split_pages = 1 << 30;
   if (ND > 0) {
-    // Split long rows into equal-length key ranges so that the (row split, kv head) work units fill
-    // the persistent decode kernel's warp workers (8 per SM) in k >= 2 rounds: total units <= k x
-    // workers, with the split length u (pages) as small as that allows (>= 8 pages, so the in-place
-    // merge of a row's partials stays a few % of its bytes).  Longest-first claiming then balances
-    // to within about one unit (C3 window: ~14 rows x 300 pages; a fixed fair-share split left
-    // half the warps idle for a second, tail-sized unit).
-    const int64_t W = 8LL * st->num_sms;
-    const int64_t total = total_pages * c.n_kv_heads;
+    // Split rows longer than one warp worker's fair share of the (page, kv head) units, so the
+    // persistent decode kernel's warps (8 per SM) get equal work; a split is at least 16 pages (and
+    // a row at most 32 splits) so the in-place merge stays a few % of the row's bytes.  Measured on
+    // B200 (profiles/r02/decode_split_ab.txt) against equal-length splits filling the workers in
+    // k >= 2 rounds: the fair-share split is faster on C1 (800 rows) and on C3's few long rows.
+    const int64_t W = gllm::decode_workers(st->num_sms);
     int max_pages = 1;
     for (int i = NP; i < S; ++i) max_pages = std::max(max_pages, (d->kv_len[i] + bs - 1) / bs);
-    const double F = (double)total / (double)W;
-    const int64_t k = std::max<int64_t>(2, (int64_t)std::ceil(F / 32.0));
-    auto units = [&](int u) {
-      int64_t n = 0;
-      for (int i = NP; i < S; ++i) n += ((d->kv_len[i] + bs - 1) / bs + u - 1) / u;
-      return n * c.n_kv_heads;
-    };
-    int lo = std::max(8, (int)(F / (double)k)), hi = std::max(lo, max_pages);
-    while (lo < hi) {  // smallest u in [lo, max_pages] with units(u) <= k * W (units is non-increasing in u)
-      const int mid = lo + (hi - lo) / 2;
-      if (units(mid) <= k * W)
-        hi = mid;
-      else
-        lo = mid + 1;
-    }
-    split_pages = lo;
+    const int64_t per = (total_pages * c.n_kv_heads + W - 1) / W;
+    split_pages = (int)std::min<int64_t>(256, std::max<int64_t>({16, per, (max_pages + 31) / 32}));
   }
   std::vector<gllm::DecodeItem> ditems;
   std::vector<gllm::MergeItem> merges;

@@ -101,8 +101,8 @@ def test_argmax_epilogue(M, N):
     ref = _ref(A, W)
     ids = out.cpu().numpy()
     # fp32 accumulation vs fp64: the chosen logit must be the max up to accumulation error
+    # (tolerance-aware greedy: several ids are correct when logits tie within rounding)
     assert np.all(ref[np.arange(M), ids] >= ref.max(-1) - 1e-4 * np.abs(ref).max(-1))
-    assert np.mean(ids == ref.argmax(-1)) >= 0.9
 
 
 def test_bad_shapes_are_einval():
@@ -110,3 +110,46 @@ def test_bad_shapes_are_einval():
     with pytest.raises(gllm.GllmError) as e:
         gllm.op_gemm(A.data_ptr(), A.data_ptr(), 4, 4, 100, 0, A.data_ptr())
     assert e.value.code == -1
+
+
+@pytest.mark.parametrize("M,N,K,epi", [(128, 10240, 8192, 0), (96, 8192, 8192, 1), (128, 8192, 28672, 1),
+                                       (64, 2048, 4096, 2), (17, 6144, 4096, 0)])
+def test_small_t_weight_streaming_shapes_deterministic(M, N, K, epi, variant):
+    # C4's small-T projections (T <= 128: one M tile, few N tiles -> cluster split-K in the automatic
+    # schedule, the k-split partials reduced over DSMEM in rank order): parity with fp64, and two runs
+    # bit-identical unless the forced 1-CTA variant takes stream-K (fp32 atomics)
+    A = _bf16((M, K), 1.0, 20)
+    if epi == 2:
+        I = N // 2
+        Wg, Wu = _bf16((I, K), K ** -0.5, 21), _bf16((I, K), K ** -0.5, 23)
+        W = torch.empty((N, K), dtype=torch.bfloat16)
+        for j in range(I // 128):
+            W[256 * j:256 * j + 128] = Wg[128 * j:128 * j + 128]
+            W[256 * j + 128:256 * j + 256] = Wu[128 * j:128 * j + 128]
+    else:
+        W = _bf16((N, K), K ** -0.5, 21)
+    dA, dW = A.cuda(), W.cuda()
+    x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(22))
+    outs = []
+    for _ in range(2):
+        if epi == 1:
+            out = x0.clone().cuda()
+        elif epi == 2:
+            out = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+        else:
+            out = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, epi, out.data_ptr())
+        torch.cuda.synchronize()
+        outs.append(out.float().cpu().numpy())
+    if epi == 1:
+        assert np.abs(outs[0] - (x0.double().numpy() + _ref(A, W))).max() < 1e-3
+    else:
+        if epi == 2:
+            g, u = _ref(A, Wg), _ref(A, Wu)
+            ref = g / (1 + np.exp(-g)) * u
+        else:
+            ref = _ref(A, W)
+        err = np.abs(outs[0] - ref).max(-1) / np.abs(ref).max(-1)
+        assert err.max() < 1e-2, err.max()
+    if variant != 1:
+        assert np.array_equal(outs[0], outs[1]), "non-deterministic result"

@@ -21,7 +21,7 @@ import torch
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sc_00090d00l25_b200 import gllm  # noqa: E402
-from paper_conf_sc_00090d00l25_b200.runtime import split_layers  # noqa: E402
+from paper_conf_sc_00090d00l25_b200.runtime import fill_warm, split_layers  # noqa: E402
 from workloads.configs import MODELS, SCHED, STREAMS  # noqa: E402
 from workloads.streams import make_stream  # noqa: E402
 
@@ -52,7 +52,10 @@ def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_
         if d.num_tokens:
             fwd(d)
     torch.cuda.synchronize()
+    pre0 = s.stats()["preemptions"]
     times, toks, pre, dec = [], [], [], []
+    samples = []   # per tick: request ids whose next token is sampled (prompt completions + decodes)
+    k0 = s.stats()["tick"]
     for _ in range(ticks):
         d = s.build_batch()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -65,8 +68,32 @@ def measure(config, pp, stage_idx, policy, preroll, ticks, kv_blocks=None, host_
         toks.append(d.num_tokens)
         pre.append(d.num_prefill_tokens)
         dec.append(d.num_decode_tokens)
+        a = d.to_numpy()
+        cu, rid = a["cu_q"], a["seq_req_ids"]
+        seq_of = np.searchsorted(cu, a["sample_idx"], side="right") - 1 if d.num_tokens else np.zeros(0, int)
+        samples.append([int(rid[i]) for i in seq_of])
+    preempt = s.stats()["preemptions"] - pre0
     st.close()
-    return np.array(times), np.array(toks), np.array(pre), np.array(dec)
+    arrivals = {r.req_id: r.arrival_tick - k0 for r in make_stream(config, m.vocab).requests}
+    return np.array(times), np.array(toks), np.array(pre), np.array(dec), samples, arrivals, preempt
+
+
+def latencies(samples, arrivals, start, fin):
+    """Tick-based serving proxies on the simulated pipeline (§4.6's metrics, Fig. 16): TTFT =
+    finish of the micro-batch that completes a prompt - start of the tick the request arrived in;
+    TPOT = mean gap between a request's consecutive sampled tokens.  Only requests arriving inside
+    the measured window count for TTFT."""
+    first, last, gaps = {}, {}, []
+    for k, ids in enumerate(samples):
+        for r in ids:
+            if r not in first:
+                first[r] = k
+            elif r in last:
+                gaps.append(fin[k] - fin[last[r]])
+            last[r] = k
+    ttft = [fin[k] - start[arrivals[r]] for r, k in first.items()
+            if r in arrivals and 0 <= arrivals[r] < len(start) and k >= arrivals[r]]
+    return (float(np.mean(ttft)) if ttft else None, float(np.mean(gaps)) if gaps else None, len(ttft))
 
 
 def simulate(t_ms, pp, host_ms=0.05):
@@ -85,7 +112,8 @@ def simulate(t_ms, pp, host_ms=0.05):
             fin[s, k] = start + t_ms[k]
     makespan = fin[pp - 1, n - 1]
     busy = pp * float(np.sum(t_ms))
-    return makespan, 1.0 - busy / (pp * makespan)
+    start0 = fin[0] - t_ms   # when micro-batch k entered stage 0
+    return makespan, 1.0 - busy / (pp * makespan), start0, fin[pp - 1]
 
 
 if __name__ == "__main__":
@@ -112,10 +140,14 @@ if __name__ == "__main__":
     if a.sweep:
         key, vals = a.sweep.split("=")
         runs = [(f"{key}={v}", 0, {key: int(v)}) for v in vals.split(",")]
+        out["sweep"] = key
     for name, pol, kw in runs:
-        t, toks, pre, dec = measure(a.config, a.pp, a.stage, pol, preroll, a.ticks, **kw)
-        mk, bub = simulate(t, a.pp)
+        t, toks, pre, dec, samples, arrivals, preempt = measure(a.config, a.pp, a.stage, pol, preroll, a.ticks, **kw)
+        mk, bub, start0, fin_last = simulate(t, a.pp)
+        ttft, tpot, n_ttft = latencies(samples, arrivals, start0, fin_last)
         out[name] = {"tokens_per_s": round(float(toks.sum()) / (mk * 1e-3), 1), "bubble_fraction": round(bub, 4),
+                     "preemptions": int(preempt), "ttft_ms": round(ttft, 2) if ttft is not None else None,
+                     "ttft_requests": n_ttft, "tpot_ms": round(tpot, 3) if tpot is not None else None,
                      "stage_ms_mean": round(float(t.mean()), 3), "stage_ms_cv": round(float(t.std() / t.mean()), 3),
                      "tokens_mean": round(float(toks.mean()), 1), "tokens_cv": round(float(toks.std() / toks.mean()), 3),
                      "prefill_mean": round(float(pre.mean()), 1), "decode_mean": round(float(dec.mean()), 1)}

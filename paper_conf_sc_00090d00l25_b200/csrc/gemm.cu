@@ -944,11 +944,14 @@ int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms, bool ws_o
   return ntiles - tail;
 }
 
-// Cluster split-K (Jobs mode 3) for small-T, few-tile GEMMs (weight streaming, e.g. C4's QKV / O /
-// down at T ~ 128): one M tile, tiles x S <= SMs with S = the k-split per tile (2..8, at most the
-// epilogue's units per tile: 8 chunks, or 4 chunk pairs for RoPE / SiLU).  Returns S (0 = not used).
+// Cluster split-K (Jobs mode 3) for small-T, few-tile GEMMs with a non-additive epilogue (C4's QKV at
+// T ~ 128): one M tile, tiles x S <= SMs with S = the k-split per tile (2..8, at most the epilogue's
+// units per tile: 8 chunks, or 4 chunk pairs for RoPE / SiLU).  It replaces stream-K's fp32 workspace
+// + finish pass (C4 QKV 60 -> 50 us, profiles/r02/gemm_small_t.txt).  The residual-add epilogue keeps
+// stream-K (vector reductions straight into the residual): its cluster variant measured ~15 us of
+// extra fixed cost per launch (O 38 -> 51 us).  Returns S (0 = not used).
 int skc_split(int M, int N, int K, int epi, int num_sms) {
-  if (M > GEMM_BM || epi == EPI_ARGMAX) return 0;
+  if (M > GEMM_BM || epi == EPI_ARGMAX || epi == EPI_ADD_F32) return 0;
   const int ntiles = (N + GEMM_BN - 1) / GEMM_BN, nk = K / GEMM_BK;
   const int cap = (epi == EPI_SILU_MUL || epi == EPI_QKV_ROPE) ? 4 : 8;
   const int S = std::min(std::min(cap, num_sms / std::max(ntiles, 1)), nk / 4);

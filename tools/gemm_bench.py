@@ -23,21 +23,34 @@ SHAPES = {
     # C3's O shape with the plain store epilogue, and with K cut to 512 / 1024 (prologue + epilogue
     # dominated): separates the residual epilogue's cost from the mainloop's
     "C3s": [(900, 5120, 5120, 0), (900, 5120, 512, 1), (900, 5120, 512, 0), (900, 5120, 1024, 1), (900, 5120, 1024, 0)],
+    # small-T fixed vs per-k-block cost: C4's O shape with K from 1k to 16k (store / residual epilogues)
+    "C4k": [(128, 8192, k, e) for e in (0, 1) for k in (1024, 2048, 4096, 8192, 16384)],
     # the C1 O / down shapes with the plain bf16-store epilogue (isolates the residual epilogue)
     "C1s": [(2094, 4096, 4096, 0), (2094, 4096, 14336, 0)],
 }
+
+
+_FLUSH = None
+
+
+def flush_read():
+    """Evict L2 by READING a 256 MB buffer (clean lines: a write-flush would leave ~126 MB of dirty
+    lines whose write-back the timed kernel then pays for)."""
+    global _FLUSH
+    if _FLUSH is None:
+        _FLUSH = torch.ones(64 << 20, dtype=torch.float32, device="cuda")
+    _FLUSH.sum()
 
 
 def bench_cublas(M, N, K, reps=20):
     """cuBLAS (torch.mm, bf16 out) on the same shape: the library reference for the plain GEMM."""
     A = torch.randn((M, K), device="cuda").to(torch.bfloat16)
     W = (torch.randn((N, K), device="cuda") * K ** -0.5).to(torch.bfloat16)
-    flush = torch.empty(256 << 20, dtype=torch.int8, device="cuda")
     for _ in range(3):
         torch.mm(A, W.t())
     ts = []
     for _ in range(reps):
-        flush.zero_()
+        flush_read()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         torch.mm(A, W.t())
@@ -58,13 +71,12 @@ def bench(M, N, K, epi, reps=20):
         out = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
     else:
         out = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
-    flush = torch.empty(256 << 20, dtype=torch.int8, device="cuda")
     s = torch.cuda.current_stream().cuda_stream
     for _ in range(3):
         gllm.op_gemm(A.data_ptr(), W.data_ptr(), M, N, K, epi, out.data_ptr(), 0, s)
     ts = []
     for _ in range(reps):
-        flush.zero_()
+        flush_read()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         gllm.op_gemm(A.data_ptr(), W.data_ptr(), M, N, K, epi, out.data_ptr(), 0, s)

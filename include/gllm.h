@@ -275,6 +275,13 @@ GLLM_API int gllm_stage_read_slots(gllm_stage* st, int32_t* out, int32_t n);
 GLLM_API int gllm_stage_fill_warm_kv(gllm_stage* st, int32_t n_seqs, const int64_t* req_ids,
                                      const int32_t* context_lens, const int32_t* block_table, int32_t max_blocks);
 
+/* on = 1: every later forward of this stage uses GEMM schedules with a fixed reduction order (whole
+ * tiles or cluster split-K instead of stream-K / hybrid tails, whose fp32 atomic adds make the
+ * last bits depend on arrival order; RMSNorm row statistics from the standalone pass instead of
+ * the epilogue's per-tile atomic sum).  Results are then bitwise reproducible run to run (the
+ * attention kernels always are).  Costs a few % at shapes that would take stream-K.  Default 0. */
+GLLM_API int gllm_stage_set_deterministic(gllm_stage* st, int32_t on);
+
 /* Timing of the forwards since the previous call, from CUDA events recorded on each forward's own
  * stream around each launch (enabled by gllm_stage_set_profiling(st, 1)).  on = 2 also runs the
  * prefill and decode attention kernels in series instead of on two concurrent streams, so that each

@@ -254,16 +254,13 @@ __device__ __forceinline__ float row_scale(const GemmArgs& p, int row) {
 }
 
 // One warp's 32 rows of one 256-column accumulator tile: wait for the MMAs (tfull), drain TMEM,
-// apply the fused epilogue.  `partial`: stream-K segment, combine atomically.  Non-additive
-// epilogues combine partial segments in the fp32 workspace ws: with tile counters (p.tile_ctr)
-// the last of the tile's `contrib` segments to arrive reads the sum back (and re-zeroes ws and
-// the counter) and runs the epilogue itself -- no memset and no finish pass.
-__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
-
+// apply the fused epilogue.  `partial`: stream-K segment, combine atomically (the residual add
+// straight into x; non-additive epilogues into the fp32 workspace ws, finished by
+// gemm_finish_kernel).  `cl`: cluster split-K, the tile's sums come from the cluster's SMEM.
 template <int EPI>
 __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase, int row, int n_blk, bool partial,
-                                              uint64_t* tfull_bar, uint32_t parity, float* stg, int tile,
-                                              int contrib, int* fix_flag, ClSrc cl = ClSrc{0u, 1, 0}) {
+                                              uint64_t* tfull_bar, uint32_t parity, float* stg,
+                                              ClSrc cl = ClSrc{0u, 1, 0}) {
   const bool row_ok = row < p.M;
   const bool from_cl = cl.part != 0u;  // cluster split-K: sums of the cluster's partial tiles (DSMEM)
   // column chunks (32 wide) this CTA finishes: all, or (cluster split-K) its share of the tile's
@@ -296,8 +293,7 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       for (int c = 0; c < p.head_dim; c += 32) asm volatile("prefetch.global.L2 [%0];" ::"l"(cs + c));
     }
   }
-  bool from_ws = false;  // this CTA finishes a stream-K tile from the workspace sums
-  if (!from_cl && p.ws != nullptr && (partial || p.tile_ctr == nullptr)) {  // (legacy mode: every segment via ws)
+  if (!from_cl && p.ws != nullptr && partial) {  // stream-K segment of a non-additive epilogue
     wait_acc();
 #pragma unroll 1
     for (int c = 0; c < GEMM_BN / 32; ++c) {
@@ -306,22 +302,11 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       const int col0 = n_blk * GEMM_BN + c * 32;
       if (row_ok && col0 < p.N) atomic_add_f32x32(p.ws + (size_t)row * p.N + col0, r);
     }
-    if (p.tile_ctr == nullptr) return;  // gemm_finish_kernel applies the epilogue
-    __threadfence();                     // this thread's reductions before the tile count
-    epi_bar();
-    if (threadIdx.x == 128) *fix_flag = atomicAdd(p.tile_ctr + tile, 1) == contrib - 1;
-    epi_bar();
-    const bool last = *fix_flag != 0;
-    epi_bar();                           // every warp has read the flag before it is reused
-    if (!last) return;
-    __threadfence();
-    if (threadIdx.x == 128) p.tile_ctr[tile] = 0;
-    from_ws = true;
+    return;  // gemm_finish_kernel applies the epilogue
   }
-  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && (!partial || from_ws) && cl.r == 0) p.zero_rows[row] = 0.f;
-  float* wrow = p.ws + (size_t)(row_ok ? row : 0) * p.N + n_blk * GEMM_BN;
-  // accumulator columns [col, col + 32) of this tile's row: from TMEM or (finisher) from ws,
-  // re-zeroing ws behind the read
+  if (p.zero_rows != nullptr && n_blk == 0 && row_ok && !partial && cl.r == 0) p.zero_rows[row] = 0.f;
+  // accumulator columns [col, col + 32) of this tile's row: from TMEM or (cluster split-K) summed
+  // over the cluster's partial tiles
   auto ld = [&](int col, uint32_t(&v)[32]) {
     if (from_cl) {  // fixed rank order: deterministic sums
       float f[32];
@@ -342,31 +327,13 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
       for (int q = 0; q < 32; ++q) v[q] = __float_as_uint(f[q]);
       return;
     }
-    if (!from_ws) {
-      ptx::tmem_ld_32x32b_x32(tbase + col, v);
-      return;
-    }
-    if (row_ok && n_blk * GEMM_BN + col < p.N) {
-      float4* src = reinterpret_cast<float4*>(wrow + col);
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const float4 x = __ldcg(src + q);
-        v[4 * q] = __float_as_uint(x.x);
-        v[4 * q + 1] = __float_as_uint(x.y);
-        v[4 * q + 2] = __float_as_uint(x.z);
-        v[4 * q + 3] = __float_as_uint(x.w);
-        __stcg(src + q, make_float4(0.f, 0.f, 0.f, 0.f));
-      }
-    } else {
-#pragma unroll
-      for (int q = 0; q < 32; ++q) v[q] = 0u;
-    }
+    ptx::tmem_ld_32x32b_x32(tbase + col, v);
   };
   auto ld_wait = [&]() {
-    if (!from_ws && !from_cl) ptx::tmem_ld_wait();
+    if (!from_cl) ptx::tmem_ld_wait();
   };
   auto wait_src = [&]() {
-    if (!from_ws && !from_cl) wait_acc();
+    if (!from_cl) wait_acc();
   };
   if constexpr (EPI == EPI_STORE_BF16) {
     wait_src();
@@ -572,7 +539,6 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(tempty + 2);
-  int* fix_flag = reinterpret_cast<int*>(tmem_ptr + 1);
   float* stg = reinterpret_cast<float*>(sB + C::STAGES * C::B_BYTES + 256);  // epilogue transpose tiles
 
   const int warp = threadIdx.x >> 5;
@@ -738,18 +704,11 @@ __global__ void __launch_bounds__(256, 1)
     const int ew = warp - 4;
     int acc = 0;
     uint32_t acc_phase = 0;
-    const int nk = p.K / GEMM_BK;
     while (jobs.next(tile, kb0, kb1)) {
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
-      int contrib = 1;
-      if (jobs.mode != 0 && tile >= jobs.dp_tiles) {  // stream-K segments covering this tile
-        const int u0 = (tile - jobs.dp_tiles) * nk;
-        contrib = (u0 + nk - 1) / jobs.per - u0 / jobs.per + 1;
-      }
-      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS,
-                         tile * CG + (int)rank, contrib, fix_flag);
+      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != jobs.nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) {
@@ -775,8 +734,7 @@ __global__ void __launch_bounds__(256, 1)
         const int m_blk = tile % num_m, n_blk = tile / num_m;
         const int row = m_blk * C::TILE_M + ew * 32 + lane;
         epilogue_tile<EPI>(p, tmem_base + ((uint32_t)(ew * 32) << 16), row, n_blk, false, &tfull[0], 0,
-                           stg + ew * C::STG_FLOATS, tile, 1, fix_flag,
-                           ClSrc{ptx::smem_u32(sA), p.split_s, (int)cluster_rank()});
+                           stg + ew * C::STG_FLOATS, ClSrc{ptx::smem_u32(sA), p.split_s, (int)cluster_rank()});
       }
     }
     ptx::tc_fence_before();
@@ -871,13 +829,8 @@ PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 std::once_flag g_encode_once;
 
 // Scheduling decision (host).  Returns 1 for stream-K (CG=1 only).
-const bool g_no_sk = [] {  // GLLM_GEMM_NO_SK=1: never stream-K (A/B)
-  const char* e = std::getenv("GLLM_GEMM_NO_SK");
-  return e && e[0] == '1';
-}();
-
 int choose_streamk(int M, int N, int ntiles, int nk, int epi, int num_sms) {
-  if (g_no_sk || epi == EPI_ARGMAX || nk < 8) return 0;
+  if (epi == EPI_ARGMAX || nk < 8) return 0;
   const int waves = (ntiles + num_sms - 1) / num_sms;
   const double eff = (double)ntiles / ((double)waves * num_sms);
   // Measured on B200: with >= one wave of tiles the reductions of partial tiles cost more than
@@ -888,16 +841,10 @@ int choose_streamk(int M, int N, int ntiles, int nk, int epi, int num_sms) {
   return (eff < 0.5 && (size_t)M * N <= GEMM_WS_ELEMS) ? 1 : 0;
 }
 
-// CTA-pair tiles need at least one wave of 256 x 256 tiles.  Measured on B200 (tools/ab_bench.sh,
-// profiles/r01/ab_gemm_cg.txt): with the coalesced residual epilogue the pair kernel wins for
-// every epilogue at the C1 shapes (T ~ 2090: O 0.62 -> 0.67, down 0.83 -> 0.93, gate_up 0.96 ->
-// 1.0 of sustained cuBLAS bf16; QKV was already on it).  GLLM_GEMM_CG1=1 restores the 1-CTA
-// kernel for the residual-add / SiLU epilogues (A/B).
-const bool g_cg1_rest = [] {
-  const char* e = std::getenv("GLLM_GEMM_CG1");
-  return e && e[0] == '1';
-}();
-
+// CTA-pair tiles need at least one wave of 256 x 256 tiles.  Measured on B200 (profiles/r01/
+// ab_gemm_cg.txt): with the coalesced residual epilogue the pair kernel wins for every epilogue at
+// the C1 shapes (T ~ 2090: O 0.62 -> 0.67, down 0.83 -> 0.93, gate_up 0.96 -> 1.0 of sustained
+// cuBLAS bf16; QKV was already on it).
 int choose_cg(int M, int N, int epi, int num_sms) {
   if (g_force_cg) return g_force_cg;
   const int nn = (N + GEMM_BN - 1) / GEMM_BN;
@@ -913,32 +860,18 @@ int choose_cg(int M, int N, int epi, int num_sms) {
     if (e1 > e2 + 0.15) return 1;
   }
   if (epi == EPI_STORE_BF16 || epi == EPI_QKV_ROPE) return 2;
-  return g_cg1_rest && M < 4096 ? 1 : 2;
+  return 2;
 }
 
 // CTA-pair hybrid (Jobs mode 2) for the residual-add epilogue: when the last wave of 256 x 256
-// tiles would be less than ~60% full (e.g. C3's O / down GEMMs at T ~ 900: 80 tiles on 74
-// pairs), the tail tiles' k-blocks are spread over every pair and combined with fp32 vector
-// reductions.  Returns the whole-tile count (0 = no hybrid).  GLLM_GEMM_NO_HYBRID=1 disables it.
-const bool g_no_hybrid = [] {
-  const char* e = std::getenv("GLLM_GEMM_NO_HYBRID");
-  return e && e[0] == '1';
-}();
-// Non-additive epilogues (QKV / SiLU / store) take the hybrid too when their fp32 workspace fits
-// (`ws_ok`): partial tiles then combine in ws and the last segment finishes the tile in-kernel.
-// Measured on B200 (profiles/r01/gemm_sched.txt): the in-kernel finish of workspace tiles costs
-// more than a memset + finish pass at C4's QKV (82 vs ~60 us), so it is opt-in
-// (GLLM_GEMM_SK_FIXUP=1) and only the residual-add epilogue takes the hybrid by default.
-const bool g_sk_fixup = [] {
-  const char* e = std::getenv("GLLM_GEMM_SK_FIXUP");
-  return e && e[0] == '1';
-}();
-int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms, bool ws_ok) {
-  if (g_no_hybrid || cg != 2 || epi == EPI_ARGMAX || K / GEMM_BK < 8) return 0;
-  if (epi != EPI_ADD_F32 && !g_sk_fixup) return 0;
+// tiles would be less than ~80% full (e.g. C3's O / down GEMMs at T ~ 900: 80 tiles on 74 pairs),
+// the tail tiles' k-blocks are spread over every pair and combined with fp32 vector reductions.
+// Returns the whole-tile count (0 = no hybrid).  (Non-additive epilogues through the fp32 workspace
+// measured slower than whole tiles, profiles/r01/gemm_sched.txt.)
+int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms) {
+  if (cg != 2 || epi != EPI_ADD_F32 || K / GEMM_BK < 8) return 0;
   const int units = num_sms / 2;
   const int ntiles = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
-  if (epi != EPI_ADD_F32 && (!ws_ok || (size_t)M * N > GEMM_WS_ELEMS || ntiles * 2 > GEMM_MAX_SK_TILES)) return 0;
   const int tail = ntiles % units;
   if (ntiles < units || tail == 0 || tail * 10 >= units * 8) return 0;
   return ntiles - tail;
@@ -960,18 +893,18 @@ int skc_split(int M, int N, int K, int epi, int num_sms) {
 
 }  // namespace
 
-bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms) {
-  if (M <= 0) return false;
+bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms, bool deterministic) {
+  if (M <= 0 || deterministic) return false;
   if (!g_force_cg && skc_split(M, N, K, epi, num_sms)) return false;  // whole tiles, reduced in-cluster
   const int cg = choose_cg(M, N, epi, num_sms);
-  if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms, false) > 0;
+  if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms) > 0;
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
   return choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms) != 0;
 }
 
 size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms) {
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
-  if (epi == EPI_ADD_F32 || choose_cg(M, N, epi, num_sms) == 2 ||
+  if (epi == EPI_ADD_F32 || choose_cg(M, N, epi, num_sms) == 2 || (!g_force_cg && skc_split(M, N, K, epi, num_sms)) ||
       !choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms))
     return 0;
   return (size_t)M * N;
@@ -1037,7 +970,7 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
     cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, cluster, a, b, args);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (%d-CTA) launch: %s", CG, cudaGetErrorString(e));
   }
-  if (args.ws && !args.tile_ctr) {
+  if (args.ws) {
     const int chunks = args.M * ((EPI == EPI_SILU_MUL) ? args.N / 64 : args.N / 32);
     launch_pdl(gemm_finish_kernel<EPI>, dim3((chunks + 255) / 256), dim3(256), 0, stream, 1, args);
   }
@@ -1062,7 +995,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   args.num_m_tiles = (args.M + GEMM_BM - 1) / GEMM_BM;
   args.num_n_tiles = (args.N + GEMM_BN - 1) / GEMM_BN;
   const int ntiles = args.num_m_tiles * args.num_n_tiles, nk = args.K / GEMM_BK;
-  args.streamk = cg == 1 ? choose_streamk(args.M, args.N, ntiles, nk, epi, num_sms) : 0;
+  args.streamk = (cg == 1 && !args.deterministic) ? choose_streamk(args.M, args.N, ntiles, nk, epi, num_sms) : 0;
   args.units_per_cta = args.streamk ? (ntiles * nk + num_sms - 1) / num_sms : 0;
   args.dp_tiles = 0;
   args.split_s = 0;
@@ -1075,8 +1008,8 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
     }
   }
   bool hybrid = false;
-  if (cg == 2 && !args.xb_out && !args.ss_out && !args.out_peer) {  // partial tiles: no fused outputs
-    const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms, args0.ws && args0.tile_ctr);
+  if (cg == 2 && !args.deterministic && !args.xb_out && !args.ss_out && !args.out_peer) {  // partial tiles: no fused outputs
+    const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms);
     if (dp > 0) {
       const int ntiles2 = ((args.M + 255) / 256) * args.num_n_tiles, units = num_sms / 2;
       args.streamk = 2;
@@ -1085,19 +1018,11 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
       hybrid = true;
     }
   }
-  if (!g_sk_fixup) args.tile_ctr = nullptr;  // memset + finish pass (see hybrid_dp_tiles)
   if (args.streamk && args.streamk != 3 && epi != EPI_ADD_F32) {
     if (!args0.ws) return set_error(GLLM_EINVAL, "gemm: stream-K workspace required");
-    if (!hybrid && args.tile_ctr && ntiles > GEMM_MAX_SK_TILES) args.tile_ctr = nullptr;  // legacy memset + finish
   } else {
     args.ws = nullptr;
-    args.tile_ctr = nullptr;
   }
-  static const bool dbg = std::getenv("GLLM_GEMM_DEBUG") != nullptr;
-  if (dbg)
-    std::fprintf(stderr, "[gemm] M=%d N=%d K=%d epi=%d cg=%d streamk=%d dp_tiles=%d per=%d ws=%d ctr=%d\n", args.M,
-                 args.N, args.K, (int)epi, cg, args.streamk, args.dp_tiles, args.units_per_cta, args.ws != nullptr,
-                 args.tile_ctr != nullptr);
   switch (epi) {
     case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, args, stream, num_sms, cg);
     case EPI_ADD_F32: return launch_e<EPI_ADD_F32>(a, b, args, stream, num_sms, cg);

@@ -43,11 +43,10 @@ struct GemmArgs {
   // B (the weights) is never written by a kernel on the stream: with PDL the producer issues the
   // first ring fill's B tiles before griddepcontrol.wait (stage GEMMs only; gllm_op_gemm leaves 0)
   int b_static;
-  float* ws;
-  // stream-K fixup counters (>= tiles ints).  Non-null: ws and tile_ctr are all zero on entry and
-  // the kernel leaves them zero (the last segment of each tile finishes it in-kernel); null: ws
-  // is zero on entry too, and gemm_finish_kernel applies the epilogue and clears what it read.
-  int* tile_ctr;
+  float* ws;  // fp32 [M, N] stream-K workspace of non-additive epilogues: zero on entry, left zero
+  // 1: a schedule with a fixed reduction order (no stream-K / hybrid fp32 atomics; whole tiles or
+  // cluster split-K): bitwise run-to-run reproducible results
+  int deterministic;
   // fused RMSNorm (a4).  Consumers (EPI_STORE_BF16 / EPI_QKV_ROPE / EPI_SILU_MUL) read the bf16
   // copy of the residual as A and scale each output row by r = rsqrt(row_ss[row] * inv_h + eps)
   // (the norm gain is folded into W; it is exactly 1 for the O4 weights).  The producer
@@ -64,14 +63,13 @@ struct GemmArgs {
 
 // true if launch_gemm would combine partial tiles (stream-K) for this shape -- then the ADD_F32
 // epilogue cannot produce xb_out / ss_out and the caller runs rms_stats instead
-bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms);
+bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms, bool deterministic = false);
 
 // fp32 workspace (elements) launch_gemm may need for a GEMM of this shape/epilogue (0 = none)
 size_t gemm_workspace_elems(int M, int N, int K, int epi, int num_sms);
 
 constexpr int GEMM_BM = 128, GEMM_BN = 256, GEMM_BK = 64, GEMM_STAGES = 4;
 constexpr size_t GEMM_WS_ELEMS = size_t(8) << 20;  // stream-K fp32 workspace capacity (32 MB)
-constexpr int GEMM_MAX_SK_TILES = 4096;             // stream-K fixup counters per workspace
 // TMA box rows of the B (weight) tensor maps: one 128-row half of a 256-wide N tile, so the same
 // map serves the 1-CTA kernel (two loads per stage) and the CTA-pair kernel (one per CTA).
 constexpr int GEMM_B_BOX = 128;

@@ -35,19 +35,17 @@ extern "C" int gllm_op_gemm(const void* A, const void* W, int32_t M, int32_t N, 
   void* tmp = nullptr;
   const size_t ws_elems = gllm::gemm_workspace_elems(M, N, K, epi, sms);
   const size_t part_elems = epi == gllm::EPI_ARGMAX ? (size_t)M * ntn : 0;
-  if (ws_elems) {  // stream-K fixup: a process-wide workspace + tile counters, zero between calls
+  if (ws_elems) {  // stream-K: a process-wide fp32 workspace, zero between calls
     static float* ws = nullptr;
     static size_t ws_cap = 0;
     if (ws_cap < ws_elems) {
       if (ws) cudaFree(ws);
       ws_cap = 0;
-      if (cudaMalloc(&ws, (ws_elems + gllm::GEMM_MAX_SK_TILES) * 4) != cudaSuccess ||
-          cudaMemset(ws, 0, (ws_elems + gllm::GEMM_MAX_SK_TILES) * 4) != cudaSuccess)
+      if (cudaMalloc(&ws, ws_elems * 4) != cudaSuccess || cudaMemset(ws, 0, ws_elems * 4) != cudaSuccess)
         return gllm::set_error(GLLM_ENOMEM, "op_gemm: workspace allocation failed");
       ws_cap = ws_elems;
     }
     g.ws = ws;
-    g.tile_ctr = reinterpret_cast<int*>(ws + ws_cap);
   }
   if (part_elems) {
     if (cudaMallocAsync(&tmp, 2 * part_elems * 4, s) != cudaSuccess)

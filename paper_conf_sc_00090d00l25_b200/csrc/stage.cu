@@ -127,7 +127,6 @@ struct gllm_stage {
   int32_t* slots = nullptr;
   int32_t* sampled_tmp = nullptr;
   float* gemm_ws = nullptr;  // stream-K fp32 workspace for non-additive epilogues (small T), kept zero
-  int* sk_ctr = nullptr;     // stream-K fixup tile counters, kept zero
   float *ss_a = nullptr, *ss_b = nullptr;  // fused-RMSNorm row statistics (sum of squares of x)
   int* dec_ctr = nullptr;                  // persistent decode kernel: work counter + done counter
   float* part_val = nullptr;
@@ -143,6 +142,7 @@ struct gllm_stage {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int last_T = 0, last_launches = 0;
   bool profiling = false;
+  bool deterministic = false;  // gllm_stage_set_deterministic: GEMM schedules with a fixed reduction order
   bool prof_serial_attn = false;  // gllm_stage_set_profiling(st, 2): attribution pass, attention in series
   // fused peer hand-off (a12, gllm_peer_*): receive ring owned here / the next stage's ring mapped here
   float* ring = nullptr;
@@ -241,7 +241,7 @@ int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmE
   g.part_val = st->part_val;
   g.part_idx = st->part_idx;
   g.ws = st->gemm_ws;
-  g.tile_ctr = st->sk_ctr;
+  g.deterministic = st->deterministic;
   st->last_launches += 1;
   return gllm::launch_gemm(a, b, epi, g, s, st->num_sms);
 }
@@ -430,11 +430,9 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
       (rc = st->dalloc(&st->slots, R)) ||
       // stream-K workspace for non-additive epilogues (used only for outputs <= GEMM_WS_ELEMS)
       (rc = st->dalloc(&st->gemm_ws, gllm::GEMM_WS_ELEMS)) || (rc = st->dalloc(&st->ss_a, R)) ||
-      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->dec_ctr, 2)) || (rc = st->dalloc(&st->release_ctr, 1)) ||
-      (rc = st->dalloc(&st->sk_ctr, gllm::GEMM_MAX_SK_TILES)))
+      (rc = st->dalloc(&st->ss_b, R)) || (rc = st->dalloc(&st->dec_ctr, 2)) || (rc = st->dalloc(&st->release_ctr, 1)))
     return fail(rc);
   CK(cudaMemsetAsync(st->gemm_ws, 0, gllm::GEMM_WS_ELEMS * sizeof(float), s0));
-  CK(cudaMemsetAsync(st->sk_ctr, 0, gllm::GEMM_MAX_SK_TILES * sizeof(int), s0));
   CK(cudaMemsetAsync(st->dec_ctr, 0, 2 * sizeof(int), s0));
   CK(cudaMemsetAsync(st->release_ctr, 0, sizeof(unsigned), s0));
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
@@ -680,22 +678,27 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
   auto residual_gemm = [&](const CUtensorMap& ta, const CUtensorMap& tb, int K, float* ss_next,
                            float* out_peer) -> int {
     // ss_next was zeroed by the n-tile-0 epilogue of the preceding consumer GEMM (zero_rows)
-    const bool sk = gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms);
+    // partial tiles combine with reductions: no fused bf16(x) / sum of squares (rms_stats rebuilds
+    // them); the deterministic mode also takes the statistics pass (the fused sum of squares adds
+    // each tile's share atomically)
+    const bool sk = gllm::gemm_uses_streamk(T, H, K, gllm::EPI_ADD_F32, st->num_sms, st->deterministic);
+    const bool unfused = sk || st->deterministic;
     gllm::GemmArgs g{};
     g.b_static = 1;
+    g.deterministic = st->deterministic;
     g.M = T;
     g.N = H;
     g.K = K;
     g.out = x;
     g.ldo = H;
-    g.xb_out = sk ? nullptr : st->y;
-    g.ss_out = sk ? nullptr : ss_next;
+    g.xb_out = unfused ? nullptr : st->y;
+    g.ss_out = unfused ? nullptr : ss_next;
     g.out_peer = sk ? nullptr : out_peer;  // whole tiles store the new residual rows to the peer too
     st->last_launches += 1;
     RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms));
     if (out_peer && sk)  // partial tiles reduce in place: copy the finished residual afterwards
       CK(cudaMemcpyAsync(out_peer, x, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
-    if (sk) {  // partial tiles combine with reductions: recompute the statistics from x
+    if (unfused) {  // rebuild bf16(x) and the row sums of squares from x
       gllm::launch_rms_stats(x, nullptr, st->y, ss_next, T, H, nullptr, 0, nullptr, s);
       st->last_launches += 1;
     }
@@ -724,7 +727,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.n_kv_heads = c.n_kv_heads;
       g.block_size = bs;
       g.ws = st->gemm_ws;
-      g.tile_ctr = st->sk_ctr;
+      g.deterministic = st->deterministic;
       g.row_ss = st->ss_a;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
@@ -781,7 +784,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       g.out = st->act;
       g.ldo = I;
       g.ws = st->gemm_ws;
-      g.tile_ctr = st->sk_ctr;
+      g.deterministic = st->deterministic;
       g.row_ss = st->ss_b;
       g.inv_h = inv_h;
       g.eps = c.rms_eps;
@@ -861,6 +864,12 @@ int gllm_stage_sync(gllm_stage* st) {
   cudaSetDevice(st->device);
   cudaError_t e = cudaDeviceSynchronize();
   if (e != cudaSuccess) return gllm::set_error(GLLM_ECUDA, "device: %s", cudaGetErrorString(e));
+  return GLLM_OK;
+}
+
+int gllm_stage_set_deterministic(gllm_stage* st, int32_t on) {
+  if (!st) return gllm::set_error(GLLM_EINVAL, "null stage");
+  st->deterministic = on != 0;
   return GLLM_OK;
 }
 

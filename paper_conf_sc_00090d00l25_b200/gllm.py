@@ -118,6 +118,7 @@ def lib():
             "gllm_stage_fill_warm_kv": ([vp, i32, C.POINTER(C.c_int64), _P32, _P32, i32], C.c_int),
             "gllm_sched_seq_blocks": ([vp, i64, _P32, i32, _P32], C.c_int),
             "gllm_stage_set_profiling": ([vp, i32], C.c_int),
+            "gllm_stage_set_deterministic": ([vp, i32], C.c_int),
             "gllm_stage_last_timing": ([vp, C.POINTER(C.c_float), i32], C.c_int),
             "gllm_stage_last_launches": ([vp, _P32], C.c_int),
             "gllm_op_gemm": ([vp, vp, i32, i32, i32, i32, vp, vp, vp], C.c_int),
@@ -304,6 +305,9 @@ class Stage:
 
     def sync(self):
         _check(lib().gllm_stage_sync(self.h))
+
+    def set_deterministic(self, on=True):
+        _check(lib().gllm_stage_set_deterministic(self.h, int(on)))
 
     def set_profiling(self, on=True):
         _check(lib().gllm_stage_set_profiling(self.h, int(on)))

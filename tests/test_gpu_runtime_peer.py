@@ -63,6 +63,7 @@ def _peer_rank(rank, world, port, q, transport="peer", gpus=1):
     torch.cuda.set_device(dev)
     lb, le = split_layers(m.n_layers, world)[rank]
     stage = gllm.Stage(m, lb, le, sp.num_blocks, max_tokens, sp.max_seqs, device=dev)
+    stage.set_deterministic(True)   # fixed reduction order: the split run must equal the 1-process run exactly
     ex = GpuExecutor(stage, torch.device("cuda", dev), max_tokens, m.hidden, pp=world)
     if transport == "peer":
         tr = PeerTransport(ex, rank, world, dist.group.WORLD)
@@ -94,6 +95,7 @@ def _reference(q):
     from paper_conf_sc_00090d00l25_b200.runtime import GpuExecutor, Pipeline
     torch.cuda.set_device(0)
     stage = gllm.Stage(m, 0, m.n_layers, sp.num_blocks, max_tokens, sp.max_seqs, device=0)
+    stage.set_deterministic(True)
     ex = GpuExecutor(stage, torch.device("cuda", 0), max_tokens, m.hidden, pp=2)
     sched = gllm.Sched(sp)
     sched.add_stream(st)
@@ -137,4 +139,5 @@ def test_pipeline_runtime_handoff_matches_one_process(transport, gpus):
         a, b = np.asarray(got[k]), np.asarray(want[k])
         n += len(a)
         agree += int((a == b).sum())
-    assert n > 100 and agree / n >= 0.98, (agree, n)
+    # deterministic mode on both sides: the pipelined run reproduces the one-process ids exactly
+    assert n > 100 and agree == n, (agree, n)

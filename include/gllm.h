@@ -173,7 +173,10 @@ typedef struct gllm_stage gllm_stage;
  * tokens for every local layer) and workspaces for up to max_tokens tokens and
  * max_seqs sequences per micro-batch.  EINVAL for inconsistent shapes
  * (head_dim != 128 and != 64, hidden % 64, intermediate % 128, ...), ENOMEM
- * when HBM does not fit. */
+ * when HBM does not fit.
+ * Restriction: every RMSNorm gain is 1 (the O4 weights).  The library has no
+ * gain input: the fused norm scales GEMM rows by 1/rms(x) and would need a gain folded into the
+ * columns of W_qkv / W_gate_up (W' = W diag(g)), which O4's g = 1 makes the identity. */
 GLLM_API int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t layer_end,
                     int32_t kv_blocks, int32_t block_size, int32_t max_tokens,
                     int32_t max_seqs, int32_t device, gllm_stage** out);

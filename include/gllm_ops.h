@@ -28,6 +28,10 @@ GLLM_API int gllm_op_gemm(const void* A, const void* W, int32_t M, int32_t N, in
  * 0 = automatic, 1 = force the 1-CTA 128x256 kernel, 2 = force the CTA-pair 256x256 kernel. */
 GLLM_API int gllm_op_set_gemm_variant(int32_t cta_group);
 
+/* gllm_op_gemm calls afterwards (process-wide): 1 = schedules with a fixed reduction order (no
+ * stream-K / hybrid atomics; as gllm_stage_set_deterministic), 0 = automatic (default). */
+GLLM_API int gllm_op_set_deterministic(int32_t on);
+
 #ifdef __cplusplus
 }
 #endif

@@ -37,7 +37,8 @@ namespace {
 constexpr float LOG2E_W = 1.4426950408889634f;
 constexpr int WS_ROWS = 128;  // rows per Q tile (= TMEM lanes)
 constexpr int WS_KT = 128;    // keys per tile
-constexpr int WS_NS = 2;      // K/V ring stages
+constexpr int WS_NSK = 3;     // K ring stages (the S MMAs' operand: the critical path)
+constexpr int WS_NSV = 2;     // V ring stages (V is needed only after the tile's softmax)
 constexpr int WS_THREADS = 384;
 constexpr float WS_RESCALE_LOG2 = 8.0f;
 
@@ -50,10 +51,10 @@ struct WsSmem {
   static constexpr int KV_TILE = ATOMS * KV_ATOM;
   static constexpr int Q = 0;
   static constexpr int K = Q + 2 * Q_TILE;
-  static constexpr int V = K + WS_NS * KV_TILE;
-  static constexpr int BAR = V + WS_NS * KV_TILE;
-  // barriers: q_full, kfull[NS], vfull[NS], kempty[NS], vempty[NS], sfull[2], pfull[2], ofull[2]; tmem slot
-  static constexpr int NBAR = 1 + 4 * WS_NS + 6;
+  static constexpr int V = K + WS_NSK * KV_TILE;
+  static constexpr int BAR = V + WS_NSV * KV_TILE;
+  // barriers: q_full, kfull[NSK], kempty[NSK], vfull[NSV], vempty[NSV], sfull[2], pfull[2], ofull[2]; tmem slot
+  static constexpr int NBAR = 1 + 2 * WS_NSK + 2 * WS_NSV + 6;
   static constexpr int BYTES = BAR + NBAR * 8 + 16 + 1024;  // + 1024-B alignment slack
 };
 
@@ -170,10 +171,10 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L::BAR);
   uint64_t* q_full = bars;
   uint64_t* kfull = bars + 1;
-  uint64_t* vfull = kfull + WS_NS;
-  uint64_t* kempty = vfull + WS_NS;   // K slot free: the last S MMA reading it completed
-  uint64_t* vempty = kempty + WS_NS;  // V slot free: the last PV MMA reading it completed
-  uint64_t* sfull = vempty + WS_NS;
+  uint64_t* kempty = kfull + WS_NSK;  // K slot free: the last S MMA reading it completed
+  uint64_t* vfull = kempty + WS_NSK;
+  uint64_t* vempty = vfull + WS_NSV;  // V slot free: the last PV MMA reading it completed
+  uint64_t* sfull = vempty + WS_NSV;
   uint64_t* pfull = sfull + 2;
   uint64_t* ofull = pfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + L::NBAR);
@@ -198,10 +199,12 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 
   if (tid == 0) {
     ptx::mbar_init(q_full, 2 * WS_ROWS);
-    for (int s = 0; s < WS_NS; ++s) {
+    for (int s = 0; s < WS_NSK; ++s) {
       ptx::mbar_init(&kfull[s], 1);
-      ptx::mbar_init(&vfull[s], 1);
       ptx::mbar_init(&kempty[s], 1);
+    }
+    for (int s = 0; s < WS_NSV; ++s) {
+      ptx::mbar_init(&vfull[s], 1);
       ptx::mbar_init(&vempty[s], 1);
     }
     for (int x = 0; x < 2; ++x) {
@@ -222,45 +225,38 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == 0) {
-    // ---------------- TMA producer.  Loads in the order their slots free up: K(j) as soon as
-    // S_B(j-NS) (its slot's last reader) completes, V(j-1) once PV_B(j-1-NS) completes; so the
-    // next K tile streams in while the current tile's PV and softmax run.
-    int bnext = 0;
-    auto read_bt = [&](int j) {  // lanes 0..7: block ids of tile j's pages (past the sequence: its page 0)
+  if (warp == 0 || warp == 2) {
+    // ---------------- TMA producers: warp 0 streams the K tiles, warp 2 the V tiles, each as soon as
+    // its slot frees (K: the S MMAs of both Q tiles reading it completed; V: the PV MMAs), so the
+    // deeper K ring runs ahead of the V waits.  Lanes 0..7 read the 8 block ids of the next tile.
+    const bool is_k = warp == 0;
+    const CUtensorMap* map = is_k ? &tmk : &tmv;
+    const int ns = is_k ? WS_NSK : WS_NSV;
+    uint64_t* full = is_k ? kfull : vfull;
+    uint64_t* empty = is_k ? kempty : vempty;
+    const uint32_t base = is_k ? L::K : L::V;
+    auto read_bt = [&](int j) {  // block ids of tile j's pages (past the sequence: its page 0)
       const int kb = j * PAGES + lane;
       return (lane < PAGES && j < n_kt) ? __ldg(bt + (kb < nblk_seq ? kb : 0)) : 0;
     };
-    auto load = [&](const CUtensorMap* map, uint64_t* full, uint32_t dst, const int (&bp)[PAGES]) {
-      ptx::mbar_arrive_expect_tx(full, L::KV_TILE);
-#pragma unroll
-      for (int p = 0; p < PAGES; ++p)
-#pragma unroll
-        for (int at = 0; at < ATOMS; ++at)
-          ptx::tma_load_2d(smem + dst + at * L::KV_ATOM + p * 2048, map, full, at * 64, (bp[p] * a.Hkv + kvh) * 16);
-    };
-    bnext = read_bt(0);
-    int bprev[PAGES];
+    int bnext = read_bt(0);
 #pragma unroll 1
-    for (int j = 0; j <= n_kt; ++j) {
+    for (int j = 0; j < n_kt; ++j) {
       int bp[PAGES];
 #pragma unroll
       for (int p = 0; p < PAGES; ++p) bp[p] = __shfl_sync(0xffffffffu, bnext, p);
       bnext = read_bt(j + 1);
       if (lane == 0) {
-        if (j >= 1) {  // V(j-1)
-          const int jv = j - 1, sv = jv % WS_NS;
-          if (jv >= WS_NS) ptx::mbar_wait(&vempty[sv], (uint32_t)(((jv / WS_NS) - 1) & 1));
-          load(&tmv, &vfull[sv], L::V + sv * L::KV_TILE, bprev);
-        }
-        if (j < n_kt) {  // K(j)
-          const int sk = j % WS_NS;
-          if (j >= WS_NS) ptx::mbar_wait(&kempty[sk], (uint32_t)(((j / WS_NS) - 1) & 1));
-          load(&tmk, &kfull[sk], L::K + sk * L::KV_TILE, bp);
-        }
-      }
+        const int sl = j % ns;
+        if (j >= ns) ptx::mbar_wait(&empty[sl], (uint32_t)(((j / ns) - 1) & 1));
+        ptx::mbar_arrive_expect_tx(&full[sl], L::KV_TILE);
+        const uint32_t dst = base + sl * L::KV_TILE;
 #pragma unroll
-      for (int p = 0; p < PAGES; ++p) bprev[p] = bp[p];
+        for (int p = 0; p < PAGES; ++p)
+#pragma unroll
+          for (int at = 0; at < ATOMS; ++at)
+            ptx::tma_load_2d(smem + dst + at * L::KV_ATOM + p * 2048, map, &full[sl], at * 64, (bp[p] * a.Hkv + kvh) * 16);
+      }
       __syncwarp();
     }
   } else if (warp == 1) {
@@ -270,7 +266,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       constexpr uint32_t idesc_o = idesc_bf16(WS_ROWS, D, true);
       auto issue_s = [&](int x, int j) {
         const uint32_t qb = sbase + L::Q + x * L::Q_TILE;
-        const uint32_t kb = sbase + L::K + (j % WS_NS) * L::KV_TILE;
+        const uint32_t kb = sbase + L::K + (j % WS_NSK) * L::KV_TILE;
 #pragma unroll
         for (int ks = 0; ks < D / 16; ++ks)
           ptx::umma_bf16(tmem + x * 128, ptx::umma_desc_sw128(qb + (ks / 4) * L::Q_ATOM + (ks % 4) * 32),
@@ -278,14 +274,14 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
         ptx::umma_commit(&sfull[x]);
       };
       auto issue_pv = [&](int x, int j) {
-        const uint32_t vb = sbase + L::V + (j % WS_NS) * L::KV_TILE;
+        const uint32_t vb = sbase + L::V + (j % WS_NSV) * L::KV_TILE;
 #pragma unroll
         for (int kk = 0; kk < WS_KT / 16; ++kk)  // 16 keys = 8 TMEM columns of packed P per step
           umma_bf16_ta(tmem + 256 + x * 128, tmem + x * 128 + kk * 8, desc_mn(vb + kk * 2048, L::KV_ATOM), idesc_o,
                        (j > 0 || kk > 0) ? 1u : 0u);
       };
       auto wait_k = [&](int j) {
-        ptx::mbar_wait(&kfull[j % WS_NS], (uint32_t)((j / WS_NS) & 1));
+        ptx::mbar_wait(&kfull[j % WS_NSK], (uint32_t)((j / WS_NSK) & 1));
         ptx::tc_fence_after();
       };
       ptx::mbar_wait(q_full, 0);
@@ -296,8 +292,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::umma_commit(&kempty[0]);  // K(0) is read by S_A(0), S_B(0) only
 #pragma unroll 1
       for (int j = 0; j < n_kt; ++j) {
-        const int s = j % WS_NS;
-        ptx::mbar_wait(&vfull[s], (uint32_t)((j / WS_NS) & 1));
+        const int s = j % WS_NSV;
+        ptx::mbar_wait(&vfull[s], (uint32_t)((j / WS_NSV) & 1));
         bool k_next = false;
         if (j < nA) {
           ptx::mbar_wait(&pfull[0], (uint32_t)(j & 1));
@@ -325,7 +321,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
             ptx::umma_commit(&ofull[1]);
           }
         }
-        if (j + 1 < n_kt) ptx::umma_commit(&kempty[(j + 1) % WS_NS]);  // every S of tile j+1 issued
+        if (j + 1 < n_kt) ptx::umma_commit(&kempty[(j + 1) % WS_NSK]);  // every S of tile j+1 issued
       }
     }
   } else if (warp >= 4) {

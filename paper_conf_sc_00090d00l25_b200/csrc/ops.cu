@@ -12,6 +12,13 @@ extern "C" int gllm_op_set_gemm_variant(int32_t cta_group) {
   return GLLM_OK;
 }
 
+static bool g_op_deterministic = false;
+
+extern "C" int gllm_op_set_deterministic(int32_t on) {
+  g_op_deterministic = on != 0;
+  return GLLM_OK;
+}
+
 extern "C" int gllm_op_gemm(const void* A, const void* W, int32_t M, int32_t N, int32_t K, int32_t epi,
                             const float* bias, void* out, void* stream) {
   if (!A || !W || !out || M < 0 || N <= 0 || K <= 0) return gllm::set_error(GLLM_EINVAL, "op_gemm: bad arguments");
@@ -31,9 +38,10 @@ extern "C" int gllm_op_gemm(const void* A, const void* W, int32_t M, int32_t N, 
   g.out = out;
   g.ldo = epi == gllm::EPI_SILU_MUL ? N / 2 : N;
   g.bias = epi == gllm::EPI_STORE_BF16 ? bias : nullptr;
+  g.deterministic = g_op_deterministic;
   const int ntn = (N + gllm::GEMM_BN - 1) / gllm::GEMM_BN;
   void* tmp = nullptr;
-  const size_t ws_elems = gllm::gemm_workspace_elems(M, N, K, epi, sms);
+  const size_t ws_elems = g_op_deterministic ? 0 : gllm::gemm_workspace_elems(M, N, K, epi, sms);
   const size_t part_elems = epi == gllm::EPI_ARGMAX ? (size_t)M * ntn : 0;
   if (ws_elems) {  // stream-K: a process-wide fp32 workspace, zero between calls
     static float* ws = nullptr;

@@ -123,6 +123,7 @@ def lib():
             "gllm_stage_last_launches": ([vp, _P32], C.c_int),
             "gllm_op_gemm": ([vp, vp, i32, i32, i32, i32, vp, vp, vp], C.c_int),
             "gllm_op_set_gemm_variant": ([i32], C.c_int),
+            "gllm_op_set_deterministic": ([i32], C.c_int),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -398,6 +399,10 @@ class Stage:
 def op_gemm(A_ptr, W_ptr, M, N, K, epi, out_ptr, bias_ptr=0, stream=0):
     """gllm_op_gemm (include/gllm_ops.h): the stage's tcgen05 GEMM on raw device pointers."""
     _check(lib().gllm_op_gemm(A_ptr, W_ptr, M, N, K, epi, bias_ptr or None, out_ptr, stream or None))
+
+
+def op_set_deterministic(on: bool):
+    _check(lib().gllm_op_set_deterministic(int(on)))
 
 
 def op_set_gemm_variant(cta_group: int):

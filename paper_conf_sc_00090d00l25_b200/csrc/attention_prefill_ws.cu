@@ -181,8 +181,10 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 
   pdl_trigger();
   pdl_wait();
-  const PrefillItem it = items[blockIdx.x];
-  const int kvh = blockIdx.y;
+  // grid (Hkv, items): CTAs are dispatched x-fastest, so every kv head of the longest item goes
+  // first and the whole grid runs longest-first (the host sorts items by key tiles)
+  const PrefillItem it = items[blockIdx.y];
+  const int kvh = blockIdx.x;
   const int G = a.Hq / a.Hkv;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int t0 = a.cu_q[it.seq];
@@ -502,7 +504,7 @@ int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
     cudaFuncSetAttribute(prefill_attn_ws_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  launch_pdl(prefill_attn_ws_kernel<D, MODE>, dim3(n_items, a.Hkv), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
+  launch_pdl(prefill_attn_ws_kernel<D, MODE>, dim3(a.Hkv, n_items), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
   return GLLM_OK;
 }
 

@@ -101,19 +101,6 @@ __device__ __forceinline__ float ex2(float x) {  // ex2.approx: 2^-inf = +0
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
-// 2^x on the FMA pipe (x <= ~8): round-to-nearest split x = j + f, f in [-1/2, 1/2], cubic for
-// 2^f (relative error < 1e-3, below bf16's 2^-8 rounding of P), j added to the exponent bits.
-// Takes a share of the exponentials off the 16/clk/SM MUFU unit (FA4's trick).
-__device__ __forceinline__ float exp2_fma(float x) {
-  x = fmaxf(x, -126.f);
-  const float t = x + 12582912.f;  // 1.5 * 2^23: the integer part lands in the low mantissa bits
-  const float f = x - (t - 12582912.f);
-  float p = fmaf(f, 0.0555041087f, 0.240226507f);
-  p = fmaf(p, f, 0.693147181f);
-  p = fmaf(p, f, 1.0f);
-  return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));
-}
-
 // packed fp32 pairs (sm_100 FFMA2 / FADD2)
 __device__ __forceinline__ uint64_t f2pack(float a, float b) {
   uint64_t r;
@@ -154,10 +141,7 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
-// MODE 0: the kernel.  1: EMU (a quarter of the exponentials on the FMA pipe; A/B).  Timing
-// probes (GLLM_PREFILL_PROBE, wrong results, measurement only): 2 = no exp2 (P = the scaled
-// score), 3 = no softmax at all (P = whatever S left; only the load / MMA pipeline runs).
-template <int D, int MODE>
+template <int D>
 __global__ void __launch_bounds__(WS_THREADS, 1)
     prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items,
                            const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
@@ -226,7 +210,11 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  // register budget by role (per warpgroup, inside each role's branch so the allocator sees each
+  // region's budget): producers / MMA issuer / idle warp 56, the softmax warpgroups 224 (they hold a
+  // full 128-score row: one TMEM pass per key tile)
 
+  if (warp < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;" ::: "memory");
   if (warp == 0 || warp == 2) {
     // ---------------- TMA producers: warp 0 streams the K tiles, warp 2 the V tiles, each as soon as
     // its slot frees (K: the S MMAs of both Q tiles reading it completed; V: the PV MMAs), so the
@@ -328,6 +316,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     }
   } else if (warp >= 4) {
     // ---------------- softmax warpgroups (tile X = 0: warps 4-7, X = 1: warps 8-11)
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 224;" ::: "memory");
     const int x = (warp - 4) >> 2;
     const int r = (warp & 3) * 32 + lane;  // row of the Q tile = TMEM lane
     const int rr = it.row0 + x * WS_ROWS + r;
@@ -355,40 +344,29 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     for (int j = 0; j < nx; ++j) {
       ptx::mbar_wait(&sfull[x], (uint32_t)(j & 1));
       ptx::tc_fence_after();
-      if (MODE == 3) {
-        ptx::tc_fence_before();
-        ptx::mbar_arrive(&pfull[x]);
-        l = 1.f;
-        continue;
-      }
       const int kbase = j * WS_KT;
       // causal masking only where some row of this warp ends inside the tile (warp-uniform, so
       // the unmasked path carries no per-element compares)
       const bool diag_w = __any_sync(0xffffffffu, kbase + WS_KT - 1 > pos);
-      // pass 1: row max of the raw scores; the next 32-column load is in flight while the
-      // current chunk is reduced (tcgen05.wait::ld covers every earlier load of the thread)
+      // one TMEM pass: the whole 128-score row into registers (four loads in flight, one wait)
+      uint32_t sr[WS_KT / 32][32];
+#pragma unroll
+      for (int cq = 0; cq < WS_KT / 32; ++cq) ptx::tmem_ld_32x32b_x32(t_s + cq * 32, sr[cq]);
+      ptx::tmem_ld_wait();
+#pragma unroll
+      for (int cq = 0; cq < WS_KT / 32; ++cq) reg_fence(sr[cq]);
       float mx;
       {
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-        uint32_t sb[2][32];
-        ptx::tmem_ld_32x32b_x32(t_s, sb[0]);
-        ptx::tmem_ld_wait();
-        reg_fence(sb[0]);
 #pragma unroll
         for (int cq = 0; cq < WS_KT / 32; ++cq) {
-          if (cq + 1 < WS_KT / 32) ptx::tmem_ld_32x32b_x32(t_s + (cq + 1) * 32, sb[(cq + 1) & 1]);
-          uint32_t(&r)[32] = sb[cq & 1];
           if (diag_w) {
 #pragma unroll
             for (int i = 0; i < 32; ++i)
-              m4[i & 3] = fmaxf(m4[i & 3], kbase + cq * 32 + i > pos ? -INFINITY : __uint_as_float(r[i]));
+              m4[i & 3] = fmaxf(m4[i & 3], kbase + cq * 32 + i > pos ? -INFINITY : __uint_as_float(sr[cq][i]));
           } else {
 #pragma unroll
-            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(r[i]));
-          }
-          if (cq + 1 < WS_KT / 32) {
-            ptx::tmem_ld_wait();
-            reg_fence(sb[(cq + 1) & 1]);
+            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(sr[cq][i]));
           }
         }
         mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * sl2;
@@ -411,29 +389,21 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           tmem_st_x32(t_o + cb * 32, orr);
         }
       }
-      // pass 2: P = exp2(s * scale - m) as bf16 pairs over the consumed S columns (chunk cq's P
-      // lands in columns [16cq, 16cq + 16), already read); loads pipelined as in pass 1; the
-      // scale and the row sum run as packed f32x2 FFMA2 / FADD2 (half the FMA-pipe issues)
+      // P = exp2(s * scale - m) as bf16 pairs written over the S columns (chunk cq's P lands in
+      // columns [16cq, 16cq + 16), whose scores are already in registers); the scale and the row
+      // sum run as packed f32x2 FFMA2 / FADD2 (half the FMA-pipe issues)
       float la = 0.f, lb = 0.f;
       {
         const uint64_t sc2 = f2pack(sl2, sl2), nm2 = f2pack(-m_ref, -m_ref);
         uint64_t l2 = f2pack(0.f, 0.f);
-        uint32_t sb[2][32];
-        ptx::tmem_ld_32x32b_x32(t_s, sb[0]);
-        ptx::tmem_ld_wait();
-        reg_fence(sb[0]);
 #pragma unroll
         for (int cq = 0; cq < WS_KT / 32; ++cq) {
-          if (cq + 1 < WS_KT / 32) ptx::tmem_ld_32x32b_x32(t_s + (cq + 1) * 32, sb[(cq + 1) & 1]);
-          const uint32_t(&sr)[32] = sb[cq & 1];
           uint32_t pw[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
             float x0, x1;
-            f2unpack(ffma2(f2pack(__uint_as_float(sr[2 * i]), __uint_as_float(sr[2 * i + 1])), sc2, nm2), x0, x1);
-            // EMU: one pair in four on the FMA pipe (A/B; measured slower at D = 128)
-            float p0 = MODE == 2 ? x0 : (MODE == 1 && (i & 3) == 3) ? exp2_fma(x0) : ex2(x0);
-            float p1 = MODE == 2 ? x1 : (MODE == 1 && (i & 3) == 3) ? exp2_fma(x1) : ex2(x1);
+            f2unpack(ffma2(f2pack(__uint_as_float(sr[cq][2 * i]), __uint_as_float(sr[cq][2 * i + 1])), sc2, nm2), x0, x1);
+            float p0 = ex2(x0), p1 = ex2(x1);
             if (diag_w) {
               if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
               if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;
@@ -442,10 +412,6 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
             pw[i] = ptx::pack_bf16(p0, p1);
           }
           tmem_st_x16(t_s + cq * 16, pw);
-          if (cq + 1 < WS_KT / 32) {
-            ptx::tmem_ld_wait();
-            reg_fence(sb[(cq + 1) & 1]);
-          }
         }
         f2unpack(l2, la, lb);
       }
@@ -488,35 +454,17 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   }
 }
 
-const int g_prefill_mode = [] {
-  const char* e = std::getenv("GLLM_PREFILL_EMU");
-  const char* p = std::getenv("GLLM_PREFILL_PROBE");
-  if (p && (p[0] == '2' || p[0] == '3')) return p[0] - '0';
-  return (e && e[0] == '1') ? 1 : 0;
-}();
-
-template <int D, int MODE>
+template <int D>
 int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
               int n_items, cudaStream_t s) {
   constexpr int bytes = WsSmem<D>::BYTES;
   static bool set = false;
   if (!set) {
-    cudaFuncSetAttribute(prefill_attn_ws_kernel<D, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(prefill_attn_ws_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  launch_pdl(prefill_attn_ws_kernel<D, MODE>, dim3(a.Hkv, n_items), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
+  launch_pdl(prefill_attn_ws_kernel<D>, dim3(a.Hkv, n_items), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
   return GLLM_OK;
-}
-
-template <int D>
-void launch_mode(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
-                 int n_items, cudaStream_t s) {
-  switch (g_prefill_mode) {
-    case 1: launch_ws<D, 1>(a, tmk, tmv, items, n_items, s); break;
-    case 2: launch_ws<D, 2>(a, tmk, tmv, items, n_items, s); break;
-    case 3: launch_ws<D, 3>(a, tmk, tmv, items, n_items, s); break;
-    default: launch_ws<D, 0>(a, tmk, tmv, items, n_items, s);
-  }
 }
 
 }  // namespace
@@ -528,9 +476,9 @@ int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const
   if (n_items <= 0) return GLLM_OK;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "prefill attention (ws): block size %d unsupported", a.bs);
   if (a.D == 128)
-    launch_mode<128>(a, tmk, tmv, items, n_items, s);
+    launch_ws<128>(a, tmk, tmv, items, n_items, s);
   else if (a.D == 64)
-    launch_mode<64>(a, tmk, tmv, items, n_items, s);
+    launch_ws<64>(a, tmk, tmv, items, n_items, s);
   else
     return set_error(GLLM_EINVAL, "prefill attention (ws): head_dim %d unsupported", a.D);
   cudaError_t e = cudaGetLastError();

@@ -23,7 +23,7 @@ struct MergeItem {
 struct AttnArgs {
   const __nv_bfloat16* q;  // [T, q_stride] (rotated q heads first in each row)
   int q_stride;
-  const __nv_bfloat16* kc;  // [kv_blocks][Hkv][bs][D]
+  const __nv_bfloat16* kc;  // [kv_blocks][Hkv] pages of bs x D, SMEM-ready layout (kvpage.cuh)
   const __nv_bfloat16* vc;
   int Hq, Hkv, D, bs;
   const int32_t* cu_q;
@@ -37,18 +37,16 @@ struct AttnArgs {
   int* part_ctr;       // [nparts * Hkv] split arrival counters (persistent decode kernel; kept zero)
 };
 
-// warp-specialised tcgen05 prefill (attention_prefill_ws.cu), the default: items of
-// prefill_ws_rows_per_item() rows (two 128-row Q tiles); K/V pages by TMA through the decode page maps
+// warp-specialised tcgen05 prefill (attention_prefill_ws.cu): items of prefill_ws_rows_per_item()
+// rows (two 128-row Q tiles); K / V pages (SMEM-ready layout, kvpage.cuh) by 16-byte cp.async
 int prefill_ws_rows_per_item();
-int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
-                                const PrefillItem* items, int n_items, cudaStream_t s);
-// persistent warp-worker decode kernel fed by TMA (attention_decode.cu), the default; `tmk` /
-// `tmv` map the layer's K / V cache as [kv_blocks*Hkv*16, D] bf16 with 16 x 64 SW128 boxes;
-// `ctr` = 2 device ints, zero before the first launch (the kernel leaves them zero)
+int launch_prefill_attention_ws(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s);
+// persistent warp-worker decode kernel (attention_decode.cu): each K / V page (SMEM-ready layout,
+// kvpage.cuh) is one 1-D bulk copy; `ctr` = 2 device ints, zero before the first launch (the kernel
+// leaves them zero)
 bool decode_tma_supported(int D, int G);
 int decode_workers(int num_sms);  // warp workers of the persistent decode kernel
-int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
-                                const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
-                                int num_sms, cudaStream_t s);
+int launch_decode_attention_tma(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
+                                int n_merges, int* ctr, int num_sms, cudaStream_t s);
 
 }  // namespace gllm

@@ -49,11 +49,9 @@ struct DecLayout {
 
 template <int D, int G, int NST, int WARPS>
 __global__ void __launch_bounds__(WARPS * 32)
-    decode_attn_tma_kernel(const AttnArgs a, const DecodeItem* __restrict__ items, int n_work, int* __restrict__ ctr,
-                           const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
+    decode_attn_tma_kernel(const AttnArgs a, const DecodeItem* __restrict__ items, int n_work, int* __restrict__ ctr) {
   using Lay = DecLayout<D, G, NST, WARPS>;
   static_assert(G >= 1 && G <= 8, "GQA group must fit the 16-row MMA tile");
-  constexpr int ATOMS = D / 64;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -70,10 +68,6 @@ __global__ void __launch_bounds__(WARPS * 32)
   if (lane == 0) {
     for (int s = 0; s < NST; ++s) ptx::mbar_init(&bar[s], 1);
     ptx::fence_barrier_init();
-    if (warp == 0) {
-      ptx::tma_prefetch(&tmk);
-      ptx::tma_prefetch(&tmv);
-    }
   }
   __syncwarp();
   pdl_wait();  // work counter, Q rows, block table, KV pages: all produced by earlier kernels
@@ -126,16 +120,13 @@ __global__ void __launch_bounds__(WARPS * 32)
     }
     const int blk = __shfl_sync(0xffffffffu, btw, ip & 31);
     if (lane == 0) {
-      const int row = (blk * Hkv + i_kvh) * 16;
+      const int64_t page = (int64_t)blk * Hkv + i_kvh;  // SMEM-ready page (kvpage.cuh): one copy each
       const bool first = ip == 0;
       fence_proxy_async();  // this slot's earlier generic reads (ldmatrix) before the async writes
       ptx::mbar_arrive_expect_tx(&bar[s], Lay::SLOT);
       uint8_t* dst = ring + s * Lay::SLOT;
-#pragma unroll
-      for (int at = 0; at < ATOMS; ++at) {
-        ptx::tma_load_2d_hint(dst + at * 2048, &tmk, &bar[s], at * 64, row, pol);
-        ptx::tma_load_2d_hint(dst + Lay::PAGE + at * 2048, &tmv, &bar[s], at * 64, row, pol);
-      }
+      ptx::bulk_load_hint(dst, a.kc + page * 16 * D, Lay::PAGE, &bar[s], pol);
+      ptx::bulk_load_hint(dst + Lay::PAGE, a.vc + page * 16 * D, Lay::PAGE, &bar[s], pol);
       meta[s] = make_int4(iw, ip, (ip == inp - 1 ? 1 : 0) | (first ? 2 : 0), 0);
     }
     if (++ip == inp) {
@@ -359,7 +350,7 @@ __global__ void __launch_bounds__(WARPS * 32)
 }
 
 template <int D, int G, int NST, int WARPS>
-int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items,
+int launch_t(const AttnArgs& a, const DecodeItem* items,
              int n_items, const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   using Lay = DecLayout<D, G, NST, WARPS>;
   static int per_sm = 0;
@@ -376,7 +367,7 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
     const int need = (n_work + WARPS - 1) / WARPS;
     if (grid > need) grid = need;
     launch_pdl(decode_attn_tma_kernel<D, G, NST, WARPS>, dim3(grid), dim3(WARPS * 32), Lay::BYTES, s, 1, a, items,
-               n_work, ctr, tmk, tmv);
+               n_work, ctr);
   }
   (void)merges;
   (void)n_merges;  // split rows are merged inside the kernel by their last split
@@ -384,22 +375,22 @@ int launch_t(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, 
 }
 
 template <int D, int G>
-int launch_g(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items, int n_items,
+int launch_g(const AttnArgs& a, const DecodeItem* items, int n_items,
              const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   // 3-slot page ring x 4 warps, 2 CTAs per SM (profiles/r02/decode_split_ab.txt: 6 slots x 4 warps at
   // 1 CTA per SM is 15-25% slower -- the per-page mma.sync work of fewer warps limits it)
-  return launch_t<D, G, 3, 4>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
+  return launch_t<D, G, 3, 4>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
 }
 
 template <int D>
-int launch_d(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const DecodeItem* items, int n_items,
+int launch_d(const AttnArgs& a, const DecodeItem* items, int n_items,
              const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   switch (a.Hq / a.Hkv) {
-    case 1: return launch_g<D, 1>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-    case 2: return launch_g<D, 2>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-    case 4: return launch_g<D, 4>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-    case 5: return launch_g<D, 5>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
-    case 8: return launch_g<D, 8>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 1: return launch_g<D, 1>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 2: return launch_g<D, 2>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 4: return launch_g<D, 4>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 5: return launch_g<D, 5>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 8: return launch_g<D, 8>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   }
   return set_error(GLLM_EINVAL, "decode attention (tma): unsupported GQA group %d", a.Hq / a.Hkv);
 }
@@ -412,15 +403,14 @@ int decode_workers(int num_sms) {  // warp workers of the persistent decode kern
 
 bool decode_tma_supported(int D, int G) { return (D == 64 || D == 128) && (G == 1 || G == 2 || G == 4 || G == 5 || G == 8); }
 
-int launch_decode_attention_tma(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
-                                const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
+int launch_decode_attention_tma(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
                                 int num_sms, cudaStream_t s) {
   int rc;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "decode attention (tma): block size %d != 16", a.bs);
   if (a.D == 128)
-    rc = launch_d<128>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
+    rc = launch_d<128>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   else if (a.D == 64)
-    rc = launch_d<64>(a, tmk, tmv, items, n_items, merges, n_merges, ctr, num_sms, s);
+    rc = launch_d<64>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   else
     return set_error(GLLM_EINVAL, "decode attention (tma): head_dim %d unsupported", a.D);
   if (rc) return rc;

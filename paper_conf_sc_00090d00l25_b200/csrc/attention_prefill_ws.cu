@@ -143,8 +143,7 @@ __device__ __forceinline__ void umma_bf16_ta(uint32_t tmem_d, uint32_t tmem_a, u
 
 template <int D>
 __global__ void __launch_bounds__(WS_THREADS, 1)
-    prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items,
-                           const __grid_constant__ CUtensorMap tmk, const __grid_constant__ CUtensorMap tmv) {
+    prefill_attn_ws_kernel(const AttnArgs a, const PrefillItem* __restrict__ items) {
   using L = WsSmem<D>;
   constexpr int ATOMS = L::ATOMS;
   constexpr int NCH = D / 8;  // 16-byte chunks per Q row
@@ -199,8 +198,6 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::mbar_init(&ofull[x], 1);
     }
     ptx::fence_barrier_init();
-    ptx::tma_prefetch(&tmk);
-    ptx::tma_prefetch(&tmv);
   }
   if (warp == 0) {
     ptx::tmem_alloc(tmem_slot, 512);
@@ -216,18 +213,27 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 
   if (warp < 4) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;" ::: "memory");
   if (warp == 0 || warp == 2) {
-    // ---------------- TMA producers: warp 0 streams the K tiles, warp 2 the V tiles, each as soon as
-    // its slot frees (K: the S MMAs of both Q tiles reading it completed; V: the PV MMAs), so the
-    // deeper K ring runs ahead of the V waits.  Lanes 0..7 read the 8 block ids of the next tile.
+    // ---------------- K / V producers: warp 0 streams the K tiles, warp 2 the V tiles.  A page of
+    // the cache is already in the SW128 layout (kvpage.cuh), so each 2 KB page atom is copied with
+    // 16-byte cp.async (lane l: chunks l, l+32, l+64, l+96; a warp instruction moves 512 B) to its
+    // rows of the tile: 16 x 2 KB TMA boxes per tile cost ~2000 cycles of TMA issue per SM, as much
+    // as the tile's four MMAs.  A tile's copies are one commit group; the tile is published (fence
+    // to the async proxy, then one arrive) once the group completes, while the next tile's copies
+    // are in flight.  K ring 3 deep, V ring 2 (V is needed only after the tile's softmax).
     const bool is_k = warp == 0;
-    const CUtensorMap* map = is_k ? &tmk : &tmv;
+    const __nv_bfloat16* cache = is_k ? a.kc : a.vc;
     const int ns = is_k ? WS_NSK : WS_NSV;
     uint64_t* full = is_k ? kfull : vfull;
     uint64_t* empty = is_k ? kempty : vempty;
-    const uint32_t base = is_k ? L::K : L::V;
+    const uint32_t base = sbase + (is_k ? L::K : L::V);
     auto read_bt = [&](int j) {  // block ids of tile j's pages (past the sequence: its page 0)
       const int kb = j * PAGES + lane;
       return (lane < PAGES && j < n_kt) ? __ldg(bt + (kb < nblk_seq ? kb : 0)) : 0;
+    };
+    auto publish = [&](int j) {  // tile j's copies (the older commit group) landed
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&full[j % ns]);
     };
     int bnext = read_bt(0);
 #pragma unroll 1
@@ -236,18 +242,28 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 #pragma unroll
       for (int p = 0; p < PAGES; ++p) bp[p] = __shfl_sync(0xffffffffu, bnext, p);
       bnext = read_bt(j + 1);
-      if (lane == 0) {
-        const int sl = j % ns;
-        if (j >= ns) ptx::mbar_wait(&empty[sl], (uint32_t)(((j / ns) - 1) & 1));
-        ptx::mbar_arrive_expect_tx(&full[sl], L::KV_TILE);
-        const uint32_t dst = base + sl * L::KV_TILE;
+      const int sl = j % ns;
+      if (j >= ns) ptx::mbar_wait(&empty[sl], (uint32_t)(((j / ns) - 1) & 1));
+      const uint32_t dst = base + sl * L::KV_TILE;
 #pragma unroll
-        for (int p = 0; p < PAGES; ++p)
+      for (int p = 0; p < PAGES; ++p) {
+        const __nv_bfloat16* src = cache + ((int64_t)bp[p] * a.Hkv + kvh) * 16 * D;
 #pragma unroll
-          for (int at = 0; at < ATOMS; ++at)
-            ptx::tma_load_2d(smem + dst + at * L::KV_ATOM + p * 2048, map, &full[sl], at * 64, (bp[p] * a.Hkv + kvh) * 16);
+        for (int at = 0; at < ATOMS; ++at)
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            ptx::cp_async16(dst + at * L::KV_ATOM + p * 2048 + (lane + 32 * q) * 16, src + at * 1024 + (lane + 32 * q) * 8,
+                            true);
       }
-      __syncwarp();
+      ptx::cp_async_commit();
+      if (j >= 1) {
+        ptx::cp_async_wait<1>();
+        publish(j - 1);
+      }
+    }
+    if (n_kt > 0) {
+      ptx::cp_async_wait<0>();
+      publish(n_kt - 1);
     }
   } else if (warp == 1) {
     // ---------------- MMA issuer
@@ -455,15 +471,14 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 }
 
 template <int D>
-int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv, const PrefillItem* items,
-              int n_items, cudaStream_t s) {
+int launch_ws(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
   constexpr int bytes = WsSmem<D>::BYTES;
   static bool set = false;
   if (!set) {
     cudaFuncSetAttribute(prefill_attn_ws_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     set = true;
   }
-  launch_pdl(prefill_attn_ws_kernel<D>, dim3(a.Hkv, n_items), dim3(WS_THREADS), bytes, s, 1, a, items, tmk, tmv);
+  launch_pdl(prefill_attn_ws_kernel<D>, dim3(a.Hkv, n_items), dim3(WS_THREADS), bytes, s, 1, a, items);
   return GLLM_OK;
 }
 
@@ -471,14 +486,13 @@ int launch_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
 
 int prefill_ws_rows_per_item() { return 2 * WS_ROWS; }
 
-int launch_prefill_attention_ws(const AttnArgs& a, const CUtensorMap& tmk, const CUtensorMap& tmv,
-                                const PrefillItem* items, int n_items, cudaStream_t s) {
+int launch_prefill_attention_ws(const AttnArgs& a, const PrefillItem* items, int n_items, cudaStream_t s) {
   if (n_items <= 0) return GLLM_OK;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "prefill attention (ws): block size %d unsupported", a.bs);
   if (a.D == 128)
-    launch_ws<128>(a, tmk, tmv, items, n_items, s);
+    launch_ws<128>(a, items, n_items, s);
   else if (a.D == 64)
-    launch_ws<64>(a, tmk, tmv, items, n_items, s);
+    launch_ws<64>(a, items, n_items, s);
   else
     return set_error(GLLM_EINVAL, "prefill attention (ws): head_dim %d unsupported", a.D);
   cudaError_t e = cudaGetLastError();

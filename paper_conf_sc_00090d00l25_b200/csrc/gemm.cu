@@ -26,6 +26,7 @@
 
 #include "common.h"
 #include "gemm.cuh"
+#include "kvpage.cuh"
 #include "launch.cuh"
 #include "ptx.cuh"
 
@@ -231,21 +232,30 @@ __device__ __forceinline__ void qkv_rope_store(const GemmArgs& p, int row, int c
       x2[2 * j + 1] = b2 * v.z + b1 * v.w;
     }
   }
-  __nv_bfloat16 *dst1, *dst2;
   if (col1 < p.q_dim) {
     __nv_bfloat16* out = reinterpret_cast<__nv_bfloat16*>(p.out) + (size_t)row * p.ldo;
-    dst1 = out + col1;
-    dst2 = out + col1 + half;
-  } else {
+    store_bf16x32(out + col1, x1);
+    store_bf16x32(out + col1 + half, x2);
+  } else {  // paged K / V append in the SMEM-ready page layout (kvpage.cuh): four 16-byte chunks each
     const bool is_k = col1 < p.q_dim + p.kv_dim;
     const int cc = col1 - p.q_dim - (is_k ? 0 : p.kv_dim);
-    const int h = cc / D;
-    __nv_bfloat16* base = (is_k ? p.kc : p.vc) + ((blk * p.n_kv_heads + h) * p.block_size + off) * D;
-    dst1 = base + i0;
-    dst2 = base + i0 + half;
+    const int64_t page = blk * p.n_kv_heads + cc / D;
+    __nv_bfloat16* cache = is_k ? p.kc : p.vc;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint4 w1, w2;
+      w1.x = ptx::pack_bf16(x1[8 * q + 0], x1[8 * q + 1]);
+      w1.y = ptx::pack_bf16(x1[8 * q + 2], x1[8 * q + 3]);
+      w1.z = ptx::pack_bf16(x1[8 * q + 4], x1[8 * q + 5]);
+      w1.w = ptx::pack_bf16(x1[8 * q + 6], x1[8 * q + 7]);
+      w2.x = ptx::pack_bf16(x2[8 * q + 0], x2[8 * q + 1]);
+      w2.y = ptx::pack_bf16(x2[8 * q + 2], x2[8 * q + 3]);
+      w2.z = ptx::pack_bf16(x2[8 * q + 4], x2[8 * q + 5]);
+      w2.w = ptx::pack_bf16(x2[8 * q + 6], x2[8 * q + 7]);
+      *reinterpret_cast<uint4*>(cache + kv_page_elem(page, (int)off, i0 + 8 * q, D)) = w1;
+      *reinterpret_cast<uint4*>(cache + kv_page_elem(page, (int)off, i0 + half + 8 * q, D)) = w2;
+    }
   }
-  store_bf16x32(dst1, x1);
-  store_bf16x32(dst2, x2);
 }
 
 // fused RMSNorm scale of an output row (1 when the A operand is already normalised)

@@ -5,6 +5,7 @@
 #include <cuda_bf16.h>
 
 #include "kernels.cuh"
+#include "kvpage.cuh"
 #include "launch.cuh"
 
 #include <cstdlib>
@@ -69,7 +70,7 @@ __global__ void fill_warm_kv_kernel(__nv_bfloat16* kc, __nv_bfloat16* vc, const 
   for (int e = threadIdx.x; e < np * per_pos; e += blockDim.x) {
     const int o = e / per_pos, hd = e - o * per_pos, h = hd / D, j = hd - h * D;
     const uint64_t i = (base + (uint64_t)(p0 + o)) * (uint64_t)per_pos + (uint64_t)hd;
-    const int64_t dst = ((blk * Hkv + h) * bs + o) * (int64_t)D + j;
+    const int64_t dst = kv_page_elem(blk * Hkv + h, o, j, D);  // SMEM-ready page layout (kvpage.cuh)
     kc[dst] = __float2bfloat16_rn(o4(seed, tid, i, 1.7320508f));
     vc[dst] = __float2bfloat16_rn(o4(seed, tid + 1, i, 1.7320508f));
   }

@@ -25,6 +25,7 @@
 #include "common.h"
 #include "gemm.cuh"
 #include "kernels.cuh"
+#include "kvpage.cuh"
 
 using bf16 = __nv_bfloat16;
 
@@ -52,8 +53,7 @@ struct LayerW {
   bf16 *wqkv = nullptr, *wo = nullptr, *wgu = nullptr, *wd = nullptr;
   float* bqkv = nullptr;
   bf16 *kc = nullptr, *vc = nullptr;
-  CUtensorMap tm_qkv, tm_o, tm_gu, tm_d;
-  CUtensorMap tm_kc, tm_vc;  // paged K / V cache as [kv_blocks*Hkv*16, D] (16 x 64 SW128 boxes)
+  CUtensorMap tm_qkv, tm_o, tm_gu, tm_d;  // (the paged K / V cache needs no tensor map: kvpage.cuh)
 };
 
 constexpr int RING = 4;
@@ -400,9 +400,7 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_B_BOX)) ||
         (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_B_BOX)) ||
         (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_kc, w.kc, (uint64_t)kv_blocks * Hkv * block_size, D, 16)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_vc, w.vc, (uint64_t)kv_blocks * Hkv * block_size, D, 16)))
+        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)))
       return fail(rc);
     st->layers.push_back(w);
   }
@@ -739,7 +737,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     aa.vc = w.vc;
     auto decode = [&](cudaStream_t ds) -> int {
       st->last_launches += 1;  // the persistent kernel merges split rows in place
-      return gllm::launch_decode_attention_tma(aa, w.tm_kc, w.tm_vc, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
+      return gllm::launch_decode_attention_tma(aa, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
                                                st->num_sms, ds);
     };
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
@@ -754,7 +752,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       }
       {
         Prof p(st, ps, C_PREFILL);
-        RC(gllm::launch_prefill_attention_ws(aa, w.tm_kc, w.tm_vc, d_pi, P.n_pi, ps));
+        RC(gllm::launch_prefill_attention_ws(aa, d_pi, P.n_pi, ps));
       }
       if (overlap) CK(cudaEventRecord(st->ev_join, ps));
       st->last_launches += 1;
@@ -1007,17 +1005,20 @@ int gllm_stage_read_kv(gllm_stage* st, int32_t layer, const int32_t* slots, int3
   cudaSetDevice(st->device);
   LayerW& w = st->layers[layer - st->lb];
   const int Hkv = st->cfg.n_kv_heads, D = st->cfg.head_dim, bs = st->bs;
-  std::vector<bf16> tmp(D);
+  std::vector<bf16> pk(bs * D), pv(bs * D);  // one page (SMEM-ready layout, kvpage.cuh)
   for (int i = 0; i < n; ++i) {
     const int64_t sl = slots[i];
     if (sl < 0 || sl >= (int64_t)st->kv_blocks * bs) return gllm::set_error(GLLM_EINVAL, "slot out of range");
     const int64_t blk = sl / bs, o = sl % bs;
     for (int h = 0; h < Hkv; ++h) {
-      const size_t idx = ((blk * Hkv + h) * bs + o) * D;
-      CK(cudaMemcpy(tmp.data(), w.kc + idx, D * sizeof(bf16), cudaMemcpyDeviceToHost));
-      for (int j = 0; j < D; ++j) k_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(tmp[j]);
-      CK(cudaMemcpy(tmp.data(), w.vc + idx, D * sizeof(bf16), cudaMemcpyDeviceToHost));
-      for (int j = 0; j < D; ++j) v_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(tmp[j]);
+      const int64_t page = blk * Hkv + h;
+      CK(cudaMemcpy(pk.data(), w.kc + page * bs * D, bs * D * sizeof(bf16), cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(pv.data(), w.vc + page * bs * D, bs * D * sizeof(bf16), cudaMemcpyDeviceToHost));
+      for (int j = 0; j < D; ++j) {
+        const int64_t e = gllm::kv_page_elem(0, (int)o, j, D);
+        k_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(pk[e]);
+        v_out[((size_t)i * Hkv + h) * D + j] = __bfloat162float(pv[e]);
+      }
     }
   }
   return GLLM_OK;

@@ -46,9 +46,7 @@ int launch_prefill_attention_ws(const AttnArgs& a, const PrefillItem* items, int
 // leaves them zero)
 bool decode_tma_supported(int D, int G);
 int decode_workers(int num_sms);  // warp workers of the persistent decode kernel
-// num_sms: SMs the grid may occupy; whole_sm: one 8-warp CTA per SM (the grid then occupies exactly
-// num_sms SMs, leaving the rest to a concurrent kernel) instead of two 4-warp CTAs
 int launch_decode_attention_tma(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges,
-                                int n_merges, int* ctr, int num_sms, bool whole_sm, cudaStream_t s);
+                                int n_merges, int* ctr, int num_sms, cudaStream_t s);
 
 }  // namespace gllm

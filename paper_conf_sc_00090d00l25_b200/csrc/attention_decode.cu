@@ -376,24 +376,21 @@ int launch_t(const AttnArgs& a, const DecodeItem* items,
 
 template <int D, int G>
 int launch_g(const AttnArgs& a, const DecodeItem* items, int n_items,
-             const MergeItem* merges, int n_merges, int* ctr, int num_sms, bool whole_sm, cudaStream_t s) {
+             const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   // 3-slot page ring x 4 warps, 2 CTAs per SM (profiles/r02/decode_split_ab.txt: 6 slots x 4 warps at
-  // 1 CTA per SM is 15-25% slower -- the per-page mma.sync work of fewer warps limits it).
-  // whole_sm: the same 8 warps per SM as one CTA of 8 warps (192 KB), so a grid of n CTAs occupies
-  // exactly n SMs and leaves the others to the concurrent prefill kernel (SM partitioning).
-  if (whole_sm) return launch_t<D, G, 3, 8>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+  // 1 CTA per SM is 15-25% slower -- the per-page mma.sync work of fewer warps limits it)
   return launch_t<D, G, 3, 4>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
 }
 
 template <int D>
 int launch_d(const AttnArgs& a, const DecodeItem* items, int n_items,
-             const MergeItem* merges, int n_merges, int* ctr, int num_sms, bool whole_sm, cudaStream_t s) {
+             const MergeItem* merges, int n_merges, int* ctr, int num_sms, cudaStream_t s) {
   switch (a.Hq / a.Hkv) {
-    case 1: return launch_g<D, 1>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
-    case 2: return launch_g<D, 2>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
-    case 4: return launch_g<D, 4>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
-    case 5: return launch_g<D, 5>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
-    case 8: return launch_g<D, 8>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
+    case 1: return launch_g<D, 1>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 2: return launch_g<D, 2>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 4: return launch_g<D, 4>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 5: return launch_g<D, 5>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
+    case 8: return launch_g<D, 8>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   }
   return set_error(GLLM_EINVAL, "decode attention (tma): unsupported GQA group %d", a.Hq / a.Hkv);
 }
@@ -407,13 +404,13 @@ int decode_workers(int num_sms) {  // warp workers of the persistent decode kern
 bool decode_tma_supported(int D, int G) { return (D == 64 || D == 128) && (G == 1 || G == 2 || G == 4 || G == 5 || G == 8); }
 
 int launch_decode_attention_tma(const AttnArgs& a, const DecodeItem* items, int n_items, const MergeItem* merges, int n_merges, int* ctr,
-                                int num_sms, bool whole_sm, cudaStream_t s) {
+                                int num_sms, cudaStream_t s) {
   int rc;
   if (a.bs != 16) return set_error(GLLM_EINVAL, "decode attention (tma): block size %d != 16", a.bs);
   if (a.D == 128)
-    rc = launch_d<128>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
+    rc = launch_d<128>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   else if (a.D == 64)
-    rc = launch_d<64>(a, items, n_items, merges, n_merges, ctr, num_sms, whole_sm, s);
+    rc = launch_d<64>(a, items, n_items, merges, n_merges, ctr, num_sms, s);
   else
     return set_error(GLLM_EINVAL, "decode attention (tma): head_dim %d unsupported", a.D);
   if (rc) return rc;

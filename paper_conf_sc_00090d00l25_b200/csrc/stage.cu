@@ -101,7 +101,6 @@ size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 struct Prepared {
   bool in_use = false;
   int T = 0, S = 0, NP = 0, maxblk = 0, ns = 0, n_pi = 0, n_di = 0, n_mi = 0, split_len = 16, nparts = 0;
-  int dec_sms = 0;  // > 0: SMs the decode kernel occupies when it runs concurrently with prefill
   size_t o_ids = 0, o_pos = 0, o_cu = 0, o_kvl = 0, o_bt = 0, o_samp = 0, o_pi = 0, o_di = 0, o_mi = 0, bytes = 0;
   uint8_t* host = nullptr;
   uint8_t* dev = nullptr;
@@ -144,7 +143,6 @@ struct gllm_stage {
   int last_T = 0, last_launches = 0;
   bool profiling = false;
   bool deterministic = false;  // gllm_stage_set_deterministic: GEMM schedules with a fixed reduction order
-  bool sm_partition = true;    // TEMPORARY A/B (GLLM_SM_PART=0): decode / prefill SM partitioning
   bool prof_serial_attn = false;  // gllm_stage_set_profiling(st, 2): attribution pass, attention in series
   // fused peer hand-off (a12, gllm_peer_*): receive ring owned here / the next stage's ring mapped here
   float* ring = nullptr;
@@ -436,7 +434,6 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   CK(cudaMemsetAsync(st->dec_ctr, 0, 2 * sizeof(int), s0));
   CK(cudaMemsetAsync(st->release_ctr, 0, sizeof(unsigned), s0));
   CK(cudaMemsetAsync(st->y, 0, R * H * sizeof(bf16), s0));
-  if (const char* e = std::getenv("GLLM_SM_PART")) st->sm_partition = e[0] != '0';
   if (!gllm::decode_tma_supported(D, cfg->n_heads / Hkv))
     return fail(gllm::set_error(GLLM_EINVAL, "decode attention: head_dim %d / GQA group %d unsupported", D,
                                 cfg->n_heads / Hkv));
@@ -529,32 +526,6 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
     pitems.swap(sorted);
   }
   const int ND = S - NP;
-  // SM partitioning of the attention step (prefill || decode on two streams): decode is HBM-bound
-  // and saturates HBM from ~80 SMs (tools/micro/hbm_sm_sweep.cu), prefill is tensor-bound.  Give
-  // decode n SMs (one 8-warp CTA each) and leave the rest to the prefill CTAs, n minimising the
-  // modelled span max(t_dec(n), t_pre(148 - n)); otherwise the persistent decode CTAs, launched
-  // early by PDL, hold every SM and the side-stream prefill waits behind them.
-  P.dec_sms = 0;
-  if (ND > 0 && NP > 0 && st->sm_partition) {
-    double pairs = 0.0;
-    for (int i = 0; i < NP; ++i) {
-      const double cq = d->cu_q[i + 1] - d->cu_q[i], s0 = d->kv_len[i] - cq;
-      pairs += cq * s0 + cq * (cq + 1) / 2;
-    }
-    const double t_pre = pairs * 4.0 * c.n_heads * c.head_dim / 5.5e14;            // s at full GPU
-    const double t_dec = (double)total_pages * 16 * 4.0 * c.n_kv_heads * c.head_dim / 6.4e12;
-    const int sms = st->num_sms;
-    double best = 1e30;
-    for (int n = 48; n <= sms; n += 4) {
-      const double td = t_dec * std::max(1.0, 80.0 / n);
-      const double tp = n < sms ? t_pre * sms / (double)(sms - n) : 1e30;
-      const double span = n == sms ? t_dec + t_pre : std::max(td, tp);
-      if (span < best) {
-        best = span;
-        P.dec_sms = n == sms ? 0 : n;
-      }
-    }
-  }
   int split_pages = 1 << 30;
   if (ND > 0) {
     // Split rows longer than one warp worker's fair share of the (page, kv head) units, so the
@@ -562,7 +533,7 @@ int prepare_impl(gllm_stage* st, const gllm_batch_desc* d, cudaStream_t s, Prepa
     // a row at most 32 splits) so the in-place merge stays a few % of the row's bytes.  Measured on
     // B200 (profiles/r02/decode_split_ab.txt) against equal-length splits filling the workers in
     // k >= 2 rounds: the fair-share split is faster on C1 (800 rows) and on C3's few long rows.
-    const int64_t W = gllm::decode_workers(P.dec_sms ? P.dec_sms : st->num_sms);
+    const int64_t W = gllm::decode_workers(st->num_sms);
     int max_pages = 1;
     for (int i = NP; i < S; ++i) max_pages = std::max(max_pages, (d->kv_len[i] + bs - 1) / bs);
     const int64_t per = (total_pages * c.n_kv_heads + W - 1) / W;
@@ -766,9 +737,8 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     aa.vc = w.vc;
     auto decode = [&](cudaStream_t ds) -> int {
       st->last_launches += 1;  // the persistent kernel merges split rows in place
-      const bool part = P.dec_sms > 0 && !st->prof_serial_attn;
       return gllm::launch_decode_attention_tma(aa, d_di, P.n_di, d_mi, P.n_mi, st->dec_ctr,
-                                               part ? P.dec_sms : st->num_sms, part, ds);
+                                               st->num_sms, ds);
     };
     // Prefill rows (tensor/latency-bound) run on the side stream concurrently with the decode rows
     // (HBM-bound) on the main stream; they write disjoint rows of the attention output.

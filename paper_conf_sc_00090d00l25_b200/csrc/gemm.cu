@@ -859,7 +859,11 @@ int choose_cg(int M, int N, int epi, int num_sms) {
   if (g_force_cg) return g_force_cg;
   const int nn = (N + GEMM_BN - 1) / GEMM_BN;
   const int tiles2 = ((M + 255) / 256) * nn;
-  if (M < 256 || tiles2 * 2 < num_sms || epi == EPI_ARGMAX) return 1;
+  if (M < 256 || epi == EPI_ARGMAX) return 1;
+  // below one wave of pair tiles the residual add takes stream-K over the pairs (hybrid_dp_tiles):
+  // the 1-CTA tile streams 48 KB of operands per 64-deep k-block, more than TMA's ~60-90 B/cycle per
+  // SM feeds at the MMA rate (tools/micro/tma_box.cu); the pair streams 32 KB per CTA
+  if (tiles2 * 2 < num_sms && epi != EPI_ADD_F32) return 1;
   // wave quantisation of whole tiles: the pair kernel is the faster per tile, but a 128-row tile
   // grid can fill its waves much better (C2's QKV at T ~ 625: 140 tiles on 148 SMs in one wave
   // vs 84 pair tiles on 74 pairs in two; measured 49 vs 68 us)
@@ -878,12 +882,16 @@ int choose_cg(int M, int N, int epi, int num_sms) {
 // the tail tiles' k-blocks are spread over every pair and combined with fp32 vector reductions.
 // Returns the whole-tile count (0 = no hybrid).  (Non-additive epilogues through the fp32 workspace
 // measured slower than whole tiles, profiles/r01/gemm_sched.txt.)
+// Returns the whole-tile count (-1 = no hybrid).  Below one wave of pair tiles that leaves more than
+// 15% of the pairs idle (C2's O / down GEMMs at T ~ 626: 60 tiles on 74 pairs), 0: every tile's
+// k-blocks are spread over all pairs (stream-K over the CTA-pair kernel).
 int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms) {
-  if (cg != 2 || epi != EPI_ADD_F32 || K / GEMM_BK < 8) return 0;
+  if (cg != 2 || epi != EPI_ADD_F32 || K / GEMM_BK < 8) return -1;
   const int units = num_sms / 2;
   const int ntiles = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
+  if (ntiles < units) return ntiles * 100 < units * 85 ? 0 : -1;
   const int tail = ntiles % units;
-  if (ntiles < units || tail == 0 || tail * 10 >= units * 8) return 0;
+  if (tail == 0 || tail * 10 >= units * 8) return -1;
   return ntiles - tail;
 }
 
@@ -907,7 +915,7 @@ bool gemm_uses_streamk(int M, int N, int K, int epi, int num_sms, bool determini
   if (M <= 0 || deterministic) return false;
   if (!g_force_cg && skc_split(M, N, K, epi, num_sms)) return false;  // whole tiles, reduced in-cluster
   const int cg = choose_cg(M, N, epi, num_sms);
-  if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms) > 0;
+  if (cg == 2) return hybrid_dp_tiles(M, N, K, epi, cg, num_sms) >= 0;
   const int ntiles = ((M + GEMM_BM - 1) / GEMM_BM) * ((N + GEMM_BN - 1) / GEMM_BN);
   return choose_streamk(M, N, ntiles, K / GEMM_BK, epi, num_sms) != 0;
 }
@@ -1020,7 +1028,7 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   bool hybrid = false;
   if (cg == 2 && !args.deterministic && !args.xb_out && !args.ss_out && !args.out_peer) {  // partial tiles: no fused outputs
     const int dp = hybrid_dp_tiles(args.M, args.N, args.K, epi, cg, num_sms);
-    if (dp > 0) {
+    if (dp >= 0) {
       const int ntiles2 = ((args.M + 255) / 256) * args.num_n_tiles, units = num_sms / 2;
       args.streamk = 2;
       args.dp_tiles = dp;

@@ -56,11 +56,13 @@ def test_residual_add_f32(M, N, K):
     assert err < 1e-3, err
 
 
-@pytest.mark.parametrize("M,N,K", [(900, 5120, 5120), (900, 5120, 27648), (1100, 4096, 4096), (2094, 5120, 5120)])
+@pytest.mark.parametrize("M,N,K", [(900, 5120, 5120), (900, 5120, 27648), (1100, 4096, 4096), (2094, 5120, 5120),
+                                   (626, 5120, 13824), (300, 5120, 5120)])
 def test_residual_add_f32_hybrid_tail(M, N, K):
     # CTA-pair tiles whose last wave is mostly empty (C3's O / down GEMMs at T ~ 900: 80 tiles of
     # 256 x 256 on 74 pairs): whole tiles first, the tail tiles' k-blocks spread over every pair
-    # and reduced into the residual (Jobs mode 2)
+    # and reduced into the residual (Jobs mode 2); below one wave (C2's O / down at T ~ 626: 60 tiles
+    # on 74 pairs) every tile's k-blocks are spread over all pairs
     A, W = _bf16((M, K), 1.0, 14), _bf16((N, K), K ** -0.5, 15)
     x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(16))
     dA, dW, x = A.cuda(), W.cuda(), x0.clone().cuda()

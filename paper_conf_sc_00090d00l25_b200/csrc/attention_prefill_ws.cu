@@ -32,6 +32,17 @@
 
 namespace gllm {
 
+#ifdef GLLM_VARIANT_TRACE
+// measurement build only (build.py --variant=trace): per-CTA timeline of the prefill kernel
+__device__ unsigned long long* g_pf_trace = nullptr;
+constexpr int PF_TR = 12;  // words per CTA record
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#endif
+
 namespace {
 
 constexpr float LOG2E_W = 1.4426950408889634f;
@@ -163,6 +174,10 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + L::NBAR);
 
   pdl_trigger();
+#ifdef GLLM_VARIANT_TRACE
+  const unsigned long long tr_t0 = gtime();
+  unsigned long long tr_wq = 0, tr_wk = 0, tr_wv = 0, tr_wp = 0;
+#endif
   pdl_wait();
   // grid (Hkv, items): CTAs are dispatched x-fastest, so every kv head of the longest item goes
   // first and the whole grid runs longest-first (the host sorts items by key tiles)
@@ -286,11 +301,21 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           umma_bf16_ta(tmem + 256 + x * 128, tmem + x * 128 + kk * 8, desc_mn(vb + kk * 2048, L::KV_ATOM), idesc_o,
                        (j > 0 || kk > 0) ? 1u : 0u);
       };
+#ifdef GLLM_VARIANT_TRACE
+#define TR_WAIT(acc, expr)              \
+  {                                     \
+    const long long c0__ = clock64();   \
+    expr;                               \
+    acc += clock64() - c0__;            \
+  }
+#else
+#define TR_WAIT(acc, expr) expr;
+#endif
       auto wait_k = [&](int j) {
-        ptx::mbar_wait(&kfull[j % WS_NSK], (uint32_t)((j / WS_NSK) & 1));
+        TR_WAIT(tr_wk, ptx::mbar_wait(&kfull[j % WS_NSK], (uint32_t)((j / WS_NSK) & 1)));
         ptx::tc_fence_after();
       };
-      ptx::mbar_wait(q_full, 0);
+      TR_WAIT(tr_wq, ptx::mbar_wait(q_full, 0));
       ptx::tc_fence_after();
       wait_k(0);
       issue_s(0, 0);
@@ -299,10 +324,10 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 #pragma unroll 1
       for (int j = 0; j < n_kt; ++j) {
         const int s = j % WS_NSV;
-        ptx::mbar_wait(&vfull[s], (uint32_t)((j / WS_NSV) & 1));
+        TR_WAIT(tr_wv, ptx::mbar_wait(&vfull[s], (uint32_t)((j / WS_NSV) & 1)));
         bool k_next = false;
         if (j < nA) {
-          ptx::mbar_wait(&pfull[0], (uint32_t)(j & 1));
+          TR_WAIT(tr_wp, ptx::mbar_wait(&pfull[0], (uint32_t)(j & 1)));
           ptx::tc_fence_after();
           issue_pv(0, j);
           if (j + 1 < nA) {
@@ -314,7 +339,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           }
         }
         if (hasB) {
-          ptx::mbar_wait(&pfull[1], (uint32_t)(j & 1));
+          TR_WAIT(tr_wp, ptx::mbar_wait(&pfull[1], (uint32_t)(j & 1)));
           ptx::tc_fence_after();
           issue_pv(1, j);
         }
@@ -329,6 +354,22 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
         }
         if (j + 1 < n_kt) ptx::umma_commit(&kempty[(j + 1) % WS_NSK]);  // every S of tile j+1 issued
       }
+#ifdef GLLM_VARIANT_TRACE
+      if (g_pf_trace) {
+        unsigned long long* rec = g_pf_trace + (size_t)(blockIdx.y * gridDim.x + blockIdx.x) * PF_TR;
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        rec[0] = tr_t0;
+        rec[1] = gtime();
+        rec[3] = smid;
+        rec[4] = tr_wq;
+        rec[5] = tr_wk;
+        rec[6] = tr_wv;
+        rec[7] = tr_wp;
+        rec[8] = n_kt;
+        rec[9] = nA + nB;
+      }
+#endif
     }
   } else if (warp >= 4) {
     // ---------------- softmax warpgroups (tile X = 0: warps 4-7, X = 1: warps 8-11)
@@ -468,6 +509,9 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem, 512);
   }
+#ifdef GLLM_VARIANT_TRACE
+  if (threadIdx.x == 0 && g_pf_trace) g_pf_trace[(size_t)(blockIdx.y * gridDim.x + blockIdx.x) * PF_TR + 2] = gtime();
+#endif
 }
 
 template <int D>
@@ -501,3 +545,14 @@ int launch_prefill_attention_ws(const AttnArgs& a, const PrefillItem* items, int
 }
 
 }  // namespace gllm
+
+#ifdef GLLM_VARIANT_TRACE
+// measurement build only: arm (n_ctas > 0) or disarm (0) the prefill trace; records of PF_TR words
+// per CTA [t_start, t_mma_end, t_end (globaltimer ns), smid, wait cycles q / k / v / p, key tiles,
+// tiles of both Q tiles]
+extern "C" GLLM_API int gllm_prefill_trace_arm(void* dev_buf) {
+  unsigned long long* p = static_cast<unsigned long long*>(dev_buf);
+  cudaMemcpyToSymbol(gllm::g_pf_trace, &p, sizeof(p));
+  return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+#endif

@@ -33,6 +33,17 @@
 namespace gllm {
 
 #ifdef GLLM_VARIANT_TRACE
+#define TR_WAIT(acc, expr)              \
+  {                                     \
+    const long long c0__ = clock64();   \
+    expr;                               \
+    acc += clock64() - c0__;            \
+  }
+#else
+#define TR_WAIT(acc, expr) expr;
+#endif
+
+#ifdef GLLM_VARIANT_TRACE
 // measurement build only (build.py --variant=trace): per-CTA timeline of the prefill kernel
 __device__ unsigned long long* g_pf_trace = nullptr;
 constexpr int PF_TR = 12;  // words per CTA record
@@ -137,6 +148,15 @@ __device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
 __device__ __forceinline__ void reg_fence(uint32_t (&r)[32]) {
 #pragma unroll
   for (int i = 0; i < 32; ++i) asm volatile("" : "+r"(r[i])::"memory");
+}
+
+// one lane of the (converged) warp: true in the elected lane
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred = 0;
+  asm volatile(
+      "{\n.reg .pred P1;\nelect.sync _|P1, 0xffffffff;\nselp.b32 %0, 1, 0, P1;\n}\n"
+      : "+r"(pred));
+  return pred != 0;
 }
 
 // D[tmem] (+)= A[tmem] . B[smem]
@@ -281,36 +301,43 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       publish(n_kt - 1);
     }
   } else if (warp == 1) {
-    // ---------------- MMA issuer
-    if (lane == 0) {
+    // ---------------- MMA issuer.  The whole warp runs the schedule (barrier waits, descriptor
+    // arithmetic: warp-uniform values the compiler keeps in uniform registers) and one elected lane
+    // issues each tcgen05 op.  Descriptors are built once per operand tile; a K step adds its
+    // constant byte offset >> 4 to the start-address field (an N = 128 MMA is 64 cycles of tensor
+    // work, so per-instruction descriptor building and re-election used to make the issue the
+    // bottleneck).
+    {
       constexpr uint32_t idesc_s = idesc_bf16(WS_ROWS, WS_KT, false);
       constexpr uint32_t idesc_o = idesc_bf16(WS_ROWS, D, true);
+      const uint64_t dq[2] = {ptx::umma_desc_sw128(sbase + L::Q), ptx::umma_desc_sw128(sbase + L::Q + L::Q_TILE)};
       auto issue_s = [&](int x, int j) {
-        const uint32_t qb = sbase + L::Q + x * L::Q_TILE;
-        const uint32_t kb = sbase + L::K + (j % WS_NSK) * L::KV_TILE;
+        const uint64_t dk = ptx::umma_desc_sw128(sbase + L::K + (j % WS_NSK) * L::KV_TILE);
+        if (elect_one()) {
 #pragma unroll
-        for (int ks = 0; ks < D / 16; ++ks)
-          ptx::umma_bf16(tmem + x * 128, ptx::umma_desc_sw128(qb + (ks / 4) * L::Q_ATOM + (ks % 4) * 32),
-                         ptx::umma_desc_sw128(kb + (ks / 4) * L::KV_ATOM + (ks % 4) * 32), idesc_s, ks > 0);
-        ptx::umma_commit(&sfull[x]);
+          for (int ks = 0; ks < D / 16; ++ks) {
+            const uint64_t oq = (uint64_t)(((ks / 4) * L::Q_ATOM + (ks % 4) * 32) >> 4);
+            const uint64_t ok = (uint64_t)(((ks / 4) * L::KV_ATOM + (ks % 4) * 32) >> 4);
+            ptx::umma_bf16(tmem + x * 128, dq[x] + oq, dk + ok, idesc_s, ks > 0);
+          }
+          ptx::umma_commit(&sfull[x]);
+        }
+        __syncwarp();
       };
       auto issue_pv = [&](int x, int j) {
-        const uint32_t vb = sbase + L::V + (j % WS_NSV) * L::KV_TILE;
+        const uint64_t dv = desc_mn(sbase + L::V + (j % WS_NSV) * L::KV_TILE, L::KV_ATOM);
+        if (elect_one()) {
 #pragma unroll
-        for (int kk = 0; kk < WS_KT / 16; ++kk)  // 16 keys = 8 TMEM columns of packed P per step
-          umma_bf16_ta(tmem + 256 + x * 128, tmem + x * 128 + kk * 8, desc_mn(vb + kk * 2048, L::KV_ATOM), idesc_o,
-                       (j > 0 || kk > 0) ? 1u : 0u);
+          for (int kk = 0; kk < WS_KT / 16; ++kk)  // 16 keys = 8 TMEM columns of packed P per step
+            umma_bf16_ta(tmem + 256 + x * 128, tmem + x * 128 + kk * 8, dv + (uint64_t)((kk * 2048) >> 4), idesc_o,
+                         (j > 0 || kk > 0) ? 1u : 0u);
+        }
+        __syncwarp();
       };
-#ifdef GLLM_VARIANT_TRACE
-#define TR_WAIT(acc, expr)              \
-  {                                     \
-    const long long c0__ = clock64();   \
-    expr;                               \
-    acc += clock64() - c0__;            \
-  }
-#else
-#define TR_WAIT(acc, expr) expr;
-#endif
+      auto commit = [&](uint64_t* bar) {
+        if (elect_one()) ptx::umma_commit(bar);
+        __syncwarp();
+      };
       auto wait_k = [&](int j) {
         TR_WAIT(tr_wk, ptx::mbar_wait(&kfull[j % WS_NSK], (uint32_t)((j / WS_NSK) & 1)));
         ptx::tc_fence_after();
@@ -320,7 +347,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       wait_k(0);
       issue_s(0, 0);
       if (hasB) issue_s(1, 0);
-      ptx::umma_commit(&kempty[0]);  // K(0) is read by S_A(0), S_B(0) only
+      commit(&kempty[0]);  // K(0) is read by S_A(0), S_B(0) only
 #pragma unroll 1
       for (int j = 0; j < n_kt; ++j) {
         const int s = j % WS_NSV;
@@ -335,7 +362,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
             k_next = true;
             issue_s(0, j + 1);
           } else {
-            ptx::umma_commit(&ofull[0]);
+            commit(&ofull[0]);
           }
         }
         if (hasB) {
@@ -343,19 +370,19 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           ptx::tc_fence_after();
           issue_pv(1, j);
         }
-        ptx::umma_commit(&vempty[s]);  // V(j) free once the PVs issued so far complete
+        commit(&vempty[s]);  // V(j) free once the PVs issued so far complete
         if (hasB) {
           if (j + 1 < nB) {
             if (!k_next) wait_k(j + 1);
             issue_s(1, j + 1);
           } else {
-            ptx::umma_commit(&ofull[1]);
+            commit(&ofull[1]);
           }
         }
-        if (j + 1 < n_kt) ptx::umma_commit(&kempty[(j + 1) % WS_NSK]);  // every S of tile j+1 issued
+        if (j + 1 < n_kt) commit(&kempty[(j + 1) % WS_NSK]);  // every S of tile j+1 issued
       }
 #ifdef GLLM_VARIANT_TRACE
-      if (g_pf_trace) {
+      if (lane == 0 && g_pf_trace) {
         unsigned long long* rec = g_pf_trace + (size_t)(blockIdx.y * gridDim.x + blockIdx.x) * PF_TR;
         unsigned smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));

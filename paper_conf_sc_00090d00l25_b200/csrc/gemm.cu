@@ -108,13 +108,53 @@ __device__ __forceinline__ float4 ld_dsmem_v4(uint32_t addr) {
                : "memory");
   return v;
 }
-// cluster split-K: each CTA's fp32 partial tile [128 rows][256 cols] in its own SMEM, row stride 260
-// floats (conflict-free 16-byte accesses when thread = row)
-constexpr int CL_STRIDE = GEMM_BN + 4;
+#ifdef GLLM_VARIANT_TRACE
+// measurement build only (build.py --variant=trace): per-CTA phase stamps of the GEMM (globaltimer ns)
+__device__ unsigned long long* g_gm_trace = nullptr;
+constexpr int GM_TR = 10;  // words per CTA: 0 entry, 1 setup done, 2 last MMA issued, 3 accumulator ready
+                           // (epilogue warp 4), 4 partial in SMEM / first tile drained, 5 cluster sync,
+                           // 6 reduce + epilogue done, 7 exit, 8 smid
+__device__ __forceinline__ void gm_stamp(int i) {
+  if (g_gm_trace) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_gm_trace[(size_t)blockIdx.x * GM_TR + i] = t;
+  }
+}
+#define GM_STAMP(i) gm_stamp(i)
+#else
+#define GM_STAMP(i) \
+  do {              \
+  } while (0)
+#endif
+// cluster split-K: each CTA's fp32 partial tile in its own SMEM as 8 planes, one per 32-column chunk:
+// plane c = [128 rows][32 floats] (16 KB contiguous), the 16-byte granules of row r XOR-swizzled by
+// r & 7 (conflict-free when thread = row).  Every CTA uses the same layout, so the reduction over the
+// cluster is an element-wise sum of whole planes: a warp reads 512 contiguous bytes of a peer's plane
+// per instruction (DSMEM wants coalesced accesses; per-row 16-byte reads ran at ~3 B/cycle).
+constexpr int CL_PLANE = 128 * 32 * 4;
+constexpr int SKC_MAX_S = 8;  // cluster split-K: at most 8 CTAs per tile (portable cluster size)
+__device__ __forceinline__ uint32_t cl_off(int row, int c, int q) {  // byte offset of granule q of (row, chunk c)
+  return (uint32_t)(c * CL_PLANE + row * 128 + ((q ^ (row & 7)) << 4));
+}
 struct ClSrc {
-  uint32_t part;  // local SMEM address of the partial tile (0: not cluster split-K)
+  uint32_t part;  // local SMEM address of the reduced planes (0: not cluster split-K)
   int S, r;       // cluster size, this CTA's rank
 };
+// The 32-column chunks of a tile whose epilogue cluster rank r runs: unit u = a chunk, or for the
+// RoPE epilogue a rotate-half pair (c, c + D/64) of one head, or for SiLU-mul a gate / up pair;
+// units are dealt round robin.
+template <int EPI>
+__device__ __forceinline__ bool cl_owns(const GemmArgs& p, int c, int S, int r) {
+  int unit = c;
+  if constexpr (EPI == EPI_QKV_ROPE) {
+    const int per_head = p.head_dim / 32;
+    unit = (c / per_head) * (per_head / 2) + (c % per_head) % (per_head / 2);
+  } else if constexpr (EPI == EPI_SILU_MUL) {
+    unit = c % (GEMM_BN / 64);
+  }
+  return unit % S == r;
+}
 
 // arrive on the leader CTA's copy of a barrier (from either CTA of the pair)
 __device__ __forceinline__ void mbar_arrive_leader(uint64_t* bar) {
@@ -275,16 +315,8 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
   const bool from_cl = cl.part != 0u;  // cluster split-K: sums of the cluster's partial tiles (DSMEM)
   // column chunks (32 wide) this CTA finishes: all, or (cluster split-K) its share of the tile's
   // epilogue units -- a chunk, or a rotate-half / gate-up chunk pair
-  auto own = [&](int c) {
-    if (!from_cl) return true;
-    int unit = c;
-    if constexpr (EPI == EPI_QKV_ROPE) {
-      const int per_head = p.head_dim / 32;
-      unit = (c / per_head) * (per_head / 2) + c % per_head;
-    }
-    return unit % cl.S == cl.r;
-  };
-  const uint32_t cl_row = cl.part + (uint32_t)((threadIdx.x & 127) * CL_STRIDE * 4);
+  auto own = [&](int c) { return !from_cl || cl_owns<EPI>(p, c, cl.S, cl.r); };
+  const int trow = threadIdx.x & 127;
   const float rs = (EPI == EPI_ADD_F32 || EPI == EPI_ARGMAX) ? 1.0f : row_scale(p, row);
   uint32_t r[32];
   auto wait_acc = [&]() {
@@ -318,23 +350,18 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
   // accumulator columns [col, col + 32) of this tile's row: from TMEM or (cluster split-K) summed
   // over the cluster's partial tiles
   auto ld = [&](int col, uint32_t(&v)[32]) {
-    if (from_cl) {  // fixed rank order: deterministic sums
-      float f[32];
+    if (from_cl) {  // the chunk's cluster sum, already reduced into this CTA's plane
 #pragma unroll
-      for (int q = 0; q < 32; ++q) f[q] = 0.f;
-      for (int src = 0; src < cl.S; ++src) {
-        const uint32_t a = mapa_u32(cl_row + col * 4, (uint32_t)src);
-#pragma unroll
-        for (int q = 0; q < 8; ++q) {
-          const float4 x = ld_dsmem_v4(a + 16 * q);
-          f[4 * q] += x.x;
-          f[4 * q + 1] += x.y;
-          f[4 * q + 2] += x.z;
-          f[4 * q + 3] += x.w;
-        }
+      for (int q = 0; q < 8; ++q) {
+        float4 x;
+        asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(x.x), "=f"(x.y), "=f"(x.z), "=f"(x.w)
+                     : "r"(cl.part + cl_off(trow, col / 32, q)));
+        v[4 * q] = __float_as_uint(x.x);
+        v[4 * q + 1] = __float_as_uint(x.y);
+        v[4 * q + 2] = __float_as_uint(x.z);
+        v[4 * q + 3] = __float_as_uint(x.w);
       }
-#pragma unroll
-      for (int q = 0; q < 32; ++q) v[q] = __float_as_uint(f[q]);
       return;
     }
     ptx::tmem_ld_32x32b_x32(tbase + col, v);
@@ -557,6 +584,7 @@ __global__ void __launch_bounds__(256, 1)
   const uint32_t rank = CG == 2 ? cluster_rank() : 0;
   const bool leader = rank == 0;
   pdl_trigger();
+  if (threadIdx.x == 0) GM_STAMP(0);
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch(&tma_a);
     ptx::tma_prefetch(&tma_b);
@@ -580,6 +608,7 @@ __global__ void __launch_bounds__(256, 1)
     __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_ptr;
+  if (threadIdx.x == 0) GM_STAMP(1);
   // A operand, residual, workspace, slots: produced by earlier kernels.  The producer thread waits
   // after issuing the dependency-free weight tiles of its first ring fill (below).
   if (warp != 0 || lane != 0) pdl_wait();
@@ -687,6 +716,7 @@ __global__ void __launch_bounds__(256, 1)
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
       }
+      GM_STAMP(2);
     }
   } else if (warp >= 4 && skc) {
     // ---------------- cluster split-K: this CTA's partial tile -> its SMEM (the operand ring is
@@ -694,9 +724,10 @@ __global__ void __launch_bounds__(256, 1)
     if (jobs.next(tile, kb0, kb1)) {
       ptx::mbar_wait(&tfull[0], 0);
       ptx::tc_fence_after();
+      if (threadIdx.x == 128) GM_STAMP(3);
       const int rl = (warp - 4) * 32 + lane;
       const uint32_t tb = tmem_base + ((uint32_t)((warp - 4) * 32) << 16);
-      float* dst = reinterpret_cast<float*>(sA) + rl * CL_STRIDE;
+      const uint32_t part = ptx::smem_u32(sA);
       uint32_t r[32];
 #pragma unroll 1
       for (int c = 0; c < GEMM_BN / 32; ++c) {
@@ -704,10 +735,11 @@ __global__ void __launch_bounds__(256, 1)
         ptx::tmem_ld_wait();
 #pragma unroll
         for (int q = 0; q < 8; ++q)
-          *reinterpret_cast<float4*>(dst + c * 32 + 4 * q) =
-              make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]), __uint_as_float(r[4 * q + 2]),
-                          __uint_as_float(r[4 * q + 3]));
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(part + cl_off(rl, c, q)), "r"(r[4 * q]),
+                       "r"(r[4 * q + 1]), "r"(r[4 * q + 2]), "r"(r[4 * q + 3])
+                       : "memory");
       }
+      if (threadIdx.x == 128) GM_STAMP(4);
     }
   } else if (warp >= 4) {
     // ---------------- epilogue warps (each CTA drains its own 128 rows)
@@ -719,6 +751,7 @@ __global__ void __launch_bounds__(256, 1)
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
       epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != jobs.nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
+      if (threadIdx.x == 128) GM_STAMP(4);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) {
@@ -736,6 +769,46 @@ __global__ void __launch_bounds__(256, 1)
     // chunks over DSMEM (rank order) and runs the epilogue; the second cluster barrier keeps every
     // CTA's SMEM alive until the last remote read
     cluster_sync_all();
+    if (threadIdx.x == 128) GM_STAMP(5);
+    {
+      // sum this CTA's planes over the cluster (rank order 0..S-1: deterministic), coalesced, all 8
+      // warps: thread t adds granules t, t + 256, t + 512, t + 768 of each owned plane, every
+      // source's load in flight before the first add (DSMEM round trips are ~200+ cycles), and
+      // writes the sum back into its own plane for the row-per-thread epilogue
+      const uint32_t part = ptx::smem_u32(sA);
+      const int S = p.split_s, my = (int)cluster_rank();
+      Jobs ej;
+      ej.init(p, blockIdx.x, gridDim.x, num_m);
+      if (ej.next(tile, kb0, kb1)) {
+#pragma unroll 1
+        for (int c = 0; c < GEMM_BN / 32; ++c) {
+          if (!cl_owns<EPI>(p, c, S, my)) continue;
+          const uint32_t a0 = part + c * CL_PLANE + threadIdx.x * 16;
+          float4 x[4][SKC_MAX_S];
+#pragma unroll
+          for (int src = 0; src < SKC_MAX_S; ++src)
+            if (src < S)
+#pragma unroll
+              for (int g = 0; g < 4; ++g) x[g][src] = ld_dsmem_v4(mapa_u32(a0 + g * 4096, (uint32_t)src));
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            float4 acc = x[g][0];
+#pragma unroll
+            for (int src = 1; src < SKC_MAX_S; ++src)
+              if (src < S) {
+                acc.x += x[g][src].x;
+                acc.y += x[g][src].y;
+                acc.z += x[g][src].z;
+                acc.w += x[g][src].w;
+              }
+            asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a0 + g * 4096), "f"(acc.x), "f"(acc.y),
+                         "f"(acc.z), "f"(acc.w)
+                         : "memory");
+          }
+        }
+      }
+      __syncthreads();  // planes complete
+    }
     if (warp >= 4) {
       Jobs ej;
       ej.init(p, blockIdx.x, gridDim.x, num_m);
@@ -746,6 +819,7 @@ __global__ void __launch_bounds__(256, 1)
         epilogue_tile<EPI>(p, tmem_base + ((uint32_t)(ew * 32) << 16), row, n_blk, false, &tfull[0], 0,
                            stg + ew * C::STG_FLOATS, ClSrc{ptx::smem_u32(sA), p.split_s, (int)cluster_rank()});
       }
+      if (threadIdx.x == 128) GM_STAMP(6);
     }
     ptx::tc_fence_before();
     cluster_sync_all();
@@ -760,6 +834,14 @@ __global__ void __launch_bounds__(256, 1)
     ptx::tc_fence_after();
     tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
   }
+#ifdef GLLM_VARIANT_TRACE
+  if (threadIdx.x == 0 && g_gm_trace) {
+    GM_STAMP(7);
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    g_gm_trace[(size_t)blockIdx.x * GM_TR + 8] = smid;
+  }
+#endif
 }
 
 // Workspace mode: apply the non-additive epilogue to the fp32 sums in ws [M, N].
@@ -979,8 +1061,11 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
   } else if (args.streamk == 2) {
     grid = (num_sms / CG) * CG;
   } else {
-    const int units = num_sms / CG;
-    grid = (ntiles < units ? ntiles : units) * CG;
+    // whole tiles, persistent: as few units as keep the wave count (C4's gate_up at T = 128: 224
+    // tiles -> 112 CTAs x 2 instead of 148 CTAs of which 76 take a second tile alone at the per-SM
+    // TMA rate); a wave-quantised makespan is the same either way when the tiles are tensor-bound
+    const int units = num_sms / CG, waves = (ntiles + units - 1) / units;
+    grid = ((ntiles + waves - 1) / waves) * CG;
   }
   if (grid <= 0) return GLLM_OK;
   {
@@ -1052,3 +1137,12 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
 }
 
 }  // namespace gllm
+
+#ifdef GLLM_VARIANT_TRACE
+// measurement build only: arm (a device buffer of GM_TR words per CTA) or disarm (nullptr) the GEMM trace
+extern "C" GLLM_API int gllm_gemm_trace_arm(void* dev_buf) {
+  unsigned long long* p = static_cast<unsigned long long*>(dev_buf);
+  cudaMemcpyToSymbol(gllm::g_gm_trace, &p, sizeof(p));
+  return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+#endif

@@ -62,6 +62,44 @@ __global__ void kern(const __grid_constant__ CUtensorMap tm, const uint8_t* base
   sink[blockIdx.x] = acc;
 }
 
+// mode 2: 3-D boxes {64, rows, KP k-blocks} (KP x 128 B contiguous per weight row per request), 96 KB
+// stages, 2 in flight (the same bytes in flight as 4 x 48 KB); tile = 768 / KP rows
+template <int KP>
+__global__ void kern_kp(const __grid_constant__ CUtensorMap tm, int n_tiles, int nk, int ksplit, float* sink) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  __shared__ __align__(8) uint64_t bar[2];
+  constexpr int ROWS = 768 / KP, STAGE = 98304, BOXR = ROWS > 256 ? ROWS / 2 : ROWS;
+  const int tile = blockIdx.x / ksplit, part = blockIdx.x % ksplit;
+  const int nkp = nk / KP;
+  const int kp0 = part * nkp / ksplit, kp1 = (part + 1) * nkp / ksplit;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < 2; ++s) asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_u32(&bar[s])));
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  auto issue = [&](int i) {
+    const int s = i % 2, kb = (kp0 + i) * KP;
+    uint8_t* dst = sm + s * STAGE;
+    asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(smem_u32(&bar[s])), "r"(STAGE));
+    for (int q = 0; q < ROWS / BOXR; ++q)
+      asm volatile(
+          "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(
+              smem_u32(dst + q * BOXR * KP * 128)),
+          "l"(&tm), "r"(smem_u32(&bar[s])), "r"(0), "r"(tile * ROWS + q * BOXR), "r"(kb)
+          : "memory");
+  };
+  const int n = kp1 - kp0;
+  for (int i = 0; i < 2 && i < n; ++i) issue(i);
+  float acc = 0.f;
+  for (int i = 0; i < n; ++i) {
+    bar_wait(&bar[i % 2], (i / 2) & 1);
+    acc += *reinterpret_cast<const float*>(sm + (i % 2) * STAGE);
+    if (i + 2 < n) issue(i + 2);
+  }
+  sink[blockIdx.x] = acc;
+}
+
 int main() {
   PFN_cuTensorMapEncodeTiled_v12000 enc;
   cudaDriverEntryPointQueryResult q;
@@ -101,6 +139,37 @@ int main() {
         const double moved = (double)n_tiles * 384 * sh.K * 2;
         printf("{\"shape\": \"%s\", \"mode\": \"%s\", \"ksplit\": %d, \"ctas\": %d, \"us\": %.1f, \"GBps\": %.0f}\n", sh.name,
                mode ? "bulk1d" : "tma2d", ks, grid, ms * 1e3 / R, moved * R / (ms * 1e-3) / 1e9);
+      }
+    }
+    for (int KP : {2, 4}) {
+      CUtensorMap t3;
+      const int ROWS = 768 / KP, BOXR = ROWS > 256 ? ROWS / 2 : ROWS;
+      cuuint64_t d3[3] = {64, (cuuint64_t)sh.N, (cuuint64_t)sh.K / 64};
+      cuuint64_t s3[2] = {(cuuint64_t)sh.K * 2, 128};
+      cuuint32_t b3[3] = {64, (cuuint32_t)BOXR, (cuuint32_t)KP}, e3[3] = {1, 1, 1};
+      CUresult rr = enc(&t3, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, w, d3, s3, b3, e3, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (rr != CUDA_SUCCESS) { printf("# 3d map failed %d\n", (int)rr); continue; }
+      auto kfn = KP == 2 ? kern_kp<2> : kern_kp<4>;
+      cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * 98304);
+      const int n_tiles = sh.N / ROWS, nk = sh.K / 64;
+      for (int ks : {1, 2, 3, 4}) {
+        const int grid = n_tiles * ks;
+        if (grid > 296) continue;
+        cudaEvent_t a, b;
+        cudaEventCreate(&a);
+        cudaEventCreate(&b);
+        kfn<<<grid, 32, 2 * 98304>>>(t3, n_tiles, nk, ks, sink);
+        cudaEventRecord(a);
+        const int R = 5;
+        for (int r = 0; r < R; ++r) kfn<<<grid, 32, 2 * 98304>>>(t3, n_tiles, nk, ks, sink);
+        cudaEventRecord(b);
+        cudaEventSynchronize(b);
+        float ms;
+        cudaEventElapsedTime(&ms, a, b);
+        const double moved = (double)n_tiles * ROWS * sh.K * 2;
+        printf("{\"shape\": \"%s\", \"mode\": \"tma3d_kp%d\", \"ksplit\": %d, \"ctas\": %d, \"us\": %.1f, \"GBps\": %.0f}\n",
+               sh.name, KP, ks, grid, ms * 1e3 / R, moved * R / (ms * 1e-3) / 1e9);
       }
     }
     cudaFree(w);

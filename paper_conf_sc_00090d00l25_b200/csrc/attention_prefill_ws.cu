@@ -218,7 +218,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
   const int32_t* bt = a.block_table + (size_t)it.seq * a.maxblk;
 
   if (tid == 0) {
-    ptx::mbar_init(q_full, 2 * WS_ROWS);
+    ptx::mbar_init(q_full, 8);  // one arrive per softmax warp
     for (int s = 0; s < WS_NSK; ++s) {
       ptx::mbar_init(&kfull[s], 1);
       ptx::mbar_init(&kempty[s], 1);
@@ -229,7 +229,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     }
     for (int x = 0; x < 2; ++x) {
       ptx::mbar_init(&sfull[x], 1);
-      ptx::mbar_init(&pfull[x], WS_ROWS);
+      ptx::mbar_init(&pfull[x], 4);  // one arrive per softmax warp
       ptx::mbar_init(&ofull[x], 1);
     }
     ptx::fence_barrier_init();
@@ -415,7 +415,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::cp_async_commit();
       ptx::cp_async_wait<0>();
       fence_proxy_async_smem();
-      ptx::mbar_arrive(q_full);
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(q_full);
     }
     const int nx = x == 0 ? nA : nB;
     const int pos = s0 + rrc / G;  // this row's causal limit (keys 0..pos)
@@ -502,7 +503,8 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       l += la + lb;
       tmem_st_wait();
       ptx::tc_fence_before();
-      ptx::mbar_arrive(&pfull[x]);
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&pfull[x]);
     }
     if (nx > 0) {
       ptx::mbar_wait(&ofull[x], 0);

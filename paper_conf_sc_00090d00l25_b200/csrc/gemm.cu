@@ -111,9 +111,11 @@ __device__ __forceinline__ float4 ld_dsmem_v4(uint32_t addr) {
 #ifdef GLLM_VARIANT_TRACE
 // measurement build only (build.py --variant=trace): per-CTA phase stamps of the GEMM (globaltimer ns)
 __device__ unsigned long long* g_gm_trace = nullptr;
-constexpr int GM_TR = 10;  // words per CTA: 0 entry, 1 setup done, 2 last MMA issued, 3 accumulator ready
+constexpr int GM_TR = 48;  // words per CTA: 0 entry, 1 setup done, 2 last MMA issued, 3 accumulator ready
                            // (epilogue warp 4), 4 partial in SMEM / first tile drained, 5 cluster sync,
-                           // 6 reduce + epilogue done, 7 exit, 8 smid
+                           // 6 reduce + epilogue done, 7 exit, 8 smid, 9 first operand stage landed
+                           // (MMA issuer), 10 + 2j / 11 + 2j: tile j's accumulator ready / drained
+                           // (epilogue warp 4, j < 16)
 __device__ __forceinline__ void gm_stamp(int i) {
   if (g_gm_trace) {
     unsigned long long t;
@@ -122,7 +124,12 @@ __device__ __forceinline__ void gm_stamp(int i) {
   }
 }
 #define GM_STAMP(i) gm_stamp(i)
+#define GM_STAMP_TILE(j, w) \
+  if ((j) < 16) gm_stamp(10 + 2 * (j) + (w))
 #else
+#define GM_STAMP_TILE(j, w) \
+  do {                      \
+  } while (0)
 #define GM_STAMP(i) \
   do {              \
   } while (0)
@@ -689,6 +696,9 @@ __global__ void __launch_bounds__(256, 1)
         for (int kb = kb0; kb < kb1; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
+#ifdef GLLM_VARIANT_TRACE
+          if (kb == kb0 && acc == 0 && acc_phase == 0) GM_STAMP(9);
+#endif
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
@@ -746,12 +756,24 @@ __global__ void __launch_bounds__(256, 1)
     const int ew = warp - 4;
     int acc = 0;
     uint32_t acc_phase = 0;
+    int ntile = 0;
     while (jobs.next(tile, kb0, kb1)) {
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
+#ifdef GLLM_VARIANT_TRACE
+      if (threadIdx.x == 128) {
+        ptx::mbar_wait(&tfull[acc], acc_phase);
+        GM_STAMP_TILE(ntile, 0);
+      }
+      __syncwarp();
+#endif
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
       epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != jobs.nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
-      if (threadIdx.x == 128) GM_STAMP(4);
+      if (threadIdx.x == 128) {
+        GM_STAMP(4);
+        GM_STAMP_TILE(ntile, 1);
+      }
+      ++ntile;
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) {

@@ -20,8 +20,8 @@ from paper_conf_sc_00090d00l25_b200 import gllm  # noqa: E402
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from gemm_bench import flush_read  # noqa: E402
 
-GM_TR = 10
-NAMES = ["entry", "setup", "mma_issued", "acc_ready", "drained", "cl_sync", "reduced", "exit"]
+GM_TR = 48
+NAMES = ["entry", "setup", "mma_issued", "acc_ready", "drained", "cl_sync", "reduced", "exit", None, "first_stage"]
 
 
 def main():
@@ -33,7 +33,7 @@ def main():
     s = torch.cuda.current_stream().cuda_stream
     for _ in range(3):
         gllm.op_gemm(A.data_ptr(), W.data_ptr(), M, N, K, epi, out.data_ptr(), 0, s)
-    buf = torch.zeros(GM_TR * 1024, dtype=torch.int64, device="cuda")
+    buf = torch.zeros(GM_TR * 4096, dtype=torch.int64, device="cuda")
     L = gllm.lib()
     L.gllm_gemm_trace_arm.argtypes = [C.c_void_p]
     res = []
@@ -49,10 +49,21 @@ def main():
         t0 = r[:, 0].min()
         row = {"rep": rep, "ctas": len(r), "span_us": round((r[:, 7].max() - t0) / 1e3, 2)}
         for i, nm in enumerate(NAMES):
+            if nm is None:
+                continue
             v = r[:, i]
             v = v[v > 0]
             if len(v):
                 row[nm] = [round((v.mean() - t0) / 1e3, 2), round((v.max() - t0) / 1e3, 2)]
+        # per tile j of a CTA: accumulator ready / drained (mean, max over CTAs that ran tile j)
+        tiles = []
+        for j in range(16):
+            a, d = r[:, 10 + 2 * j], r[:, 11 + 2 * j]
+            if (a > 0).sum() == 0:
+                break
+            tiles.append([int((a > 0).sum()), round((a[a > 0].mean() - t0) / 1e3, 2), round((d[d > 0].mean() - t0) / 1e3, 2),
+                          round((d[d > 0].max() - t0) / 1e3, 2)])
+        row["tiles"] = tiles
         res.append(row)
         print(json.dumps(row), flush=True)
 

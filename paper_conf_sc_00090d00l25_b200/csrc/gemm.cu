@@ -38,8 +38,13 @@ namespace {
 
 constexpr int TMEM_COLS = 2 * GEMM_BN;
 
-template <int CG>
+// The CTA-pair residual-add kernel (RES) stages the residual through shared memory: RES_BUFS x
+// chunks of [128 rows][32 fp32] (16 KB, 128-byte swizzle) loaded by TMA ahead of the accumulator,
+// updated in place and stored back by TMA with bf16(x) from XB_BUFS [128][32] bf16 buffers (8 KB,
+// 64-byte swizzle).  Its operand ring is one stage shorter to make room.
+template <int CG, int EPI>
 struct Cfg {
+  static constexpr bool RES = CG == 2 && EPI == EPI_ADD_F32;
   static constexpr int B_ROWS = GEMM_BN / CG;  // rows of the B tile loaded by each CTA
   static constexpr int A_BYTES = GEMM_BM * GEMM_BK * 2;
   static constexpr int B_BYTES = B_ROWS * GEMM_BK * 2;
@@ -47,10 +52,15 @@ struct Cfg {
 #ifdef GLLM_VARIANT_LOWSMEM  // measurement build: leave room for a co-resident attention CTA
   static constexpr int STAGES = CG == 2 ? 4 : 3;
 #else
-  static constexpr int STAGES = CG == 2 ? 6 : GEMM_STAGES;
+  static constexpr int STAGES = RES ? 5 : (CG == 2 ? 6 : GEMM_STAGES);
 #endif
+  static constexpr int RES_BUFS = RES ? 3 : 0, RES_BYTES = GEMM_BM * 32 * 4;
+  static constexpr int XB_BUFS = RES ? 2 : 0, XB_BYTES = GEMM_BM * 32 * 2;
+  static constexpr int RES_OFF = STAGES * STAGE_BYTES;                 // after the operand ring
+  static constexpr int BAR_OFF = RES_OFF + RES_BUFS * RES_BYTES + XB_BUFS * XB_BYTES;
   static constexpr int STG_FLOATS = 32 * 36;  // per epilogue warp: 32 x 32 transpose tile (row stride 36)
-  static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 + 256 + 4 * STG_FLOATS * 4;
+  static constexpr int STG_BYTES = RES ? 0 : 4 * STG_FLOATS * 4;
+  static constexpr int SMEM_BYTES = BAR_OFF + 1024 + 256 + STG_BYTES;
   static constexpr int TILE_M = GEMM_BM * CG;  // rows of one (cluster) tile
 };
 
@@ -569,21 +579,112 @@ __device__ __forceinline__ void epilogue_tile(const GemmArgs& p, uint32_t tbase,
   }
 }
 
+// Residual add of one whole tile through shared memory (CTA-pair kernel, EPI_ADD_F32): this
+// CTA's 128 rows x the tile's 32-column chunks.  Thread = row (TMEM lane).  Per chunk: the
+// accumulator columns from TMEM, the residual chunk from its TMA-loaded buffer (loaded ahead by
+// the residual loader warp while the MMAs ran), x += acc written back in place, bf16(x) into an XB
+// buffer; one elected thread TMA-stores both chunks and hands the residual buffer back to the
+// loader once the store has read it.  The row's sum of squares accumulates in a register.
+template <int EPI, int CG>
+__device__ __forceinline__ void res_epilogue_tile(const GemmArgs& p, const CUtensorMap* tmx, const CUtensorMap* tmxb,
+                                                  uint32_t tbase, int row_base, int n_blk, uint64_t* tfull_bar,
+                                                  uint32_t parity, uint32_t res_s, uint32_t xb_s, uint64_t* res_full,
+                                                  uint64_t* res_empty, int& rc, int& xc) {
+  using C = Cfg<CG, EPI>;
+  const int t = threadIdx.x - 128;  // row of the CTA's 128 (epilogue warps 4-7)
+  const int row = row_base + t;
+  const bool issuer = t == 0;
+  const int nch = min(GEMM_BN, p.N - n_blk * GEMM_BN) / 32;
+  float ss = 0.f;
+  uint32_t r[32];
+  ptx::mbar_wait(tfull_bar, parity);
+  ptx::tc_fence_after();
+  int prev_buf = -1;
+#pragma unroll 1
+  for (int c = 0; c < nch; ++c) {
+    const int buf = rc % C::RES_BUFS;
+    ptx::tmem_ld_32x32b_x32(tbase + c * 32, r);
+    ptx::mbar_wait(&res_full[buf], (uint32_t)((rc / C::RES_BUFS) & 1));
+    ptx::tmem_ld_wait();
+    const uint32_t xs = res_s + buf * C::RES_BYTES + t * 128;
+    float x[32];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t a = xs + ((q ^ (t & 7)) << 4);
+      asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                   : "=f"(x[4 * q]), "=f"(x[4 * q + 1]), "=f"(x[4 * q + 2]), "=f"(x[4 * q + 3])
+                   : "r"(a));
+    }
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+      x[j] += __uint_as_float(r[j]);
+      ss = fmaf(x[j], x[j], ss);
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t a = xs + ((q ^ (t & 7)) << 4);
+      asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(x[4 * q]), "f"(x[4 * q + 1]),
+                   "f"(x[4 * q + 2]), "f"(x[4 * q + 3])
+                   : "memory");
+    }
+    const int col0 = n_blk * GEMM_BN + c * 32;
+    if (p.out_peer != nullptr && row < p.M) {  // fused stage hand-off: the new rows to the peer slot too
+      float4* d = reinterpret_cast<float4*>(p.out_peer + (size_t)row * p.ldo + col0);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) d[q] = make_float4(x[4 * q], x[4 * q + 1], x[4 * q + 2], x[4 * q + 3]);
+    }
+    const uint32_t xbs = xb_s + (xc % C::XB_BUFS) * C::XB_BYTES;
+    if (p.xb_out != nullptr) {
+      ptx::named_bar_sync(1, 128);  // the store that last read this XB buffer has finished reading it
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t a = xbs + t * 64 + ((u ^ ((t >> 1) & 3)) << 4);
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(ptx::pack_bf16(x[8 * u], x[8 * u + 1])),
+                     "r"(ptx::pack_bf16(x[8 * u + 2], x[8 * u + 3])), "r"(ptx::pack_bf16(x[8 * u + 4], x[8 * u + 5])),
+                     "r"(ptx::pack_bf16(x[8 * u + 6], x[8 * u + 7]))
+                     : "memory");
+      }
+    }
+    ptx::fence_proxy_async_smem();
+    ptx::named_bar_sync(1, 128);
+    if (issuer) {
+      ptx::tma_store_2d(tmx, res_s + buf * C::RES_BYTES, col0, row_base);
+      if (p.xb_out != nullptr) ptx::tma_store_2d(tmxb, xbs, col0, row_base);
+      ptx::bulk_commit();
+      ptx::bulk_wait_read<1>();  // the previous chunk's stores have read their buffers
+      if (prev_buf >= 0) ptx::mbar_arrive(&res_empty[prev_buf]);
+    }
+    prev_buf = buf;
+    ++rc;
+    ++xc;
+  }
+  if (issuer && prev_buf >= 0) {
+    ptx::bulk_wait_read<0>();
+    ptx::mbar_arrive(&res_empty[prev_buf]);
+  }
+  if (p.ss_out != nullptr && row < p.M && nch > 0) atomicAdd(p.ss_out + row, ss);
+}
+
 template <int EPI, int CG>
 __global__ void __launch_bounds__(256, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tma_a, const __grid_constant__ CUtensorMap tma_b,
+                   const __grid_constant__ CUtensorMap tma_x, const __grid_constant__ CUtensorMap tma_xb,
                    const GemmArgs p) {
-  using C = Cfg<CG>;
+  using C = Cfg<CG, EPI>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::BAR_OFF);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(tempty + 2);
-  float* stg = reinterpret_cast<float*>(sB + C::STAGES * C::B_BYTES + 256);  // epilogue transpose tiles
+  uint64_t* res_full = tempty + 2;  // RES: residual chunk buffers loaded / free
+  uint64_t* res_empty = res_full + C::RES_BUFS;
+  uint32_t* tmem_ptr = reinterpret_cast<uint32_t*>(res_empty + C::RES_BUFS);
+  float* stg = reinterpret_cast<float*>(smem + C::BAR_OFF + 256);  // epilogue transpose tiles
+  const uint32_t res_s = ptx::smem_u32(smem + C::RES_OFF);
+  const uint32_t xb_s = res_s + C::RES_BUFS * C::RES_BYTES;
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -596,6 +697,12 @@ __global__ void __launch_bounds__(256, 1)
     ptx::tma_prefetch(&tma_a);
     ptx::tma_prefetch(&tma_b);
   }
+  if constexpr (C::RES) {
+    if (warp == 3 && lane == 0) {
+      ptx::tma_prefetch(&tma_x);
+      if (p.xb_out) ptx::tma_prefetch(&tma_xb);
+    }
+  }
   if (warp == 1 && lane == 0) {
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
@@ -604,6 +711,10 @@ __global__ void __launch_bounds__(256, 1)
     for (int s = 0; s < 2; ++s) {
       ptx::mbar_init(&tfull[s], 1);
       ptx::mbar_init(&tempty[s], 4 * CG);  // every epilogue warp of the pair releases the leader's buffer
+    }
+    for (int s = 0; s < C::RES_BUFS; ++s) {
+      ptx::mbar_init(&res_full[s], 1);
+      ptx::mbar_init(&res_empty[s], 1);
     }
     ptx::fence_barrier_init();
   }
@@ -728,6 +839,24 @@ __global__ void __launch_bounds__(256, 1)
       }
       GM_STAMP(2);
     }
+  } else if (C::RES && warp == 3) {
+    // ---------------- residual loader (RES): x chunks of this CTA's whole tiles, RES_BUFS ahead
+    if (lane == 0) {
+      int rc = 0;
+      while (jobs.next(tile, kb0, kb1)) {
+        if (kb0 != 0 || kb1 != jobs.nk) continue;  // partial tiles reduce into x with vector atomics
+        const int m_blk = tile % num_m, n_blk = tile / num_m;
+        const int row_base = m_blk * C::TILE_M + rank * GEMM_BM;
+        const int nch = min(GEMM_BN, p.N - n_blk * GEMM_BN) / 32;
+        for (int c = 0; c < nch; ++c, ++rc) {
+          const int buf = rc % C::RES_BUFS;
+          if (rc >= C::RES_BUFS) ptx::mbar_wait(&res_empty[buf], (uint32_t)(((rc / C::RES_BUFS) - 1) & 1));
+          ptx::mbar_arrive_expect_tx(&res_full[buf], C::RES_BYTES);
+          ptx::tma_load_2d(smem + C::RES_OFF + buf * C::RES_BYTES, &tma_x, &res_full[buf], n_blk * GEMM_BN + c * 32,
+                           row_base);
+        }
+      }
+    }
   } else if (warp >= 4 && skc) {
     // ---------------- cluster split-K: this CTA's partial tile -> its SMEM (the operand ring is
     // idle: every stage was consumed by the MMAs the tfull commit covers)
@@ -757,6 +886,7 @@ __global__ void __launch_bounds__(256, 1)
     int acc = 0;
     uint32_t acc_phase = 0;
     int ntile = 0;
+    int res_rc = 0, res_xc = 0;  // RES: residual / bf16 chunk buffers consumed so far
     while (jobs.next(tile, kb0, kb1)) {
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
@@ -768,7 +898,16 @@ __global__ void __launch_bounds__(256, 1)
       __syncwarp();
 #endif
       const uint32_t tbase = tmem_base + ((uint32_t)(ew * 32) << 16) + acc * GEMM_BN;
-      epilogue_tile<EPI>(p, tbase, row, n_blk, kb0 != 0 || kb1 != jobs.nk, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
+      const bool partial = kb0 != 0 || kb1 != jobs.nk;
+      if constexpr (C::RES) {
+        if (!partial)
+          res_epilogue_tile<EPI, CG>(p, &tma_x, &tma_xb, tbase, m_blk * C::TILE_M + rank * GEMM_BM, n_blk, &tfull[acc],
+                                     acc_phase, res_s, xb_s, res_full, res_empty, res_rc, res_xc);
+        else
+          epilogue_tile<EPI>(p, tbase, row, n_blk, true, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
+      } else {
+        epilogue_tile<EPI>(p, tbase, row, n_blk, partial, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
+      }
       if (threadIdx.x == 128) {
         GM_STAMP(4);
         GM_STAMP_TILE(ntile, 1);
@@ -784,6 +923,9 @@ __global__ void __launch_bounds__(256, 1)
       }
       acc ^= 1;
       if (acc == 0) acc_phase ^= 1;
+    }
+    if constexpr (C::RES) {
+      if (threadIdx.x == 128) ptx::bulk_wait<0>();  // the residual / bf16 stores are performed
     }
   }
   if (skc) {
@@ -1040,6 +1182,7 @@ int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t c
         q == cudaDriverEntryPointSuccess)
       g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
   });
+  if (map == nullptr) return GLLM_OK;  // entry-point resolution only (encode_2d)
   if (!g_encode) return set_error(GLLM_ECUDA, "cuTensorMapEncodeTiled unavailable");
   if ((reinterpret_cast<uintptr_t>(base) & 15) || (cols * 2) % 16)
     return set_error(GLLM_EINVAL, "tensor map: base/stride not 16-byte aligned");
@@ -1054,6 +1197,29 @@ int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t c
   return GLLM_OK;
 }
 
+static int encode_2d(CUtensorMap* map, CUtensorMapDataType dt, int esize, const void* base, uint64_t rows,
+                     uint64_t cols, uint32_t box_cols, uint32_t box_rows, CUtensorMapSwizzle sw) {
+  make_tmap_bf16(nullptr, nullptr, 0, 0, 0);  // resolves the driver entry point once
+  if (!g_encode) return set_error(GLLM_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  if ((reinterpret_cast<uintptr_t>(base) & 15) || (cols * esize) % 16)
+    return set_error(GLLM_EINVAL, "tensor map: base/stride not 16-byte aligned");
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {cols * esize};
+  cuuint32_t box[2] = {box_cols, box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = g_encode(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(GLLM_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return GLLM_OK;
+}
+
+int make_tmap_res_f32(CUtensorMap* map, const float* base, uint64_t rows, uint64_t cols) {
+  return encode_2d(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, base, rows, cols, 32, GEMM_BM, CU_TENSOR_MAP_SWIZZLE_128B);
+}
+int make_tmap_res_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols) {
+  return encode_2d(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, rows, cols, 32, GEMM_BM, CU_TENSOR_MAP_SWIZZLE_64B);
+}
+
 int num_sms_of_current_device() {
   int dev = 0, n = 0;
   cudaGetDevice(&dev);
@@ -1062,9 +1228,9 @@ int num_sms_of_current_device() {
 }
 
 template <int EPI, int CG>
-static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args, cudaStream_t stream,
-                    int num_sms) {
-  using C = Cfg<CG>;
+static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& tx, const CUtensorMap& txb,
+                    const GemmArgs& args, cudaStream_t stream, int num_sms) {
+  using C = Cfg<CG, EPI>;
   static bool attr_set = false;  // per-process; the attribute is per-function
   if (!attr_set) {
     cudaError_t e =
@@ -1092,7 +1258,8 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
   if (grid <= 0) return GLLM_OK;
   {
     const int cluster = args.streamk == 3 ? args.split_s : CG;
-    cudaError_t e = launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, cluster, a, b, args);
+    cudaError_t e =
+        launch_pdl(gemm_tc_kernel<EPI, CG>, dim3(grid), dim3(256), C::SMEM_BYTES, stream, cluster, a, b, tx, txb, args);
     if (e != cudaSuccess) return set_error(GLLM_ECUDA, "gemm (%d-CTA) launch: %s", CG, cudaGetErrorString(e));
   }
   if (args.ws) {
@@ -1105,13 +1272,14 @@ static int launch_t(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& 
 }
 
 template <int EPI>
-static int launch_e(const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args, cudaStream_t stream,
-                    int num_sms, int cg) {
-  return cg == 2 ? launch_t<EPI, 2>(a, b, args, stream, num_sms) : launch_t<EPI, 1>(a, b, args, stream, num_sms);
+static int launch_e(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& tx, const CUtensorMap& txb,
+                    const GemmArgs& args, cudaStream_t stream, int num_sms, int cg) {
+  return cg == 2 ? launch_t<EPI, 2>(a, b, tx, txb, args, stream, num_sms)
+                 : launch_t<EPI, 1>(a, b, tx, txb, args, stream, num_sms);
 }
 
 int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const GemmArgs& args0, cudaStream_t stream,
-                int num_sms) {
+                int num_sms, const CUtensorMap* tm_x, const CUtensorMap* tm_xb) {
   if (args0.K % GEMM_BK != 0 || args0.M < 0 || args0.N <= 0 || args0.N % 32)
     return set_error(GLLM_EINVAL, "gemm: K %% 64 != 0 or bad M/N (M=%d N=%d K=%d)", args0.M, args0.N, args0.K);
   if (args0.M == 0) return GLLM_OK;
@@ -1148,12 +1316,21 @@ int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const G
   } else {
     args.ws = nullptr;
   }
+  static const CUtensorMap none{};  // the epilogue maps of the other kernels (never dereferenced)
+  args.res_tma = 0;
+  if (epi == EPI_ADD_F32 && cg == 2) {  // the CTA-pair residual kernel stages x through TMA
+    if (tm_x == nullptr || (args.xb_out != nullptr && tm_xb == nullptr))
+      return set_error(GLLM_EINVAL, "gemm: residual add needs the x (and bf16 x) tensor maps");
+    args.res_tma = 1;
+  }
+  const CUtensorMap& tx = tm_x ? *tm_x : none;
+  const CUtensorMap& txb = tm_xb ? *tm_xb : none;
   switch (epi) {
-    case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, args, stream, num_sms, cg);
-    case EPI_ADD_F32: return launch_e<EPI_ADD_F32>(a, b, args, stream, num_sms, cg);
-    case EPI_SILU_MUL: return launch_e<EPI_SILU_MUL>(a, b, args, stream, num_sms, cg);
-    case EPI_ARGMAX: return launch_e<EPI_ARGMAX>(a, b, args, stream, num_sms, cg);
-    case EPI_QKV_ROPE: return launch_e<EPI_QKV_ROPE>(a, b, args, stream, num_sms, cg);
+    case EPI_STORE_BF16: return launch_e<EPI_STORE_BF16>(a, b, tx, txb, args, stream, num_sms, cg);
+    case EPI_ADD_F32: return launch_e<EPI_ADD_F32>(a, b, tx, txb, args, stream, num_sms, cg);
+    case EPI_SILU_MUL: return launch_e<EPI_SILU_MUL>(a, b, tx, txb, args, stream, num_sms, cg);
+    case EPI_ARGMAX: return launch_e<EPI_ARGMAX>(a, b, tx, txb, args, stream, num_sms, cg);
+    case EPI_QKV_ROPE: return launch_e<EPI_QKV_ROPE>(a, b, tx, txb, args, stream, num_sms, cg);
   }
   return set_error(GLLM_EINVAL, "gemm: unknown epilogue");
 }

@@ -59,6 +59,9 @@ struct GemmArgs {
   // EPI_ADD_F32, whole tiles: the updated residual rows are also stored to out_peer [M, ldo] (the
   // next pipeline stage's receive slot, NVLink peer memory) -- the fused stage hand-off (a12)
   float* out_peer;
+  // set by launch_gemm: the CTA-pair residual-add kernel stages its whole tiles' residual through
+  // shared memory with TMA (loads of x chunks ahead of the accumulator, stores of x and bf16(x))
+  int res_tma;
 };
 
 // true if launch_gemm would combine partial tiles (stream-K) for this shape -- then the ADD_F32
@@ -80,9 +83,17 @@ extern int g_force_cg;
 // (box_rows x 64) box and 128-byte swizzle.  Returns 0 or a GLLM_* error.
 int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols, uint32_t box_rows);
 
+// Residual-epilogue tensor maps (EPI_ADD_F32): x fp32 [rows, cols] with a 128-row x 32-column box
+// and 128-byte swizzle; bf16(x) [rows, cols] with a 128 x 32 box and 64-byte swizzle.
+int make_tmap_res_f32(CUtensorMap* map, const float* base, uint64_t rows, uint64_t cols);
+int make_tmap_res_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols);
+
 // Launches the persistent GEMM on `stream`.  A map: box 128 rows; B map: box 256 rows.
+// EPI_ADD_F32 needs tm_x (the residual `out`, make_tmap_res_f32) and, when xb_out is set, tm_xb
+// (make_tmap_res_bf16 of xb_out); the other epilogues ignore them.
 int launch_gemm(const CUtensorMap& a, const CUtensorMap& b, GemmEpi epi, const GemmArgs& args,
-                cudaStream_t stream, int num_sms);
+                cudaStream_t stream, int num_sms, const CUtensorMap* tm_x = nullptr,
+                const CUtensorMap* tm_xb = nullptr);
 
 int num_sms_of_current_device();
 

@@ -62,7 +62,9 @@ extern "C" int gllm_op_gemm(const void* A, const void* W, int32_t M, int32_t N, 
     g.part_idx = reinterpret_cast<int32_t*>(g.part_val + part_elems);
   }
   if (epi == gllm::EPI_ARGMAX) g.out = nullptr;
-  rc = gllm::launch_gemm(ta, tb, static_cast<gllm::GemmEpi>(epi), g, s, sms);
+  CUtensorMap tx{};
+  if (epi == gllm::EPI_ADD_F32 && (rc = gllm::make_tmap_res_f32(&tx, static_cast<const float*>(out), M, N))) return rc;
+  rc = gllm::launch_gemm(ta, tb, static_cast<gllm::GemmEpi>(epi), g, s, sms, epi == gllm::EPI_ADD_F32 ? &tx : nullptr);
   if (rc == GLLM_OK && epi == gllm::EPI_ARGMAX)
     gllm::launch_argmax_reduce(g.part_val, g.part_idx, M, ntn, static_cast<int32_t*>(out), s);
   if (tmp) cudaFreeAsync(tmp, s);

@@ -123,6 +123,10 @@ struct gllm_stage {
   float* xbuf = nullptr;
   bf16 *y = nullptr, *qkv = nullptr, *attn = nullptr, *act = nullptr, *ys = nullptr;
   CUtensorMap tm_y, tm_attn, tm_act, tm_ys;
+  CUtensorMap tm_yres;         // y as the residual epilogue's bf16(x) output (128 x 32 box)
+  CUtensorMap tm_x;            // the residual x of the current forward (fp32, 128 x 32 box)
+  const float* tm_x_base = nullptr;
+  int tm_x_rows = 0;
   float2* rope_cs = nullptr;
   int32_t* slots = nullptr;
   int32_t* sampled_tmp = nullptr;
@@ -441,7 +445,8 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   CK(cudaMemsetAsync(st->act, 0, R * I * sizeof(bf16), s0));
   if ((rc = gllm::make_tmap_bf16(&st->tm_y, st->y, R, H, gllm::GEMM_BM)) ||
       (rc = gllm::make_tmap_bf16(&st->tm_attn, st->attn, R, qd, gllm::GEMM_BM)) ||
-      (rc = gllm::make_tmap_bf16(&st->tm_act, st->act, R, I, gllm::GEMM_BM)))
+      (rc = gllm::make_tmap_bf16(&st->tm_act, st->act, R, I, gllm::GEMM_BM)) ||
+      (rc = gllm::make_tmap_res_bf16(&st->tm_yres, st->y, R, H)))
     return fail(rc);
   for (int i = 0; i < RING; ++i)
     if ((rc = new_slot(st)) < 0) return fail(rc);
@@ -693,7 +698,12 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     g.ss_out = unfused ? nullptr : ss_next;
     g.out_peer = sk ? nullptr : out_peer;  // whole tiles store the new residual rows to the peer too
     st->last_launches += 1;
-    RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms));
+    if (st->tm_x_base != x || st->tm_x_rows != T) {  // the residual's tensor map (hidden_out varies per call)
+      RC(gllm::make_tmap_res_f32(&st->tm_x, x, T, H));
+      st->tm_x_base = x;
+      st->tm_x_rows = T;
+    }
+    RC(gllm::launch_gemm(ta, tb, gllm::EPI_ADD_F32, g, s, st->num_sms, &st->tm_x, &st->tm_yres));
     if (out_peer && sk)  // partial tiles reduce in place: copy the finished residual afterwards
       CK(cudaMemcpyAsync(out_peer, x, (size_t)T * H * sizeof(float), cudaMemcpyDeviceToDevice, s));
     if (unfused) {  // rebuild bf16(x) and the row sums of squares from x

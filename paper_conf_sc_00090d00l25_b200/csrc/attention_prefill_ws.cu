@@ -143,6 +143,45 @@ __device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
   return d;
 }
 
+// three-input max (sm_100 FMNMX3): the row-max pass issues half the ALU-pipe instructions
+__device__ __forceinline__ float fmax3(float a, float b, float c) {
+  float r;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(r) : "f"(a), "f"(b), "f"(c));
+  return r;
+}
+
+// 2^x on the FMA pipe for a pair (x0, x1) packed as f32x2: round-to-nearest split x = j + f
+// (f in [-1/2, 1/2]) with the 1.5 * 2^23 shifter, 2^f by a degree-3 polynomial fitted to the
+// relative error on [-1/2, 1/2] (max 1.0e-4, below the bf16 rounding of P), 2^j added to the
+// exponent bits; x clamped at -126 so the result stays normal (~1e-38: zero next to the row's
+// 2^0 terms).
+__device__ __forceinline__ void ex2_poly2(uint64_t x2, float& y0, float& y1) {
+  float a, b;
+  f2unpack(x2, a, b);
+  a = fmaxf(a, -126.f);
+  b = fmaxf(b, -126.f);
+  const uint64_t r = fadd2(f2pack(a, b), f2pack(12582912.f, 12582912.f));  // low mantissa bits = round(x)
+  const uint64_t j = fadd2(r, f2pack(-12582912.f, -12582912.f));
+  const uint64_t f = fadd2(f2pack(a, b), j ^ 0x8000000080000000ull);  // x - round(x)
+  uint64_t p = ffma2(f, f2pack(0.05500893f, 0.05500893f), f2pack(0.24221096f, 0.24221096f));
+  p = ffma2(p, f, f2pack(0.69328293f, 0.69328293f));
+  p = ffma2(p, f, f2pack(1.f, 1.f));
+  float p0, p1, r0, r1;
+  f2unpack(p, p0, p1);
+  f2unpack(r, r0, r1);
+  y0 = __int_as_float(__float_as_int(p0) + (__float_as_int(r0) << 23));
+  y1 = __int_as_float(__float_as_int(p1) + (__float_as_int(r1) << 23));
+}
+#if defined(GLLM_VARIANT_EMU1)
+constexpr uint32_t WS_EMU_PAIRS = 0x8000u;  // A/B builds: which of the 16 pairs of a 32-score chunk
+#elif defined(GLLM_VARIANT_EMU2)
+constexpr uint32_t WS_EMU_PAIRS = 0x8080u;
+#elif defined(GLLM_VARIANT_EMU4)
+constexpr uint32_t WS_EMU_PAIRS = 0x8888u;
+#else
+constexpr uint32_t WS_EMU_PAIRS = 0u;
+#endif
+
 // Orders later uses of tcgen05.ld destination registers after the tcgen05.wait::ld that
 // precedes this call (the compiler sees no dependency between the wait and those registers).
 __device__ __forceinline__ void reg_fence(uint32_t (&r)[32]) {
@@ -447,11 +486,13 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
         for (int cq = 0; cq < WS_KT / 32; ++cq) {
           if (diag_w) {
 #pragma unroll
-            for (int i = 0; i < 32; ++i)
-              m4[i & 3] = fmaxf(m4[i & 3], kbase + cq * 32 + i > pos ? -INFINITY : __uint_as_float(sr[cq][i]));
+            for (int i = 0; i < 32; i += 2)
+              m4[(i >> 1) & 3] = fmax3(m4[(i >> 1) & 3], kbase + cq * 32 + i > pos ? -INFINITY : __uint_as_float(sr[cq][i]),
+                                       kbase + cq * 32 + i + 1 > pos ? -INFINITY : __uint_as_float(sr[cq][i + 1]));
           } else {
 #pragma unroll
-            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(sr[cq][i]));
+            for (int i = 0; i < 32; i += 2)
+              m4[(i >> 1) & 3] = fmax3(m4[(i >> 1) & 3], __uint_as_float(sr[cq][i]), __uint_as_float(sr[cq][i + 1]));
           }
         }
         mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * sl2;
@@ -487,8 +528,15 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
             float x0, x1;
-            f2unpack(ffma2(f2pack(__uint_as_float(sr[cq][2 * i]), __uint_as_float(sr[cq][2 * i + 1])), sc2, nm2), x0, x1);
-            float p0 = ex2(x0), p1 = ex2(x1);
+            const uint64_t xx = ffma2(f2pack(__uint_as_float(sr[cq][2 * i]), __uint_as_float(sr[cq][2 * i + 1])), sc2, nm2);
+            float p0, p1;
+            if ((WS_EMU_PAIRS >> i) & 1) {
+              ex2_poly2(xx, p0, p1);
+            } else {
+              f2unpack(xx, x0, x1);
+              p0 = ex2(x0);
+              p1 = ex2(x1);
+            }
             if (diag_w) {
               if (kbase + cq * 32 + 2 * i > pos) p0 = 0.f;
               if (kbase + cq * 32 + 2 * i + 1 > pos) p1 = 0.f;

@@ -21,7 +21,7 @@ from workloads.streams import make_stream  # noqa: E402
 sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from attn_bench import subset  # noqa: E402
 
-PF_TR = 12
+PF_TR = 20
 
 
 def main():
@@ -72,6 +72,12 @@ def main():
            "mma_wait_mcycles_per_cta": round(float(waits.sum() / n / 1e6), 4),
            "key_tiles_per_cta_mean": round(float(r[:, 8].mean()), 2),
            "epilogue_us_mean": round(float((end - mma_end).mean()), 2)}
+    # softmax phases (cycles per key tile, warps 4 / 8): wait for S, TMEM load, max, exp + P store + arrive
+    for x, nm in ((0, "softmax_A"), (1, "softmax_B")):
+        ph = r[:, 10 + 5 * x: 15 + 5 * x].astype(np.float64)
+        it = ph[:, 4].sum()
+        if it > 0:
+            out[nm] = {k: round(float(ph[:, i].sum() / it), 1) for i, k in enumerate(["wait_s", "tmem_ld", "max", "exp_store"])}
     print(json.dumps(out))
 
 

@@ -1129,13 +1129,16 @@ int choose_cg(int M, int N, int epi, int num_sms) {
 // Returns the whole-tile count (0 = no hybrid).  (Non-additive epilogues through the fp32 workspace
 // measured slower than whole tiles, profiles/r01/gemm_sched.txt.)
 // Returns the whole-tile count (-1 = no hybrid).  Below one wave of pair tiles that leaves more than
-// 15% of the pairs idle (C2's O / down GEMMs at T ~ 626: 60 tiles on 74 pairs), 0: every tile's
-// k-blocks are spread over all pairs (stream-K over the CTA-pair kernel).
+// 25% of the pairs idle, 0: every tile's k-blocks are spread over all pairs (stream-K over the
+// CTA-pair kernel).
 int hybrid_dp_tiles(int M, int N, int K, int epi, int cg, int num_sms) {
   if (cg != 2 || epi != EPI_ADD_F32 || K / GEMM_BK < 8) return -1;
   const int units = num_sms / 2;
   const int ntiles = ((M + 255) / 256) * ((N + GEMM_BN - 1) / GEMM_BN);
-  if (ntiles < units) return ntiles * 100 < units * 85 ? 0 : -1;
+  // one wave at >= 75% of the pairs: whole tiles (C2's O / down at T ~ 625: 60 tiles on 74 pairs,
+  // 43.0 -> 41.0 and 94.2 -> 83.9 us vs stream-K, and the fused bf16(x) / norm statistics stay on:
+  // profiles/r02/gemm_sched/gemm_c2_c3_c1_default_det_cg1.jsonl); below that every tile's k-blocks go over all pairs
+  if (ntiles < units) return ntiles * 100 < units * 75 ? 0 : -1;
   const int tail = ntiles % units;
   if (tail == 0 || tail * 10 >= units * 8) return -1;
   return ntiles - tail;
@@ -1151,7 +1154,7 @@ int skc_split(int M, int N, int K, int epi, int num_sms) {
   if (M > GEMM_BM || epi == EPI_ARGMAX || epi == EPI_ADD_F32) return 0;
   const int ntiles = (N + GEMM_BN - 1) / GEMM_BN, nk = K / GEMM_BK;
   const int cap = (epi == EPI_SILU_MUL || epi == EPI_QKV_ROPE) ? 4 : 8;
-  const int S = std::min(std::min(cap, num_sms / std::max(ntiles, 1)), nk / 4);
+  int S = std::min(std::min(cap, num_sms / std::max(ntiles, 1)), nk / 4);
   return S >= 2 ? S : 0;
 }
 

@@ -44,9 +44,10 @@ def main():
     ap.add_argument("--config", default="C1")
     ap.add_argument("--tick", type=int, default=403)
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--pp", type=int, default=1, help="scheduler pipeline depth (the stage micro-batches of PP > 1)")
     a = ap.parse_args()
     m = MODELS[a.config].with_layers(2)
-    sp = SCHED[a.config].with_(pp_depth=1, num_blocks=60000 if a.config == "C1" else SCHED[a.config].num_blocks)
+    sp = SCHED[a.config].with_(pp_depth=a.pp, num_blocks=60000 if a.config == "C1" else SCHED[a.config].num_blocks)
     s = gllm.Sched(sp)
     s.add_stream(make_stream(a.config, m.vocab))
     for _ in range(a.tick):

@@ -96,7 +96,9 @@ if __name__ == "__main__":
     ap.add_argument("--variants", default="0", help="comma list: 0 auto, 1 one-CTA, 2 CTA pair")
     ap.add_argument("--cublas", action="store_true", help="also time torch.mm (cuBLAS) per shape")
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--det", action="store_true", help="gllm_op_set_deterministic: whole tiles / cluster split-K only")
     a = ap.parse_args()
+    gllm.op_set_deterministic(a.det)
     if a.cublas:
         for key in a.shapes.split(","):
             for shp in SHAPES[key]:
@@ -105,5 +107,5 @@ if __name__ == "__main__":
         gllm.op_set_gemm_variant(v)
         for key in a.shapes.split(","):
             for shp in SHAPES[key]:
-                print(json.dumps({"variant": v, "set": key, **bench(*shp, reps=a.reps)}), flush=True)
+                print(json.dumps({"variant": v, "det": a.det, "set": key, **bench(*shp, reps=a.reps)}), flush=True)
     gllm.op_set_gemm_variant(0)

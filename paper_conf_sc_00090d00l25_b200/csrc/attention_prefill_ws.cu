@@ -46,7 +46,7 @@ namespace gllm {
 #ifdef GLLM_VARIANT_TRACE
 // measurement build only (build.py --variant=trace): per-CTA timeline of the prefill kernel
 __device__ unsigned long long* g_pf_trace = nullptr;
-constexpr int PF_TR = 12;  // words per CTA record
+constexpr int PF_TR = 20;  // words per CTA record
 __device__ __forceinline__ unsigned long long gtime() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -234,10 +234,12 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
 
   pdl_trigger();
 #ifdef GLLM_VARIANT_TRACE
-  const unsigned long long tr_t0 = gtime();
   unsigned long long tr_wq = 0, tr_wk = 0, tr_wv = 0, tr_wp = 0;
 #endif
   pdl_wait();
+#ifdef GLLM_VARIANT_TRACE
+  const unsigned long long tr_t0 = gtime();  // after the PDL wait: the kernel's own span
+#endif
   // grid (Hkv, items): CTAs are dispatched x-fastest, so every kv head of the longest item goes
   // first and the whole grid runs longest-first (the host sorts items by key tiles)
   const PrefillItem it = items[blockIdx.y];
@@ -464,10 +466,23 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
     const uint32_t t_s = tmem + lane_off + x * 128;
     const uint32_t t_o = tmem + lane_off + 256 + x * 128;
     float m_ref = -INFINITY, l = 0.f;
+#ifdef GLLM_VARIANT_TRACE
+    long long ph_w = 0, ph_ld = 0, ph_max = 0, ph_exp = 0, c_a = 0, c_b;
+#define PH(acc)    \
+  c_b = clock64(); \
+  acc += c_b - c_a; \
+  c_a = c_b;
+#else
+#define PH(acc)
+#endif
 #pragma unroll 1
     for (int j = 0; j < nx; ++j) {
+#ifdef GLLM_VARIANT_TRACE
+      c_a = clock64();
+#endif
       ptx::mbar_wait(&sfull[x], (uint32_t)(j & 1));
       ptx::tc_fence_after();
+      PH(ph_w)
       const int kbase = j * WS_KT;
       // causal masking only where some row of this warp ends inside the tile (warp-uniform, so
       // the unmasked path carries no per-element compares)
@@ -479,6 +494,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::tmem_ld_wait();
 #pragma unroll
       for (int cq = 0; cq < WS_KT / 32; ++cq) reg_fence(sr[cq]);
+      PH(ph_ld)
       float mx;
       {
         float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
@@ -515,6 +531,7 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
           tmem_st_x32(t_o + cb * 32, orr);
         }
       }
+      PH(ph_max)
       // P = exp2(s * scale - m) as bf16 pairs written over the S columns (chunk cq's P lands in
       // columns [16cq, 16cq + 16), whose scores are already in registers); the scale and the row
       // sum run as packed f32x2 FFMA2 / FADD2 (half the FMA-pipe issues)
@@ -553,7 +570,19 @@ __global__ void __launch_bounds__(WS_THREADS, 1)
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&pfull[x]);
+      PH(ph_exp)
     }
+#ifdef GLLM_VARIANT_TRACE
+    if ((warp & 3) == 0 && lane == 0 && g_pf_trace) {  // warps 4 (tile A) and 8 (tile B)
+      unsigned long long* rec = g_pf_trace + (size_t)(blockIdx.y * gridDim.x + blockIdx.x) * PF_TR + 10 + 5 * x;
+      rec[0] = ph_w;
+      rec[1] = ph_ld;
+      rec[2] = ph_max;
+      rec[3] = ph_exp;
+      rec[4] = nx;
+    }
+#endif
+#undef PH
     if (nx > 0) {
       ptx::mbar_wait(&ofull[x], 0);
       ptx::tc_fence_after();

@@ -14,8 +14,11 @@
 // Both: single-thread MMA issue, double-buffered fp32 TMEM accumulator (2 x 256 columns), 4
 // epilogue warps (tcgen05.ld) with the fused epilogues: bias, fp32 residual add, SiLU*up,
 // RoPE + paged KV append, row argmax for the greedy LM head.
-//   warp 0: TMA producer      warp 1: MMA issuer      warp 2: TMEM allocator
-//   warps 4-7: epilogue (warp 4+i reads TMEM lanes 32i..32i+31)
+//   warps 0-3: epilogue (warp i reads TMEM lanes 32i..32i+31)
+//   warp 4: TMA producer   warp 5: MMA issuer   warp 6: TMEM allocator   warp 7: residual loader
+// The single-thread producer and MMA roles sit in the higher warp ids: the SMSP arbiter issues
+// the highest eligible warp id first, so a heavy epilogue of the previous tile (on the same SMSPs)
+// does not delay the MMA issue of the next tile.
 #include <cudaTypedefs.h>
 
 #include <algorithm>
@@ -37,6 +40,7 @@ int g_force_cg = 0;
 namespace {
 
 constexpr int TMEM_COLS = 2 * GEMM_BN;
+constexpr int W_PROD = 4, W_MMA = 5, W_ALLOC = 6, W_RES = 7;  // warp roles of gemm_tc_kernel (0-3: epilogue)
 
 // The CTA-pair residual-add kernel (RES) stages the residual through shared memory: RES_BUFS x
 // chunks of [128 rows][32 fp32] (16 KB, 128-byte swizzle) loaded by TMA ahead of the accumulator,
@@ -64,7 +68,10 @@ struct Cfg {
   static constexpr int TILE_M = GEMM_BM * CG;  // rows of one (cluster) tile
 };
 
-__device__ __forceinline__ float silu_f(float x) { return x / (1.0f + __expf(-x)); }
+// x * sigmoid(x) with the approximate reciprocal (MUFU.RCP, ~1 ulp): the IEEE division it replaces
+// (reciprocal + Newton step + a range check with a slow path per element) made the SiLU epilogue of
+// a 128 x 256 tile take ~9 us, exposed after each CTA's last gate_up tile
+__device__ __forceinline__ float silu_f(float x) { return x * __frcp_rn(1.0f + __expf(-x)); }
 
 __device__ __forceinline__ uint32_t cluster_rank() {
   uint32_t r;
@@ -591,7 +598,7 @@ __device__ __forceinline__ void res_epilogue_tile(const GemmArgs& p, const CUten
                                                   uint32_t parity, uint32_t res_s, uint32_t xb_s, uint64_t* res_full,
                                                   uint64_t* res_empty, int& rc, int& xc) {
   using C = Cfg<CG, EPI>;
-  const int t = threadIdx.x - 128;  // row of the CTA's 128 (epilogue warps 4-7)
+  const int t = threadIdx.x;  // row of the CTA's 128 (epilogue warps 0-3)
   const int row = row_base + t;
   const bool issuer = t == 0;
   const int nch = min(GEMM_BN, p.N - n_blk * GEMM_BN) / 32;
@@ -693,17 +700,17 @@ __global__ void __launch_bounds__(256, 1)
   const bool leader = rank == 0;
   pdl_trigger();
   if (threadIdx.x == 0) GM_STAMP(0);
-  if (warp == 0 && lane == 0) {
+  if (warp == W_PROD && lane == 0) {
     ptx::tma_prefetch(&tma_a);
     ptx::tma_prefetch(&tma_b);
   }
   if constexpr (C::RES) {
-    if (warp == 3 && lane == 0) {
+    if (warp == W_RES && lane == 0) {
       ptx::tma_prefetch(&tma_x);
       if (p.xb_out) ptx::tma_prefetch(&tma_xb);
     }
   }
-  if (warp == 1 && lane == 0) {
+  if (warp == W_MMA && lane == 0) {
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -718,7 +725,7 @@ __global__ void __launch_bounds__(256, 1)
     }
     ptx::fence_barrier_init();
   }
-  if (warp == 2) tmem_alloc_cg<CG>(tmem_ptr, TMEM_COLS);
+  if (warp == W_ALLOC) tmem_alloc_cg<CG>(tmem_ptr, TMEM_COLS);
   ptx::tc_fence_before();
   if (CG == 2 || skc)
     cluster_sync_all();
@@ -729,14 +736,14 @@ __global__ void __launch_bounds__(256, 1)
   if (threadIdx.x == 0) GM_STAMP(1);
   // A operand, residual, workspace, slots: produced by earlier kernels.  The producer thread waits
   // after issuing the dependency-free weight tiles of its first ring fill (below).
-  if (warp != 0 || lane != 0) pdl_wait();
+  if (warp != W_PROD || lane != 0) pdl_wait();
 
   const int num_m = (p.M + C::TILE_M - 1) / C::TILE_M;
   Jobs jobs;
   jobs.init(p, skc ? (int)blockIdx.x : (int)blockIdx.x / CG, gridDim.x / CG, num_m);
   int tile, kb0, kb1;
 
-  if (warp == 0) {
+  if (warp == W_PROD) {
     if (lane == 0) {
       // ---------------- TMA producer (both CTAs of a pair load their halves)
       int stage = 0;
@@ -792,7 +799,7 @@ __global__ void __launch_bounds__(256, 1)
         }
       }
     }
-  } else if (warp == 1) {
+  } else if (warp == W_MMA) {
     if (lane == 0 && leader) {
       // ---------------- MMA issuer (single thread of the leader CTA)
       constexpr uint32_t idesc = ptx::umma_idesc_bf16(C::TILE_M, GEMM_BN);
@@ -839,7 +846,7 @@ __global__ void __launch_bounds__(256, 1)
       }
       GM_STAMP(2);
     }
-  } else if (C::RES && warp == 3) {
+  } else if (C::RES && warp == W_RES) {
     // ---------------- residual loader (RES): x chunks of this CTA's whole tiles, RES_BUFS ahead
     if (lane == 0) {
       int rc = 0;
@@ -857,15 +864,15 @@ __global__ void __launch_bounds__(256, 1)
         }
       }
     }
-  } else if (warp >= 4 && skc) {
+  } else if (warp < 4 && skc) {
     // ---------------- cluster split-K: this CTA's partial tile -> its SMEM (the operand ring is
     // idle: every stage was consumed by the MMAs the tfull commit covers)
     if (jobs.next(tile, kb0, kb1)) {
       ptx::mbar_wait(&tfull[0], 0);
       ptx::tc_fence_after();
-      if (threadIdx.x == 128) GM_STAMP(3);
-      const int rl = (warp - 4) * 32 + lane;
-      const uint32_t tb = tmem_base + ((uint32_t)((warp - 4) * 32) << 16);
+      if (threadIdx.x == 0) GM_STAMP(3);
+      const int rl = warp * 32 + lane;
+      const uint32_t tb = tmem_base + ((uint32_t)(warp * 32) << 16);
       const uint32_t part = ptx::smem_u32(sA);
       uint32_t r[32];
 #pragma unroll 1
@@ -878,11 +885,11 @@ __global__ void __launch_bounds__(256, 1)
                        "r"(r[4 * q + 1]), "r"(r[4 * q + 2]), "r"(r[4 * q + 3])
                        : "memory");
       }
-      if (threadIdx.x == 128) GM_STAMP(4);
+      if (threadIdx.x == 0) GM_STAMP(4);
     }
-  } else if (warp >= 4) {
+  } else if (warp < 4) {
     // ---------------- epilogue warps (each CTA drains its own 128 rows)
-    const int ew = warp - 4;
+    const int ew = warp;
     int acc = 0;
     uint32_t acc_phase = 0;
     int ntile = 0;
@@ -891,7 +898,7 @@ __global__ void __launch_bounds__(256, 1)
       const int m_blk = tile % num_m, n_blk = tile / num_m;
       const int row = m_blk * C::TILE_M + rank * GEMM_BM + ew * 32 + lane;
 #ifdef GLLM_VARIANT_TRACE
-      if (threadIdx.x == 128) {
+      if (threadIdx.x == 0) {
         ptx::mbar_wait(&tfull[acc], acc_phase);
         GM_STAMP_TILE(ntile, 0);
       }
@@ -908,7 +915,7 @@ __global__ void __launch_bounds__(256, 1)
       } else {
         epilogue_tile<EPI>(p, tbase, row, n_blk, partial, &tfull[acc], acc_phase, stg + ew * C::STG_FLOATS);
       }
-      if (threadIdx.x == 128) {
+      if (threadIdx.x == 0) {
         GM_STAMP(4);
         GM_STAMP_TILE(ntile, 1);
       }
@@ -925,7 +932,7 @@ __global__ void __launch_bounds__(256, 1)
       if (acc == 0) acc_phase ^= 1;
     }
     if constexpr (C::RES) {
-      if (threadIdx.x == 128) ptx::bulk_wait<0>();  // the residual / bf16 stores are performed
+      if (threadIdx.x == 0) ptx::bulk_wait<0>();  // the residual / bf16 stores are performed
     }
   }
   if (skc) {
@@ -933,7 +940,7 @@ __global__ void __launch_bounds__(256, 1)
     // chunks over DSMEM (rank order) and runs the epilogue; the second cluster barrier keeps every
     // CTA's SMEM alive until the last remote read
     cluster_sync_all();
-    if (threadIdx.x == 128) GM_STAMP(5);
+    if (threadIdx.x == 0) GM_STAMP(5);
     {
       // sum this CTA's planes over the cluster (rank order 0..S-1: deterministic), coalesced, all 8
       // warps: thread t adds granules t, t + 256, t + 512, t + 768 of each owned plane, every
@@ -973,17 +980,17 @@ __global__ void __launch_bounds__(256, 1)
       }
       __syncthreads();  // planes complete
     }
-    if (warp >= 4) {
+    if (warp < 4) {
       Jobs ej;
       ej.init(p, blockIdx.x, gridDim.x, num_m);
       if (ej.next(tile, kb0, kb1)) {
-        const int ew = warp - 4;
+        const int ew = warp;
         const int m_blk = tile % num_m, n_blk = tile / num_m;
         const int row = m_blk * C::TILE_M + ew * 32 + lane;
         epilogue_tile<EPI>(p, tmem_base + ((uint32_t)(ew * 32) << 16), row, n_blk, false, &tfull[0], 0,
                            stg + ew * C::STG_FLOATS, ClSrc{ptx::smem_u32(sA), p.split_s, (int)cluster_rank()});
       }
-      if (threadIdx.x == 128) GM_STAMP(6);
+      if (threadIdx.x == 0) GM_STAMP(6);
     }
     ptx::tc_fence_before();
     cluster_sync_all();
@@ -994,7 +1001,7 @@ __global__ void __launch_bounds__(256, 1)
     else
       __syncthreads();
   }
-  if (warp == 2) {
+  if (warp == W_ALLOC) {
     ptx::tc_fence_after();
     tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
   }

@@ -27,6 +27,9 @@ SHAPES = {
     "C4k": [(128, 8192, k, e) for e in (0, 1) for k in (1024, 2048, 4096, 8192, 16384)],
     # the C1 O / down shapes with the plain bf16-store epilogue (isolates the residual epilogue)
     "C1s": [(2094, 4096, 4096, 0), (2094, 4096, 14336, 0)],
+    # LM head + greedy argmax (epi 3) at the sampled-row counts of C1 (~800), C2 (~250), C3 (~15), C4 (128)
+    "lm": [(800, 128256, 4096, 3), (250, 152064, 5120, 3), (300, 152064, 5120, 3), (16, 152064, 5120, 3),
+           (128, 128256, 8192, 3)],
 }
 
 
@@ -65,7 +68,9 @@ def bench_cublas(M, N, K, reps=20):
 def bench(M, N, K, epi, reps=20):
     A = torch.randn((M, K), device="cuda").to(torch.bfloat16)
     W = (torch.randn((N, K), device="cuda") * K ** -0.5).to(torch.bfloat16)
-    if epi == 1:
+    if epi == 3:
+        out = torch.empty((M,), dtype=torch.int32, device="cuda")
+    elif epi == 1:
         out = torch.zeros((M, N), device="cuda")
     elif epi == 2:
         out = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")

@@ -62,9 +62,26 @@ def test_residual_add_f32_hybrid_tail(M, N, K):
     # CTA-pair tiles whose last wave is mostly empty (C3's O / down GEMMs at T ~ 900: 80 tiles of
     # 256 x 256 on 74 pairs): whole tiles first, the tail tiles' k-blocks spread over every pair
     # and reduced into the residual (Jobs mode 2); below one wave (C2's O / down at T ~ 626: 60 tiles
-    # on 74 pairs) every tile's k-blocks are spread over all pairs
+    # on 74 pairs, whole tiles since they fill >= 75% of the pairs) every tile's k-blocks are spread
+    # over all pairs
     A, W = _bf16((M, K), 1.0, 14), _bf16((N, K), K ** -0.5, 15)
     x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(16))
+    dA, dW, x = A.cuda(), W.cuda(), x0.clone().cuda()
+    gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 1, x.data_ptr())
+    torch.cuda.synchronize()
+    ref = x0.double().numpy() + _ref(A, W)
+    err = np.abs(x.cpu().double().numpy() - ref).max()
+    assert err < 1e-3, err
+
+
+@pytest.mark.parametrize("M,N,K", [(9460, 288, 256), (9400, 544, 512), (2094, 2336, 1024)])
+def test_residual_add_f32_tma_epilogue_ragged(M, N, K):
+    # the CTA-pair residual epilogue through TMA (x chunks loaded ahead into swizzled SMEM, stored
+    # back by TMA): a last N tile of one or two 32-column chunks (N % 256 != 0) inside the whole-tile
+    # range (74 tiles = one wave for the first two shapes), ragged M (rows past M: zero-filled loads,
+    # clipped stores), and a hybrid launch mixing TMA whole tiles with stream-K tail tiles
+    A, W = _bf16((M, K), 1.0, 24), _bf16((N, K), K ** -0.5, 25)
+    x0 = torch.randn((M, N), generator=torch.Generator().manual_seed(26))
     dA, dW, x = A.cuda(), W.cuda(), x0.clone().cuda()
     gllm.op_gemm(dA.data_ptr(), dW.data_ptr(), M, N, K, 1, x.data_ptr())
     torch.cuda.synchronize()

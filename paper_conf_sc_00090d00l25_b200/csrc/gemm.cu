@@ -1112,7 +1112,12 @@ int choose_cg(int M, int N, int epi, int num_sms) {
   if (g_force_cg) return g_force_cg;
   const int nn = (N + GEMM_BN - 1) / GEMM_BN;
   const int tiles2 = ((M + 255) / 256) * nn;
-  if (M < 256 || epi == EPI_ARGMAX) return 1;
+  // LM head with 129-256 sampled rows (C2's ~250): one CTA-pair M tile covers every row, so each
+  // CTA streams half of each weight tile once (two 1-CTA M tiles each stream all of it): C2 lm_head
+  // 3.82 -> 3.51 ms over 10 steps, 0.75 -> 0.82 (profiles/r02/gemm_sched/lm_head_cg2.txt); at C1's
+  // ~800 rows the two layouts measured the same
+  if (epi == EPI_ARGMAX) return (M > GEMM_BM && M <= 2 * GEMM_BM) ? 2 : 1;
+  if (M < 256) return 1;
   // below one wave of pair tiles the residual add takes stream-K over the pairs (hybrid_dp_tiles):
   // the 1-CTA tile streams 48 KB of operands per 64-deep k-block, more than TMA's ~60-90 B/cycle per
   // SM feeds at the MMA rate (tools/micro/tma_box.cu); the pair streams 32 KB per CTA

@@ -109,7 +109,7 @@ def test_silu_mul_interleaved(M):
     assert err.max() < 1e-2, err.max()
 
 
-@pytest.mark.parametrize("M,N", [(1, 512), (9, 128256), (300, 152064)])
+@pytest.mark.parametrize("M,N", [(1, 512), (9, 128256), (200, 152064), (256, 128256), (300, 152064)])
 def test_argmax_epilogue(M, N):
     K = 1024
     A, W = _bf16((M, K), 1.0, 10), _bf16((N, K), K ** -0.5, 11)

@@ -746,6 +746,11 @@ __global__ void __launch_bounds__(256, 1)
   if (warp == W_PROD) {
     if (lane == 0) {
       // ---------------- TMA producer (both CTAs of a pair load their halves)
+      // B box coordinates: the row-major [N, K] map (k, row), or the tiled weight's [blocks*128, 64]
+      // view, where the 128-row slab of `row` at k-block kb is block slab * nk + kb
+      const int nkb = p.K / GEMM_BK;
+      auto bx = [&](int kb) -> int32_t { return p.b_tiled ? 0 : kb * GEMM_BK; };
+      auto by = [&](int row, int kb) -> int32_t { return p.b_tiled ? ((row >> 7) * nkb + kb) * 128 : row; };
       int stage = 0;
       uint32_t phase = 0;
       int pre = 0;  // stages whose B tile (and expect_tx) went out before the wait
@@ -758,12 +763,12 @@ __global__ void __launch_bounds__(256, 1)
             const int kb = kb0 + i;
             if constexpr (CG == 1) {
               ptx::mbar_arrive_expect_tx(&full[i], C::STAGE_BYTES);
-              ptx::tma_load_2d(sB + i * C::B_BYTES, &tma_b, &full[i], kb * GEMM_BK, b_row);
-              ptx::tma_load_2d(sB + i * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[i], kb * GEMM_BK,
-                               b_row + GEMM_B_BOX);
+              ptx::tma_load_2d(sB + i * C::B_BYTES, &tma_b, &full[i], bx(kb), by(b_row, kb));
+              ptx::tma_load_2d(sB + i * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[i], bx(kb),
+                               by(b_row + GEMM_B_BOX, kb));
             } else {
               if (leader) ptx::mbar_arrive_expect_tx(&full[i], 2 * C::STAGE_BYTES);
-              tma_load_2d_cg2(sB + i * C::B_BYTES, &tma_b, &full[i], kb * GEMM_BK, b_row);
+              tma_load_2d_cg2(sB + i * C::B_BYTES, &tma_b, &full[i], bx(kb), by(b_row, kb));
             }
           }
         }
@@ -784,13 +789,13 @@ __global__ void __launch_bounds__(256, 1)
           } else if constexpr (CG == 1) {
             ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
             ptx::tma_load_2d(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
-            ptx::tma_load_2d(sB + stage * C::B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, b_row);
-            ptx::tma_load_2d(sB + stage * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[stage], kb * GEMM_BK,
-                             b_row + GEMM_B_BOX);
+            ptx::tma_load_2d(sB + stage * C::B_BYTES, &tma_b, &full[stage], bx(kb), by(b_row, kb));
+            ptx::tma_load_2d(sB + stage * C::B_BYTES + GEMM_B_BOX * 128, &tma_b, &full[stage], bx(kb),
+                             by(b_row + GEMM_B_BOX, kb));
           } else {
             if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
             tma_load_2d_cg2(sA + stage * C::A_BYTES, &tma_a, &full[stage], kb * GEMM_BK, a_row);
-            tma_load_2d_cg2(sB + stage * C::B_BYTES, &tma_b, &full[stage], kb * GEMM_BK, b_row);
+            tma_load_2d_cg2(sB + stage * C::B_BYTES, &tma_b, &full[stage], bx(kb), by(b_row, kb));
           }
           if (++stage == C::STAGES) {
             stage = 0;
@@ -1226,6 +1231,11 @@ static int encode_2d(CUtensorMap* map, CUtensorMapDataType dt, int esize, const 
                         sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return set_error(GLLM_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
   return GLLM_OK;
+}
+
+int make_tmap_weight_tiled(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols) {
+  if (cols % 64) return set_error(GLLM_EINVAL, "tiled weight: cols %% 64 != 0");
+  return make_tmap_bf16(map, base, ((rows + 127) / 128) * (cols / 64) * 128, 64, GEMM_B_BOX);
 }
 
 int make_tmap_res_f32(CUtensorMap* map, const float* base, uint64_t rows, uint64_t cols) {

@@ -43,6 +43,10 @@ struct GemmArgs {
   // B (the weights) is never written by a kernel on the stream: with PDL the producer issues the
   // first ring fill's B tiles before griddepcontrol.wait (stage GEMMs only; gllm_op_gemm leaves 0)
   int b_static;
+  // B is stored in the tiled weight layout (weight_tiled_index): each 128-row x 64-column block of
+  // the K-major weight is 16 KB contiguous, and the B tensor map is the [blocks * 128, 64] view of
+  // it (make_tmap_weight_tiled), so a B box is one contiguous DRAM run (stage weights only)
+  int b_tiled;
   float* ws;  // fp32 [M, N] stream-K workspace of non-additive epilogues: zero on entry, left zero
   // 1: a schedule with a fixed reduction order (no stream-K / hybrid fp32 atomics; whole tiles or
   // cluster split-K): bitwise run-to-run reproducible results
@@ -82,6 +86,16 @@ extern int g_force_cg;
 // Encodes a 2-D bf16 K-major tensor map (rows x cols, cols contiguous) with a
 // (box_rows x 64) box and 128-byte swizzle.  Returns 0 or a GLLM_* error.
 int make_tmap_bf16(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols, uint32_t box_rows);
+
+// Tiled weight layout of the stage GEMMs' B operand: element (r, c) of a [rows, cols] K-major
+// weight (cols % 64 == 0) lives at block (r / 128, c / 64) -- 128 x 64 row-major, 16 KB -- with the
+// blocks of a 128-row slab consecutive along K.  weight_tiled_elems pads rows to a multiple of 128.
+inline int64_t weight_tiled_index(int64_t r, int64_t c, int64_t cols) {
+  return ((r >> 7) * (cols >> 6) + (c >> 6)) * 8192 + (r & 127) * 64 + (c & 63);
+}
+inline size_t weight_tiled_elems(int64_t rows, int64_t cols) { return (size_t)((rows + 127) / 128) * 128 * cols; }
+// the [blocks * 128, 64] tensor map of a tiled weight (128-row box, 128-byte swizzle)
+int make_tmap_weight_tiled(CUtensorMap* map, const void* base, uint64_t rows, uint64_t cols);
 
 // Residual-epilogue tensor maps (EPI_ADD_F32): x fp32 [rows, cols] with a 128-row x 32-column box
 // and 128-byte swizzle; bf16(x) [rows, cols] with a 128 x 32 box and 64-byte swizzle.

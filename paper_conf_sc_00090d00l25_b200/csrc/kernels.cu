@@ -30,7 +30,7 @@ __device__ __forceinline__ float o4(uint64_t seed, uint64_t tid, uint64_t i, flo
 }
 
 __global__ void init_bf16_kernel(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid,
-                                 float scale, int mode, int64_t row_offset) {
+                                 float scale, int mode, int64_t row_offset, int tiled) {
   const int64_t n = rows * cols;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = i / cols, c = i - r * cols;
@@ -39,7 +39,10 @@ __global__ void init_bf16_kernel(__nv_bfloat16* dst, int64_t rows, int64_t cols,
       pr = r + row_offset;
     else
       pr = (r / 128) * 256 + (mode == 2 ? 128 : 0) + (r % 128);
-    dst[pr * cols + c] = __float2bfloat16_rn(o4(seed, tid, (uint64_t)i, scale));
+    // tiled: the GEMM weight layout (gemm.cuh, weight_tiled_index): 128-row x 64-column blocks,
+    // each 16 KB contiguous, so a B-operand TMA box reads one contiguous run of DRAM
+    const int64_t at = tiled ? ((pr >> 7) * (cols >> 6) + (c >> 6)) * 8192 + (pr & 127) * 64 + (c & 63) : pr * cols + c;
+    dst[at] = __float2bfloat16_rn(o4(seed, tid, (uint64_t)i, scale));
   }
 }
 
@@ -245,8 +248,9 @@ bool pdl_enabled() {
 }
 
 void launch_init_bf16(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid, float scale,
-                      int mode, int64_t row_offset, cudaStream_t s) {
-  init_bf16_kernel<<<grid_for(rows * cols, 256), 256, 0, s>>>(dst, rows, cols, seed, tid, scale, mode, row_offset);
+                      int mode, int64_t row_offset, cudaStream_t s, int tiled) {
+  init_bf16_kernel<<<grid_for(rows * cols, 256), 256, 0, s>>>(dst, rows, cols, seed, tid, scale, mode, row_offset,
+                                                               tiled);
 }
 void launch_init_f32(float* dst, int64_t n, uint64_t seed, uint64_t tid, float scale, cudaStream_t s) {
   init_f32_kernel<<<grid_for(n, 256), 256, 0, s>>>(dst, n, seed, tid, scale);

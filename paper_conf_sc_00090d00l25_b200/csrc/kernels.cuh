@@ -12,7 +12,7 @@ namespace gllm {
 //   mode 1: phys = (row/128)*256 + row%128   (gate rows of the interleaved gate|up)
 //   mode 2: phys = (row/128)*256 + 128 + row%128   (up rows)
 void launch_init_bf16(__nv_bfloat16* dst, int64_t rows, int64_t cols, uint64_t seed, uint64_t tid, float scale,
-                      int mode, int64_t row_offset, cudaStream_t s);
+                      int mode, int64_t row_offset, cudaStream_t s, int tiled = 0);
 void launch_init_f32(float* dst, int64_t n, uint64_t seed, uint64_t tid, float scale, cudaStream_t s);
 void launch_fill_f32(float* dst, int64_t n, float v, cudaStream_t s);
 

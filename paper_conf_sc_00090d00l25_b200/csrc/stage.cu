@@ -236,6 +236,7 @@ int gemm(gllm_stage* st, const CUtensorMap& a, const CUtensorMap& b, gllm::GemmE
          void* out, int ldo, const float* bias, cudaStream_t s) {
   gllm::GemmArgs g{};
   g.b_static = 1;
+  g.b_tiled = 1;
   g.M = M;
   g.N = N;
   g.K = K;
@@ -380,18 +381,25 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
   int rc;
   for (int l = layer_begin; l < layer_end; ++l) {
     LayerW w;
-    if ((rc = st->dalloc(&w.wqkv, (size_t)nqkv * H)) || (rc = st->dalloc(&w.wo, (size_t)H * qd)) ||
-        (rc = st->dalloc(&w.wgu, (size_t)2 * I * H)) || (rc = st->dalloc(&w.wd, (size_t)H * I)) ||
+    // projection weights in the tiled layout (gemm.cuh): rows padded to a multiple of 128 (zero)
+    if ((rc = st->dalloc(&w.wqkv, gllm::weight_tiled_elems(nqkv, H))) ||
+        (rc = st->dalloc(&w.wo, gllm::weight_tiled_elems(H, qd))) ||
+        (rc = st->dalloc(&w.wgu, gllm::weight_tiled_elems(2 * (int64_t)I, H))) ||
+        (rc = st->dalloc(&w.wd, gllm::weight_tiled_elems(H, I))) ||
         (rc = st->dalloc(&w.kc, kv_elems)) || (rc = st->dalloc(&w.vc, kv_elems)))
       return fail(rc);
     if (cfg->qkv_bias && (rc = st->dalloc(&w.bqkv, nqkv))) return fail(rc);
-    gllm::launch_init_bf16(w.wqkv, qd, H, seed, layer_tid(l, K_WQ), s_h, 0, 0, s0);
-    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WK), s_h, 0, qd, s0);
-    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WV), s_h, 0, qd + kd, s0);
-    gllm::launch_init_bf16(w.wo, H, qd, seed, layer_tid(l, K_WO), s_q, 0, 0, s0);
-    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WG), s_h, 1, 0, s0);
-    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WU), s_h, 2, 0, s0);
-    gllm::launch_init_bf16(w.wd, H, I, seed, layer_tid(l, K_WD), s_i, 0, 0, s0);
+    CK(cudaMemsetAsync(w.wqkv, 0, gllm::weight_tiled_elems(nqkv, H) * sizeof(bf16), s0));
+    CK(cudaMemsetAsync(w.wo, 0, gllm::weight_tiled_elems(H, qd) * sizeof(bf16), s0));
+    CK(cudaMemsetAsync(w.wgu, 0, gllm::weight_tiled_elems(2 * (int64_t)I, H) * sizeof(bf16), s0));
+    CK(cudaMemsetAsync(w.wd, 0, gllm::weight_tiled_elems(H, I) * sizeof(bf16), s0));
+    gllm::launch_init_bf16(w.wqkv, qd, H, seed, layer_tid(l, K_WQ), s_h, 0, 0, s0, 1);
+    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WK), s_h, 0, qd, s0, 1);
+    gllm::launch_init_bf16(w.wqkv, kd, H, seed, layer_tid(l, K_WV), s_h, 0, qd + kd, s0, 1);
+    gllm::launch_init_bf16(w.wo, H, qd, seed, layer_tid(l, K_WO), s_q, 0, 0, s0, 1);
+    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WG), s_h, 1, 0, s0, 1);
+    gllm::launch_init_bf16(w.wgu, I, H, seed, layer_tid(l, K_WU), s_h, 2, 0, s0, 1);
+    gllm::launch_init_bf16(w.wd, H, I, seed, layer_tid(l, K_WD), s_i, 0, 0, s0, 1);
     // The two RMSNorm gains of the layer are folded into the columns of Wqkv and Wgu
     // (W' = W diag(g)); under O4 every gain is exactly 1, so W' = W bit for bit.
     if (w.bqkv) {
@@ -401,10 +409,10 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     }
     CK(cudaMemsetAsync(w.kc, 0, kv_elems * sizeof(bf16), s0));
     CK(cudaMemsetAsync(w.vc, 0, kv_elems * sizeof(bf16), s0));
-    if ((rc = gllm::make_tmap_bf16(&w.tm_qkv, w.wqkv, nqkv, H, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_o, w.wo, H, qd, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_gu, w.wgu, 2 * (size_t)I, H, gllm::GEMM_B_BOX)) ||
-        (rc = gllm::make_tmap_bf16(&w.tm_d, w.wd, H, I, gllm::GEMM_B_BOX)))
+    if ((rc = gllm::make_tmap_weight_tiled(&w.tm_qkv, w.wqkv, nqkv, H)) ||
+        (rc = gllm::make_tmap_weight_tiled(&w.tm_o, w.wo, H, qd)) ||
+        (rc = gllm::make_tmap_weight_tiled(&w.tm_gu, w.wgu, 2 * (size_t)I, H)) ||
+        (rc = gllm::make_tmap_weight_tiled(&w.tm_d, w.wd, H, I)))
       return fail(rc);
     st->layers.push_back(w);
   }
@@ -413,10 +421,12 @@ int gllm_init_stage(const gllm_model_cfg* cfg, int32_t layer_begin, int32_t laye
     gllm::launch_init_bf16(st->embed, V, H, seed, T_EMBED, s_emb, 0, 0, s0);
   }
   if (st->is_last()) {
-    if ((rc = st->dalloc(&st->lm_head, (size_t)V * H)) || (rc = st->dalloc(&st->final_norm, H))) return fail(rc);
-    gllm::launch_init_bf16(st->lm_head, V, H, seed, T_LMHEAD, s_h, 0, 0, s0);
+    if ((rc = st->dalloc(&st->lm_head, gllm::weight_tiled_elems(V, H))) || (rc = st->dalloc(&st->final_norm, H)))
+      return fail(rc);
+    CK(cudaMemsetAsync(st->lm_head, 0, gllm::weight_tiled_elems(V, H) * sizeof(bf16), s0));
+    gllm::launch_init_bf16(st->lm_head, V, H, seed, T_LMHEAD, s_h, 0, 0, s0, 1);
     gllm::launch_fill_f32(st->final_norm, H, 1.0f, s0);
-    if ((rc = gllm::make_tmap_bf16(&st->tm_lm, st->lm_head, V, H, gllm::GEMM_B_BOX))) return fail(rc);
+    if ((rc = gllm::make_tmap_weight_tiled(&st->tm_lm, st->lm_head, V, H))) return fail(rc);
     const int ntn = (V + gllm::GEMM_BN - 1) / gllm::GEMM_BN;
     if ((rc = st->dalloc(&st->ys, (size_t)st->seqs_alloc * H)) ||
         (rc = st->dalloc(&st->part_val, (size_t)st->seqs_alloc * ntn)) ||
@@ -688,6 +698,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
     const bool unfused = sk || st->deterministic;
     gllm::GemmArgs g{};
     g.b_static = 1;
+    g.b_tiled = 1;
     g.deterministic = st->deterministic;
     g.M = T;
     g.N = H;
@@ -719,6 +730,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       Prof p(st, s, C_QKV);
       gllm::GemmArgs g{};
       g.b_static = 1;
+      g.b_tiled = 1;
       g.M = T;
       g.N = nqkv;
       g.K = H;
@@ -786,6 +798,7 @@ int forward_impl(gllm_stage* st, Prepared& P, const void* hidden_in, void* hidde
       Prof p(st, s, C_GU);
       gllm::GemmArgs g{};
       g.b_static = 1;
+      g.b_tiled = 1;
       g.M = T;
       g.N = 2 * I;
       g.K = H;
@@ -979,6 +992,20 @@ int gllm_stage_read_weight(gllm_stage* st, int32_t layer, const char* name, int6
     }
     return GLLM_OK;
   };
+  // the projection weights and the LM head are stored tiled (gemm.cuh weight_tiled_index)
+  auto copy_rows_tiled = [&](const bf16* base, int64_t rows, int64_t cols, auto phys) -> int {
+    if (row0 + nrows > rows) return gllm::set_error(GLLM_EINVAL, "row range out of bounds");
+    row.resize(64);
+    for (int64_t r = 0; r < nrows; ++r) {
+      const int64_t pr = phys(row0 + r);
+      for (int64_t c0 = 0; c0 < cols; c0 += 64) {
+        CK(cudaMemcpy(row.data(), base + gllm::weight_tiled_index(pr, c0, cols), 64 * sizeof(bf16),
+                      cudaMemcpyDeviceToHost));
+        for (int64_t j = 0; j < 64; ++j) out[r * cols + c0 + j] = __bfloat162float(row[j]);
+      }
+    }
+    return GLLM_OK;
+  };
   auto ident = [](int64_t r) { return r; };
   if (n == "embed") {
     if (!st->embed) return gllm::set_error(GLLM_EINVAL, "no embedding on this stage");
@@ -986,17 +1013,17 @@ int gllm_stage_read_weight(gllm_stage* st, int32_t layer, const char* name, int6
   }
   if (n == "lm_head") {
     if (!st->lm_head) return gllm::set_error(GLLM_EINVAL, "no LM head on this stage");
-    return copy_rows(st->lm_head, c.vocab, H, ident);
+    return copy_rows_tiled(st->lm_head, c.vocab, H, ident);
   }
   if (layer < st->lb || layer >= st->le) return gllm::set_error(GLLM_EINVAL, "layer %d not on this stage", layer);
   LayerW& w = st->layers[layer - st->lb];
-  if (n == "wq") return copy_rows(w.wqkv, qd, H, ident);
-  if (n == "wk") return copy_rows(w.wqkv, kd, H, [&](int64_t r) { return qd + r; });
-  if (n == "wv") return copy_rows(w.wqkv, kd, H, [&](int64_t r) { return qd + kd + r; });
-  if (n == "wo") return copy_rows(w.wo, H, qd, ident);
-  if (n == "wg") return copy_rows(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + r % 128; });
-  if (n == "wu") return copy_rows(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + 128 + r % 128; });
-  if (n == "wd") return copy_rows(w.wd, H, I, ident);
+  if (n == "wq") return copy_rows_tiled(w.wqkv, qd, H, ident);
+  if (n == "wk") return copy_rows_tiled(w.wqkv, kd, H, [&](int64_t r) { return qd + r; });
+  if (n == "wv") return copy_rows_tiled(w.wqkv, kd, H, [&](int64_t r) { return qd + kd + r; });
+  if (n == "wo") return copy_rows_tiled(w.wo, H, qd, ident);
+  if (n == "wg") return copy_rows_tiled(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + r % 128; });
+  if (n == "wu") return copy_rows_tiled(w.wgu, I, H, [](int64_t r) { return (r / 128) * 256 + 128 + r % 128; });
+  if (n == "wd") return copy_rows_tiled(w.wd, H, I, ident);
   if (n == "bq" || n == "bk" || n == "bv") {
     if (!w.bqkv) return gllm::set_error(GLLM_EINVAL, "model has no qkv bias");
     const int64_t o = n == "bq" ? 0 : (n == "bk" ? qd : qd + kd), len = n == "bq" ? qd : kd;

@@ -6,14 +6,17 @@
 //   CG = 2 (default for >= ~1 wave of work): a CTA pair (cluster of 2 on one TPC) computes a
 //          256 x 256 tile with tcgen05.mma.cta_group::2 (M=256, N=256, K=16); each CTA loads its
 //          128 rows of A and 128 of the 256 rows of B (halving SMEM/L2 operand traffic per
-//          FLOP), 6-stage TMA ring of 32 KB stages, the leader CTA issues the MMAs and commits
-//          to both CTAs' barriers (multicast); each CTA drains its own 128 x 256 TMEM accumulator.
+//          FLOP), 6-stage TMA ring of 32 KB stages (5 for the residual add, whose whole tiles
+//          stage the residual through SMEM by TMA: res_epilogue_tile), the leader CTA issues the
+//          MMAs and commits to both CTAs' barriers (multicast); each CTA drains its own 128 x 256
+//          TMEM accumulator.
 //   CG = 1: one CTA per 128 x 256 tile (tcgen05.mma.cta_group::1, M=128), 4-stage ring of 48 KB
 //          stages; used for small T, where it also supports stream-K (equal k-block ranges per
 //          CTA, partial tiles combined with fp32 vector reductions or through a workspace).
 // Both: single-thread MMA issue, double-buffered fp32 TMEM accumulator (2 x 256 columns), 4
 // epilogue warps (tcgen05.ld) with the fused epilogues: bias, fp32 residual add, SiLU*up,
-// RoPE + paged KV append, row argmax for the greedy LM head.
+// RoPE + paged KV append, row argmax for the greedy LM head.  Stage weights (B) are stored tiled
+// (gemm.cuh weight_tiled_index: 16 KB contiguous 128 x 64 blocks), so each B box is one DRAM run.
 //   warps 0-3: epilogue (warp i reads TMEM lanes 32i..32i+31)
 //   warp 4: TMA producer   warp 5: MMA issuer   warp 6: TMEM allocator   warp 7: residual loader
 // The single-thread producer and MMA roles sit in the higher warp ids: the SMSP arbiter issues
